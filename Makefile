@@ -25,7 +25,7 @@ oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -shared -fPIC -o $@ $< -lm
 
 $(PKG)/libgum.so: $(GUM_SRCS) $(GUM_HDRS)
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(GUM_SRCS) -lgomp -lcuda 2> build/ptxas.log || (cat build/ptxas.log; false)
+	$(NVCC) $(NVFLAGS) -shared -o $@ $(GUM_SRCS) -lgomp 2> build/ptxas.log || (cat build/ptxas.log; false)
 	@grep -E "error|warning" build/ptxas.log || true
 
 $(shell mkdir -p build)

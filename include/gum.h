@@ -1,0 +1,194 @@
+/*
+ * gum.h -- C ABI of the B200-native GUM hot path (Meng et al., ICDE'23, "Efficient Multi-GPU Graph
+ * Processing with Remote Work Stealing"). PAPER.md lines are cited as P:<line>.
+ *
+ * The library runs the frontier-driven advance/filter iteration of GAS algorithms in BSP mode
+ * (§II "Graph algorithms") for BFS, SSSP, WCC and PageRank (§VI-A) over an n-way
+ * edge-cut partition of a CSR graph (§II "Graph partitions"), with the paper's two load
+ * balancers: frontier stealing (FSteal, §III) and ownership stealing (OSteal, §IV,
+ * P:152-211). Kernels are hand-written CUDA for sm_100a; see DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *   - plain C; no exceptions or C++/torch types cross the ABI;
+ *   - every call returns gum_status (0 = GUM_OK, < 0 = error); gum_last_error() gives the text;
+ *   - after any GUM_ECUDA the context is poisoned: later calls return GUM_ESTATE;
+ *   - pointers are HOST pointers unless a flag or parameter says "device";
+ *   - the caller owns every buffer it passes; the library copies what it keeps (gum_load_csr) and
+ *     owns its device memory until gum_destroy().
+ *   - vertex ids are uint32 in [0, V), V <= 2^32-2; GUM_INF (0xFFFFFFFF) marks "unreached".
+ */
+#ifndef GUM_H
+#define GUM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct gum_ctx gum_ctx; /* opaque, owned by the library */
+
+typedef enum {
+    GUM_OK = 0,
+    GUM_EINVAL = -1, /* null pointer, malformed CSR (row_ptr not monotone, row_ptr[V] != E, col >= V),
+                        SSSP without weights, buffer too small, bad config value */
+    GUM_ENOMEM = -2, /* device allocation failed (the paper assumes the graph fits) */
+    GUM_ESTATE = -3, /* wrong call order (run before partition, result before run) or poisoned ctx */
+    GUM_ERANGE = -4, /* source >= V, or an SSSP distance reaches 2^32-1 */
+    GUM_ECUDA = -5,  /* CUDA runtime error (context is poisoned) */
+    GUM_ENCCL = -6,  /* reserved (collective failure) */
+    GUM_EUNSUP = -7  /* configuration not supported by this build */
+} gum_status;
+
+/* Algorithms. Outputs (reading #1): BFS hop depth, SSSP distance (uint32 weights,
+ * uint64 arithmetic), WCC = minimum ORIGINAL vertex id of the weakly connected component,
+ * PR = x_K of the fixed-K power iteration with uniform dangling redistribution (fp64). */
+typedef enum { GUM_BFS = 0, GUM_SSSP = 1, GUM_WCC = 2, GUM_PR = 3 } gum_alg;
+
+/* Partitioners (P:315, P:382 Exp-6): SEG = contiguous id ranges with ~equal out-edges; RANDOM =
+ * keyed Feistel relabel of ids, then SEG (reading #17). metis is out of scope. */
+typedef enum { GUM_PART_SEG = 0, GUM_PART_RANDOM = 1 } gum_part;
+
+#define GUM_INF 0xFFFFFFFFu
+#define GUM_MAX_WORKERS 8
+
+/* gum_config.flags */
+#define GUM_CFG_TRACE 0x1u        /* record a per-iteration, per-worker trace (gum_trace) */
+#define GUM_CFG_HOST_LOOP 0x2u    /* drive iterations from the host instead of a CUDA-graph WHILE node */
+#define GUM_CFG_FORCE_SPARSE 0x4u /* filter always compacts the activation list (never the bitmap) */
+#define GUM_CFG_FORCE_DENSE 0x8u  /* filter always scans the bitmap */
+#define GUM_CFG_PROFILE 0x10u     /* host loop, one iteration per poll, CUDA events around every kernel
+                                     launch (read back with gum_profile); for measurement only */
+
+typedef struct {
+    /* Workers = GPUs of the paper (one worker per GPU, one fragment per worker).
+     * num_gpus fragments are created. device_ids[i] is worker i's CUDA device; NULL => every worker
+     * on device 0 ("virtual peers": workers are disjoint CTA groups of one GPU, peer pointers are
+     * local pointers -- the T3 fake backend of SURVEY.md §4). */
+    int num_gpus;
+    const int* device_ids;
+    /* FSteal (§III) and its gating thresholds t1, t2 (P:248 Example 5): stealing is enabled in an
+     * iteration only if max_i l_i >= t1 and max_i l_i - min_i l_i >= t2 (l_i = active edges). */
+    int fsteal;
+    uint64_t t1_min_max_edges;
+    uint64_t t2_min_spread_edges;
+    /* OSteal (§IV): when the global number of active vertices drops below osteal_active_threshold
+     * the active owner set shrinks to m' = clamp(ceil(active_edges / osteal_edges_per_worker), 1, m)
+     * survivors {0..m'-1} (uniform NVSwitch reduction tree, reading #13); shrink-only.
+     * osteal_edges_per_worker = 0 => m' = 1. */
+    int osteal;
+    uint64_t osteal_active_threshold;
+    uint64_t osteal_edges_per_worker;
+    /* Edges per claimable chunk of the edge-balanced steal queue (multiple of 32, <= 2048;
+     * 0 => 2048). */
+    uint32_t chunk_edges;
+    int pr_iterations;   /* 0 => 20 */
+    double pr_damping;   /* 0 => 0.85 */
+    uint32_t max_iterations; /* safety cap on BSP iterations, 0 => 2^31 */
+    uint32_t flags;      /* GUM_CFG_* */
+    /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
+    void* (*alloc)(uint64_t bytes, int device, void* user);
+    void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);
+    void* alloc_user;
+    void* const* streams; /* cudaStream_t per worker (NULL => library-owned non-blocking streams) */
+} gum_config;
+
+/* Fills *cfg with the defaults: 1 worker, fsteal=1, osteal=1, t1=t2=0, osteal threshold 0 (off until
+ * set), chunk 2048, PR 20 iterations d=0.85. */
+void gum_config_default(gum_config* cfg);
+
+typedef struct {
+    uint32_t iterations;      /* BSP iterations executed (advance steps) */
+    double ms;                /* device time of the run (CUDA events around the iteration loop) */
+    uint64_t edges_expanded;  /* edges processed by advance, summed over iterations (own + stolen) */
+    uint64_t edges_frontier;  /* sum over iterations of the frontier's out-edges (filter's count);
+                                 conservation: == edges_expanded */
+    uint64_t edges_stolen;    /* of edges_expanded, processed by a worker that does not own the chunk */
+    uint64_t chunks_stolen;
+    uint64_t chunks_total;
+    uint64_t remote_updates;  /* atomic updates whose target fragment is not the processing worker's */
+    uint64_t activations;     /* vertices appended to next frontiers */
+    uint64_t vertices_frontier; /* sum over iterations of |f_k| (queue entries expanded) */
+    uint32_t final_owners;    /* active owners at the end (OSteal) */
+    uint32_t osteal_iteration;/* iteration of the last owner-set shrink (0 = never) */
+    double pr_last_residual;  /* PR: sum_v |x_K - x_{K-1}| */
+} gum_run_stats;
+
+/* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:
+ * worker w's busy window is [t_start[w], t_end[w]] (min start / max end over its CTAs). */
+typedef struct {
+    uint64_t t_start[GUM_MAX_WORKERS];
+    uint64_t t_end[GUM_MAX_WORKERS];
+    uint64_t edges_own[GUM_MAX_WORKERS];    /* edges of chunks the worker owns, processed by it */
+    uint64_t edges_stolen[GUM_MAX_WORKERS]; /* edges the worker processed from others' queues */
+    uint64_t frontier_vertices;
+    uint64_t frontier_edges;
+    uint32_t owners;      /* active owners m in this iteration */
+    uint32_t steal_ok;    /* FSteal gate open in this iteration */
+} gum_iter_trace;
+
+/* ---- lifecycle ------------------------------------------------------------------------------ */
+gum_status gum_create(const gum_config* cfg, gum_ctx** out);
+void gum_destroy(gum_ctx* ctx);
+const char* gum_last_error(const gum_ctx* ctx);
+
+/* ---- a1 graph setup ---------------------------------------------------------------------------
+ * Host helper: stable counting sort of a raw edge multiset (src[i] -> dst[i], w[i]) into CSR
+ * (self-loops and parallel edges kept). row_ptr: uint64[V+1]; col, wout:
+ * uint32[E] (wout/w may be NULL). Caller-allocated outputs. OpenMP-parallel. */
+gum_status gum_build_csr(uint32_t num_vertices, uint64_t num_edges, const uint32_t* src, const uint32_t* dst,
+                         const uint32_t* w, uint64_t* row_ptr, uint32_t* col, uint32_t* wout);
+
+/* Loads graph G = (V, E). row_ptr: uint64[V+1], monotone, row_ptr[0] = 0, row_ptr[V] = E;
+ * col: uint32[E] destinations < V; weights: uint32[E] or NULL (required for SSSP).
+ * flags: GUM_LOAD_DEVICE => the three pointers are device pointers on worker 0's device.
+ * Copies everything; validates on the device (EINVAL on malformed input). Invalidates any previous
+ * partition. */
+#define GUM_LOAD_DEVICE 0x1u
+gum_status gum_load_csr(gum_ctx* ctx, uint32_t num_vertices, uint64_t num_edges, const uint64_t* row_ptr,
+                        const uint32_t* col_idx, const uint32_t* weights, uint32_t flags);
+
+/* ---- a2 partition -----------------------------------------------------------------------------
+ * n-way edge-cut: fragment g owns the relabelled id range [b_g, b_{g+1}) with ~E/n
+ * out-edges and keeps global destination ids; per-fragment device CSR, state, bitmap, queues and
+ * peer-visible control blocks are allocated on worker g's device. seed keys the RANDOM relabel. */
+gum_status gum_partition(gum_ctx* ctx, gum_part kind, uint64_t seed);
+/* Fragment bounds in relabelled id space: bounds[0..num_gpus]. */
+gum_status gum_partition_bounds(const gum_ctx* ctx, uint32_t* bounds, int n);
+
+/* Optional: build per-algorithm auxiliary structures outside the timed run (WCC: symmetric
+ * out+in fragments; PR: nothing extra). gum_run calls it implicitly. */
+gum_status gum_prepare(gum_ctx* ctx, gum_alg alg);
+
+/* ---- a3..a11 the run ---------------------------------------------------------------------------
+ * Runs algorithm alg from `source` (BFS/SSSP; ignored by WCC/PR) to convergence (BFS/SSSP/WCC:
+ * global frontier empty; PR: pr_iterations iterations). Stream-ordered on the workers' streams;
+ * returns after completion. stats may be NULL. ERANGE if source >= V or an SSSP distance
+ * overflows; EINVAL if SSSP and no weights were loaded. */
+gum_status gum_run(gum_ctx* ctx, gum_alg alg, uint32_t source, gum_run_stats* stats);
+
+/* ---- a12 result --------------------------------------------------------------------------------
+ * Writes the last run's output in ORIGINAL vertex ids into out (host): uint32[V] for BFS/SSSP/WCC,
+ * double[V] for PR. out_bytes must be >= V * element size (EINVAL otherwise). */
+gum_status gum_result(gum_ctx* ctx, void* out, uint64_t out_bytes);
+/* Same, into a device buffer on worker 0's device. */
+gum_status gum_result_device(gum_ctx* ctx, void* out_device, uint64_t out_bytes);
+
+/* Copies up to max_records per-iteration trace records of the last run (GUM_CFG_TRACE). */
+gum_status gum_trace(const gum_ctx* ctx, gum_iter_trace* out, uint32_t max_records, uint32_t* n_records);
+
+/* Per-kernel device time of the last run, from CUDA events recorded on the launching stream around
+ * every launch (only with GUM_CFG_PROFILE; single-device). */
+typedef struct {
+    double filter_ms, control_ms, advance_ms, finalize_ms, init_ms;
+    uint32_t filter_launches, control_launches, advance_launches, finalize_launches, init_launches;
+} gum_kernel_times;
+gum_status gum_profile(const gum_ctx* ctx, gum_kernel_times* out);
+
+/* Library version (major*10000 + minor*100 + patch). */
+int gum_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GUM_H */

@@ -1,0 +1,109 @@
+// Internal layout shared by the host runtime (runtime.cu) and the sm_100a kernels (kernels.cu).
+// Everything a kernel touches for fragment f lives in fragment f's device memory and is reachable
+// from every worker through the pointers in DevCtx (local pointers for virtual peers, P2P/IPC
+// pointers for real peers): the one-sided "remote memory access" design of P:398.
+#pragma once
+#include <stdint.h>
+
+#include "gum.h"
+
+namespace gum {
+
+constexpr int kMaxW = GUM_MAX_WORKERS;
+constexpr int kThreads = 256;          // CTA size of advance / filter
+constexpr int kTileMax = 2048;         // max edges per claimable chunk (smem sized for it)
+constexpr int kEdgesPerThread = kTileMax / kThreads;
+constexpr int kFilterWordsPerThread = 4;                          // dense filter: bitmap words per thread
+constexpr int kFilterWordsPerPart = kThreads * kFilterWordsPerThread;  // 1024 words = 32768 vertices
+constexpr int kFilterAppPerThread = 8;                            // sparse filter: list entries per thread
+constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
+constexpr int kTraceMax = 1 << 16;
+
+// Per-fragment control block (fragment memory, peer-visible). Counters that thieves touch
+// (claim) and that the filter publishes (qlen, qedges, ntiles) live here.
+struct alignas(128) FragCtl {
+    unsigned long long claim;    // chunk claim counter of the current advance (steal queue head)
+    unsigned long long ntiles;   // chunks in the current frontier queue
+    unsigned long long qlen;     // |f_g| (vertices with out-degree > 0)
+    unsigned long long qedges;   // l_g: out-edges of the current frontier (P:87 workload L_k)
+    unsigned int app_cnt;        // activations appended during advance (next frontier, sparse list)
+    unsigned int err;            // sticky error flag (1 = SSSP distance overflow)
+    unsigned int dense;          // last filter used the bitmap (1) or the list (0)
+    unsigned int pad0;
+    double pr_dang[2];           // PR: partial dangling mass of this fragment's new x (by iteration parity)
+    double pr_resid[2];          // PR: partial residual (by iteration parity)
+    // run-total counters
+    unsigned long long edges_done;     // edges of this fragment's chunks processed (own + stolen)
+    unsigned long long edges_stolen;   // ... of which by a non-owner
+    unsigned long long chunks_stolen;
+    unsigned long long chunks_done;
+    unsigned long long frontier_edges; // sum over iterations of qedges
+    unsigned long long remote_updates; // updates issued by this fragment's owner to other fragments
+    unsigned long long activations;
+    unsigned long long frontier_vertices; // sum over iterations of qlen
+};
+
+// Per launch unit (device) run-control replica: decisions are computed redundantly and
+// identically by every unit from the same gathered counts (no policy broadcast).
+struct alignas(128) RunCtl {
+    unsigned int iter;        // BSP iteration k
+    unsigned int done;
+    unsigned int m;           // active owners (OSteal): workers {0..m-1}
+    unsigned int steal_ok;    // FSteal gate for the current advance
+    unsigned int owner[kMaxW];// fragment -> worker (P_OSteal vector O)
+    unsigned int err;
+    unsigned int osteal_iter;
+    unsigned long long epoch; // filter look-back epoch (monotone across runs)
+    double pr_D;              // PR: global dangling mass D_k of the current x
+    double pr_resid;
+    unsigned int ticket[kMaxW];   // filter partition tickets per fragment (reset by control)
+    unsigned int filt_done[kMaxW];
+};
+
+// Decoupled look-back slot of the filter scan (one per partition per fragment, unit-local).
+struct alignas(64) LBSlot {
+    unsigned long long flag;      // epoch*4 + {1 = aggregate ready, 2 = inclusive ready}
+    unsigned long long agg_cnt, agg_deg;
+    unsigned long long inc_cnt, inc_deg;
+};
+
+struct FragPtrs {
+    const unsigned long long* row_ptr;  // [V_f + 1], rebased to 0
+    const unsigned int* col;            // [E_f] global (relabelled) destination ids
+    const unsigned int* w;              // [E_f] or null
+    unsigned int* state;                // [V_f] depth / dist / label
+    double* x;                          // PR [V_f]
+    double* acc;                        // PR [V_f]
+    const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
+    unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
+    unsigned int* app;                  // [V_f] activation list (sparse next frontier)
+    unsigned int* q_v;                  // [V_f] frontier queue (local ids, out-degree > 0)
+    unsigned long long* q_off;          // [V_f + 1] exclusive prefix of out-degrees over the queue
+    long long* q_base;                  // [V_f] col index of edge j of queue entry i = q_off[i] + j + q_base[i]
+    unsigned int* tile;                 // [ntiles_max + 1] chunk table: first queue entry of chunk t
+    FragCtl* ctl;
+    unsigned int V;                     // |V_f|
+    unsigned int base;                  // global id of local vertex 0
+    unsigned long long E;
+};
+
+struct DevCtx {
+    FragPtrs f[kMaxW];
+    RunCtl* rctl[kMaxW];        // per worker: the replica of the unit that worker belongs to
+    LBSlot* lb[kMaxW];          // per fragment: look-back slots in the filtering unit's memory
+    unsigned int lb_parts;      // slots per fragment
+    gum_iter_trace* trace[kMaxW];  // per worker's unit (nullable)
+    unsigned int bounds[kMaxW + 1];
+    int P;                      // fragments == workers
+    unsigned int chunk;         // edges per chunk
+    unsigned int num_vertices;  // |V|
+    int fsteal, osteal;
+    unsigned long long t1, t2, os_thresh, os_epw;
+    unsigned int max_iter;
+    int pr_iters;
+    double pr_d;
+    unsigned int force_mode;    // 0 auto, 1 sparse, 2 dense
+    unsigned int dense_div;     // dense filter iff app_cnt > V_f / dense_div
+};
+
+}  // namespace gum

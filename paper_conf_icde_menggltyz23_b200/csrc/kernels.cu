@@ -1,0 +1,865 @@
+// sm_100a kernels of the GUM hot path. PAPER.md lines as P:<line>.
+//
+// One BSP iteration (GAS on BSP; Example 4 P:234-242) is, per launch unit (a GPU):
+//   k_filter   a4  "Step 1: generate frontiers": the owner compacts its activation bitmap
+//                  (dense) or activation list (sparse) into a degree-filtered queue, with the
+//                  exclusive prefix of out-degrees and the edge-balanced chunk table
+//                  (Alg. 1 l.9-18 PrefixSum + SortedSearch) in ONE decoupled-look-back pass.
+//   k_control  a5/a6/a7-gate  workload sync + convergence, OSteal owner-set shrink (§IV,
+//                  P:158-160, reduction tree P:162), FSteal gating t1/t2.
+//   k_advance  a7/a8/a9  persistent CTAs claim edge-balanced chunks of their own fragments' queues
+//                  (atomic claim counter = steal-queue head); when drained they steal chunks of the
+//                  most-loaded peer queue and read the victim's CSR in place. Per edge:
+//                  GAS Apply as atomicMin / red.add into the OWNER fragment's state (local or peer),
+//                  activation = atomicOr on the owner's bitmap + warp-aggregated append.
+//   k_pr_finalize a11  x' = (1-d)/V + d(acc + D/V), dangling mass and residual (PR, fp64).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "gum_internal.h"
+#include "kernels.h"
+
+namespace gum {
+
+// ------------------------------------------------------------------------------------------ utils
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+template <typename T>
+__device__ __forceinline__ T vload(const T* p) {
+    return *(const volatile T*)p;
+}
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// owner fragment of a global (relabelled) vertex id: <= 7 compares ("global to local id").
+__device__ __forceinline__ int frag_of(const DevCtx& c, unsigned v) {
+    int f = 0;
+#pragma unroll
+    for (int i = 1; i < kMaxW; i++) f += (i < c.P && v >= c.bounds[i]) ? 1 : 0;
+    return f;
+}
+
+// ------------------------------------------------------------------------------------------ init
+template <int ALG>
+__global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
+    const int f = f0 + blockIdx.y;
+    const FragPtrs& F = c.f[f];
+    const unsigned nwords = (F.V + 31) / 32;
+    const unsigned n = F.V > nwords ? F.V : nwords;
+    for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        if (i < F.V) {
+            if (ALG == ALG_BFS || ALG == ALG_SSSP) F.state[i] = GUM_INF;
+            if (ALG == ALG_WCC) F.state[i] = F.orig ? F.orig[i] : F.base + i;
+            if (ALG == ALG_WCC || ALG == ALG_PR) F.app[i] = i;  // all-active frontier as a list too
+            if (ALG == ALG_PR) {
+                F.x[i] = 1.0 / (double)c.num_vertices;
+                F.acc[i] = 0.0;
+            }
+        }
+        if (i < nwords) {
+            unsigned wv = 0;
+            if (ALG == ALG_WCC || ALG == ALG_PR) {
+                unsigned rem = F.V - i * 32;
+                wv = rem >= 32 ? 0xFFFFFFFFu : ((1u << rem) - 1u);
+            }
+            F.bm[i] = wv;
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        FragCtl* ct = F.ctl;
+        ct->claim = 0;
+        ct->ntiles = 0;
+        ct->qlen = 0;
+        ct->qedges = 0;
+        ct->app_cnt = (ALG == ALG_WCC || ALG == ALG_PR) ? F.V : 0;
+        ct->err = 0;
+        ct->dense = 0;
+        ct->pr_dang[0] = ct->pr_dang[1] = 0.0;
+        ct->pr_resid[0] = ct->pr_resid[1] = 0.0;
+        ct->edges_done = ct->edges_stolen = ct->chunks_stolen = ct->chunks_done = 0;
+        ct->frontier_edges = ct->remote_updates = ct->activations = 0;
+        ct->frontier_vertices = 0;
+    }
+}
+
+// source activation (BFS/SSSP): runs after k_init on the source's owner unit.
+__global__ void k_init_source(const __grid_constant__ DevCtx c, int f, unsigned ls) {
+    const FragPtrs& F = c.f[f];
+    F.state[ls] = 0;
+    F.bm[ls >> 5] |= 1u << (ls & 31);
+    F.app[0] = ls;
+    F.ctl->app_cnt = 1;
+}
+
+__global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, gum_iter_trace* trace) {
+    RunCtl* rc = c.rctl[w0];
+    rc->iter = 0;
+    rc->done = 0;
+    rc->m = c.P;
+    rc->steal_ok = 0;
+    for (int i = 0; i < kMaxW; i++) {
+        rc->owner[i] = i;
+        rc->ticket[i] = 0;
+        rc->filt_done[i] = 0;
+    }
+    rc->err = 0;
+    rc->osteal_iter = 0;
+    rc->epoch = rc->epoch + 1;
+    rc->pr_D = D0;
+    rc->pr_resid = 0.0;
+}
+
+// ------------------------------------------------------------------------------------------ filter
+// Block-wide exclusive scan of (count, degree-sum) pairs; returns the block totals.
+struct Pair {
+    unsigned long long cnt, deg;
+};
+__device__ __forceinline__ Pair block_excl_scan(Pair v, Pair* s_warp, Pair& total) {
+    const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
+    Pair inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned long long c = __shfl_up_sync(0xffffffffu, inc.cnt, o);
+        unsigned long long d = __shfl_up_sync(0xffffffffu, inc.deg, o);
+        if (lane >= (unsigned)o) {
+            inc.cnt += c;
+            inc.deg += d;
+        }
+    }
+    if (lane == 31) s_warp[wid] = inc;
+    __syncthreads();
+    Pair wexcl{0, 0};
+    total = Pair{0, 0};
+    for (int i = 0; i < kThreads / 32; i++) {
+        if ((unsigned)i < wid) {
+            wexcl.cnt += s_warp[i].cnt;
+            wexcl.deg += s_warp[i].deg;
+        }
+        total.cnt += s_warp[i].cnt;
+        total.deg += s_warp[i].deg;
+    }
+    __syncthreads();
+    return Pair{wexcl.cnt + inc.cnt - v.cnt, wexcl.deg + inc.deg - v.deg};
+}
+
+__device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, unsigned v, unsigned long long rp,
+                                            unsigned long long deg, unsigned long long pos, unsigned long long off) {
+    F.q_v[pos] = v;
+    F.q_off[pos] = off;
+    F.q_base[pos] = (long long)rp - (long long)off;
+    // chunk table: every chunk whose first edge lies in [off, off+deg) starts at queue entry pos
+    unsigned long long t = (off + chunk - 1) / chunk;
+    for (; t * chunk < off + deg; t++) F.tile[t] = (unsigned)pos;
+}
+
+__global__ void __launch_bounds__(kThreads) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+    RunCtl* rc = c.rctl[w0];
+    if (vload(&rc->done)) return;
+    const int f = blockIdx.y;
+    const unsigned o = rc->owner[f];
+    if ((int)o < w0 || (int)o >= w0 + nw) return;
+    const FragPtrs& F = c.f[f];
+    FragCtl* ct = F.ctl;
+    const unsigned app_cnt = vload(&ct->app_cnt);
+    const bool dense = c.force_mode == 2 || (c.force_mode == 0 && (unsigned long long)app_cnt * c.dense_div > F.V);
+    const unsigned nwords = (F.V + 31) / 32;
+    const unsigned long long n_items = dense ? nwords : app_cnt;
+    const unsigned per = dense ? kFilterWordsPerPart : kFilterAppPerPart;
+    unsigned long long n_parts = (n_items + per - 1) / per;
+    if (n_parts == 0) n_parts = 1;
+    const unsigned long long epoch = rc->epoch;
+    const unsigned chunk = c.chunk;
+    LBSlot* slots = c.lb[f];
+
+    __shared__ unsigned s_part;
+    __shared__ Pair s_warp[kThreads / 32];
+    __shared__ Pair s_excl;
+
+    for (;;) {
+        if (threadIdx.x == 0) s_part = atomicAdd(&rc->ticket[f], 1u);
+        __syncthreads();
+        const unsigned p = s_part;
+        __syncthreads();
+        if (p >= n_parts) break;
+
+        // ---- phase 1: gather items, count vertices with out-degree > 0 and their degrees
+        unsigned items[8];
+        int nit = 0;
+        Pair mine{0, 0};
+        if (dense) {
+            const unsigned wbase = p * kFilterWordsPerPart + threadIdx.x * kFilterWordsPerThread;
+            if (wbase + kFilterWordsPerThread <= nwords) {
+                uint4 q = *reinterpret_cast<const uint4*>(F.bm + wbase);
+                items[0] = q.x; items[1] = q.y; items[2] = q.z; items[3] = q.w;
+                *reinterpret_cast<uint4*>(F.bm + wbase) = make_uint4(0, 0, 0, 0);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 4; j++) {
+                    items[j] = (wbase + j < nwords) ? F.bm[wbase + j] : 0u;
+                    if (wbase + j < nwords) F.bm[wbase + j] = 0u;
+                }
+            }
+            nit = 4;
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                unsigned wv = items[j];
+                while (wv) {
+                    unsigned b = __ffs(wv) - 1;
+                    wv &= wv - 1;
+                    unsigned v = (wbase + j) * 32 + b;
+                    unsigned long long d = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
+                    if (d) {
+                        mine.cnt++;
+                        mine.deg += d;
+                    }
+                }
+            }
+        } else {
+            const unsigned long long ibase = (unsigned long long)p * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                if (ibase + j < app_cnt) {
+                    unsigned v = F.app[ibase + j];
+                    items[j] = v;
+                    nit = j + 1;
+                    F.bm[v >> 5] = 0u;  // every set bit belongs to a listed vertex: clearing whole words is exact
+                    unsigned long long d = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
+                    if (d) {
+                        mine.cnt++;
+                        mine.deg += d;
+                    }
+                }
+            }
+        }
+        Pair agg;
+        Pair texcl = block_excl_scan(mine, s_warp, agg);
+
+        // ---- decoupled look-back (single thread) over partitions of this fragment
+        if (threadIdx.x == 0) {
+            LBSlot* S = slots + p;
+            Pair excl{0, 0};
+            if (p == 0) {
+                S->inc_cnt = agg.cnt;
+                S->inc_deg = agg.deg;
+                st_release_u64(&S->flag, epoch * 4 + 2);
+            } else {
+                S->agg_cnt = agg.cnt;
+                S->agg_deg = agg.deg;
+                st_release_u64(&S->flag, epoch * 4 + 1);
+                long long j = (long long)p - 1;
+                while (j >= 0) {
+                    unsigned long long fl = ld_acquire_u64(&slots[j].flag);
+                    if (fl < epoch * 4 + 1) continue;  // predecessor not published yet
+                    if (fl == epoch * 4 + 2) {
+                        excl.cnt += __ldcg(&slots[j].inc_cnt);
+                        excl.deg += __ldcg(&slots[j].inc_deg);
+                        break;
+                    }
+                    excl.cnt += __ldcg(&slots[j].agg_cnt);
+                    excl.deg += __ldcg(&slots[j].agg_deg);
+                    j--;
+                }
+                S->inc_cnt = excl.cnt + agg.cnt;
+                S->inc_deg = excl.deg + agg.deg;
+                st_release_u64(&S->flag, epoch * 4 + 2);
+            }
+            s_excl = excl;
+            if (p == n_parts - 1) {
+                const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
+                F.q_off[tc] = td;
+                ct->qlen = tc;
+                ct->qedges = td;
+                ct->ntiles = (td + chunk - 1) / chunk;
+                ct->claim = 0;
+                ct->app_cnt = 0;
+                ct->dense = dense ? 1u : 0u;
+                ct->frontier_edges += td;
+                ct->frontier_vertices += tc;
+            }
+        }
+        __syncthreads();
+        unsigned long long pos = s_excl.cnt + texcl.cnt;
+        unsigned long long off = s_excl.deg + texcl.deg;
+
+        // ---- phase 2: write queue entries, degree prefix and chunk table
+        if (dense) {
+            const unsigned wbase = p * kFilterWordsPerPart + threadIdx.x * kFilterWordsPerThread;
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                unsigned wv = items[j];
+                while (wv) {
+                    unsigned b = __ffs(wv) - 1;
+                    wv &= wv - 1;
+                    unsigned v = (wbase + j) * 32 + b;
+                    unsigned long long rp = __ldg(F.row_ptr + v);
+                    unsigned long long d = __ldg(F.row_ptr + v + 1) - rp;
+                    if (d) {
+                        emit_vertex(F, chunk, v, rp, d, pos, off);
+                        pos++;
+                        off += d;
+                    }
+                }
+            }
+        } else {
+            for (int j = 0; j < nit; j++) {
+                unsigned v = items[j];
+                unsigned long long rp = __ldg(F.row_ptr + v);
+                unsigned long long d = __ldg(F.row_ptr + v + 1) - rp;
+                if (d) {
+                    emit_vertex(F, chunk, v, rp, d, pos, off);
+                    pos++;
+                    off += d;
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------------------------------ control
+template <int ALG>
+__global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cudaGraphConditionalHandle h, int use_h) {
+    if (threadIdx.x != 0) return;
+    RunCtl* rc = c.rctl[w0];
+    if (rc->done) {
+        if (use_h) cudaGraphSetConditional(h, 0);
+        return;
+    }
+    const unsigned k = rc->iter;
+    unsigned long long active = 0, total_edges = 0, l[kMaxW];
+    unsigned err = 0;
+    for (int i = 0; i < kMaxW; i++) l[i] = 0;
+    double D = 0.0, R = 0.0;
+    for (int f = 0; f < c.P; f++) {
+        FragCtl* ct = c.f[f].ctl;
+        unsigned long long q = vload(&ct->qlen), e = vload(&ct->qedges);
+        err |= vload(&ct->err);
+        active += q;
+        total_edges += e;
+        l[rc->owner[f]] += e;
+        if (ALG == ALG_PR && k > 0) {
+            D += vload(&ct->pr_dang[(k - 1) & 1]);
+            R += vload(&ct->pr_resid[(k - 1) & 1]);
+        }
+    }
+    bool done;
+    if (ALG == ALG_PR) {
+        if (k > 0) {
+            rc->pr_D = D;
+            rc->pr_resid = R;
+        }
+        // the finalize of iteration k accumulates into parity slot k&1: clear it for owned fragments
+        // (other units only ever read the opposite slot in this phase)
+        for (int f = 0; f < c.P; f++) {
+            if ((int)rc->owner[f] >= w0 && (int)rc->owner[f] < w0 + nw) {
+                c.f[f].ctl->pr_dang[k & 1] = 0.0;
+                c.f[f].ctl->pr_resid[k & 1] = 0.0;
+            }
+        }
+        done = (int)k >= c.pr_iters;
+    } else {
+        done = err != 0 || active == 0 || k >= c.max_iter;
+    }
+    unsigned m = rc->m;
+    if (!done) {
+        // a6 OSteal: shrink the active owner set in the long tail (threshold trigger)
+        if (c.osteal && m > 1 && active < c.os_thresh) {
+            unsigned mp = 1;
+            if (c.os_epw) {
+                unsigned long long want = (total_edges + c.os_epw - 1) / c.os_epw;
+                mp = want < 1 ? 1 : (want > m ? m : (unsigned)want);
+            }
+            if (mp < m) {
+                for (int f = 0; f < c.P; f++)
+                    if (rc->owner[f] >= mp) rc->owner[f] = rc->owner[f] % mp;
+                m = mp;
+                rc->m = mp;
+                rc->osteal_iter = k;
+                for (int i = 0; i < kMaxW; i++) l[i] = 0;
+                for (int f = 0; f < c.P; f++) l[rc->owner[f]] += vload(&c.f[f].ctl->qedges);
+            }
+        }
+        // a7 FSteal gate (P:248 Example 5): max l >= t1 and max l - min l >= t2 over active owners
+        unsigned long long mx = 0, mn = ~0ull;
+        for (unsigned i = 0; i < m; i++) {
+            mx = l[i] > mx ? l[i] : mx;
+            mn = l[i] < mn ? l[i] : mn;
+        }
+        rc->steal_ok = (c.fsteal && m > 1 && mx >= c.t1 && mx - mn >= c.t2) ? 1u : 0u;
+        gum_iter_trace* tr = c.trace[w0];
+        if (tr && k < (unsigned)kTraceMax) {
+            gum_iter_trace* r = tr + k;
+            for (int i = 0; i < kMaxW; i++) {
+                r->t_start[i] = ~0ull;
+                r->t_end[i] = 0;
+                r->edges_own[i] = 0;
+                r->edges_stolen[i] = 0;
+            }
+            r->frontier_vertices = active;
+            r->frontier_edges = total_edges;
+            r->owners = m;
+            r->steal_ok = rc->steal_ok;
+        }
+        rc->iter = k + 1;
+    }
+    for (int f = 0; f < kMaxW; f++) rc->ticket[f] = 0;
+    rc->epoch = rc->epoch + 1;
+    if (done) {
+        rc->done = 1;
+        rc->err = err;
+    }
+    __threadfence();
+    if (use_h) cudaGraphSetConditional(h, done ? 0u : 1u);
+}
+
+// ------------------------------------------------------------------------------------------ advance
+template <int ALG>
+struct ValT {
+    typedef unsigned T;
+};
+template <>
+struct ValT<ALG_PR> {
+    typedef double T;
+};
+
+template <int ALG, bool MULTI>
+__global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
+    typedef typename ValT<ALG>::T VT;
+    __shared__ long long s_base[kTileMax + 1];
+    __shared__ VT s_val[kTileMax + 1];
+    __shared__ unsigned short s_head[kTileMax];
+    __shared__ unsigned s_wmax[kThreads / 32];
+    __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
+    __shared__ unsigned s_owner[kMaxW];
+    __shared__ int s_f;
+    __shared__ unsigned long long s_t;
+    __shared__ int s_stolen;
+
+    RunCtl* rc = c.rctl[w0];
+    if (vload(&rc->done)) return;
+    const int w = w0 + (int)(blockIdx.x % (unsigned)nw);
+    const unsigned m = rc->m;
+    if ((unsigned)w >= m) return;  // evicted by OSteal: this worker's GPU only serves as memory
+    const unsigned k = rc->iter - 1;
+    const bool steal = rc->steal_ok != 0;
+    const unsigned long long t0 = globaltimer();
+    if (threadIdx.x < (unsigned)c.P) {
+        FragCtl* ct = c.f[threadIdx.x].ctl;
+        s_ntiles[threadIdx.x] = vload(&ct->ntiles);
+        s_qlen[threadIdx.x] = vload(&ct->qlen);
+        s_qedges[threadIdx.x] = vload(&ct->qedges);
+        s_owner[threadIdx.x] = rc->owner[threadIdx.x];
+    }
+    __syncthreads();
+    const unsigned CH = c.chunk;
+    int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
+    unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0;
+
+    for (;;) {
+        if (threadIdx.x == 0) {
+            int f = -1;
+            unsigned long long t = 0;
+            int stolen = 0;
+            while (own_cursor < c.P) {
+                int g = (w + own_cursor) % c.P;
+                if (s_owner[g] == (unsigned)w) {
+                    unsigned long long tt = atomicAdd(&c.f[g].ctl->claim, 1ull);
+                    if (tt < s_ntiles[g]) {
+                        f = g;
+                        t = tt;
+                        break;
+                    }
+                }
+                own_cursor++;
+            }
+            if (f < 0 && steal) {
+                // FSteal: claim a chunk of the active owner queue with the most remaining chunks
+                for (;;) {
+                    int best = -1;
+                    unsigned long long best_rem = 0;
+                    for (int g = 0; g < c.P; g++) {
+                        if (s_owner[g] == (unsigned)w) continue;
+                        unsigned long long cl = vload(&c.f[g].ctl->claim);
+                        unsigned long long rem = s_ntiles[g] > cl ? s_ntiles[g] - cl : 0;
+                        if (rem > best_rem) {
+                            best_rem = rem;
+                            best = g;
+                        }
+                    }
+                    if (best < 0) break;
+                    unsigned long long tt = atomicAdd(&c.f[best].ctl->claim, 1ull);
+                    if (tt < s_ntiles[best]) {
+                        f = best;
+                        t = tt;
+                        stolen = 1;
+                        break;
+                    }
+                }
+            }
+            s_f = f;
+            s_t = t;
+            s_stolen = stolen;
+        }
+        __syncthreads();
+        const int f = s_f;
+        if (f < 0) break;
+        const unsigned long long t = s_t;
+        const bool stolen = s_stolen != 0;
+        const FragPtrs& F = c.f[f];
+        const unsigned long long tb = t * CH;
+        const unsigned long long qe = s_qedges[f];
+        const unsigned tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
+        const unsigned i0 = __ldg(F.tile + t);
+        const unsigned i1 = (t + 1 < s_ntiles[f]) ? __ldg(F.tile + t + 1) : (unsigned)(s_qlen[f] - 1);
+        const unsigned nv = i1 - i0 + 1;
+
+        // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
+        for (unsigned e = threadIdx.x; e < tlen; e += kThreads) s_head[e] = 0;
+        __syncthreads();
+        for (unsigned kk = threadIdx.x; kk < nv; kk += kThreads) {
+            const unsigned i = i0 + kk;
+            const unsigned u = __ldg(F.q_v + i);
+            const unsigned long long off = __ldg(F.q_off + i);
+            s_base[kk] = __ldg(F.q_base + i);
+            if (ALG == ALG_PR) {
+                const unsigned long long deg = __ldg(F.q_off + i + 1) - off;
+                s_val[kk] = (VT)(__ldcg(F.x + u) / (double)deg);
+            } else {
+                s_val[kk] = (VT)__ldcg(F.state + u);
+            }
+            const long long rel = (long long)off - (long long)tb;
+            if (rel > 0 && rel < (long long)tlen) s_head[rel] = (unsigned short)kk;
+        }
+        __syncthreads();
+        // blocked inclusive max-scan of s_head: s_head[e] = index of the vertex owning edge e
+        {
+            const unsigned b = threadIdx.x * kEdgesPerThread;
+            unsigned hv[kEdgesPerThread];
+            unsigned run = 0;
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                hv[j] = (b + j < tlen) ? s_head[b + j] : 0u;
+                run = hv[j] > run ? hv[j] : run;
+                hv[j] = run;
+            }
+            unsigned inc = run;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                unsigned x = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane_id() >= (unsigned)o) inc = x > inc ? x : inc;
+            }
+            unsigned excl = __shfl_up_sync(0xffffffffu, inc, 1);
+            if (lane_id() == 0) excl = 0;
+            if (lane_id() == 31) s_wmax[threadIdx.x >> 5] = inc;
+            __syncthreads();
+            for (unsigned i = 0; i < (threadIdx.x >> 5); i++) excl = s_wmax[i] > excl ? s_wmax[i] : excl;
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++)
+                if (b + j < tlen) s_head[b + j] = (unsigned short)(hv[j] > excl ? hv[j] : excl);
+        }
+        __syncthreads();
+
+        // ---- expand: striped edges, coalesced col/w loads; apply to the owner fragment
+        unsigned vv[kEdgesPerThread];
+        VT cv[kEdgesPerThread];
+#pragma unroll
+        for (int j = 0; j < kEdgesPerThread; j++) {
+            const unsigned e = j * kThreads + threadIdx.x;
+            vv[j] = GUM_INF;
+            if (e < tlen) {
+                const unsigned kk = s_head[e];
+                const unsigned long long ci = (unsigned long long)((long long)(tb + e) + s_base[kk]);
+                vv[j] = __ldg(F.col + ci);
+                if (ALG == ALG_BFS) cv[j] = s_val[kk] + 1u;
+                if (ALG == ALG_WCC) cv[j] = s_val[kk];
+                if (ALG == ALG_PR) cv[j] = s_val[kk];
+                if (ALG == ALG_SSSP) {
+                    const unsigned long long nd = (unsigned long long)s_val[kk] + __ldg(F.w + ci);
+                    if (nd >= (unsigned long long)GUM_INF) {
+                        atomicOr(&F.ctl->err, 1u);
+                        vv[j] = GUM_INF;
+                    }
+                    cv[j] = (unsigned)nd;
+                }
+            }
+        }
+        if (ALG == ALG_PR) {
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                if (vv[j] != GUM_INF) {
+                    const unsigned v = vv[j];
+                    int tf = 0;
+                    unsigned lv = v;
+                    if (MULTI) {
+                        tf = frag_of(c, v);
+                        lv = v - c.bounds[tf];
+                        remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
+                    }
+                    atomicAdd(c.f[tf].acc + lv, cv[j]);
+                }
+            }
+        } else {
+            unsigned cur[kEdgesPerThread];
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                cur[j] = 0;
+                if (vv[j] != GUM_INF) {
+                    const int tf = MULTI ? frag_of(c, vv[j]) : 0;
+                    const unsigned lv = MULTI ? vv[j] - c.bounds[tf] : vv[j];
+                    cur[j] = __ldcg(c.f[tf].state + lv);  // check before atomic
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                bool need = false;
+                int tf = 0;
+                unsigned lv = 0;
+                if (vv[j] != GUM_INF && cv[j] < cur[j]) {
+                    tf = MULTI ? frag_of(c, vv[j]) : 0;
+                    lv = MULTI ? vv[j] - c.bounds[tf] : vv[j];
+                    if (MULTI) remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
+                    const unsigned old = atomicMin(c.f[tf].state + lv, (unsigned)cv[j]);
+                    if ((unsigned)cv[j] < old) {
+                        const unsigned bit = 1u << (lv & 31);
+                        const unsigned ob = atomicOr(c.f[tf].bm + (lv >> 5), bit);
+                        need = (ob & bit) == 0;
+                    }
+                }
+                // warp-aggregated append to the owner's activation list (next frontier)
+                if (MULTI) {
+                    const unsigned key = need ? (unsigned)tf : 0xFFFFFFFFu;
+                    const unsigned grp = __match_any_sync(0xffffffffu, key);
+                    if (need) {
+                        const unsigned leader = __ffs(grp) - 1;
+                        unsigned basepos = 0;
+                        if (lane_id() == leader) basepos = atomicAdd(&c.f[tf].ctl->app_cnt, (unsigned)__popc(grp));
+                        basepos = __shfl_sync(grp, basepos, leader);
+                        c.f[tf].app[basepos + __popc(grp & lanemask_lt())] = lv;
+                        acts++;
+                    }
+                } else {
+                    const unsigned grp = __ballot_sync(0xffffffffu, need);
+                    if (grp) {
+                        const unsigned leader = __ffs(grp) - 1;
+                        unsigned basepos = 0;
+                        if (lane_id() == leader) basepos = atomicAdd(&c.f[0].ctl->app_cnt, (unsigned)__popc(grp));
+                        basepos = __shfl_sync(0xffffffffu, basepos, leader);
+                        if (need) {
+                            c.f[0].app[basepos + __popc(grp & lanemask_lt())] = lv;
+                            acts++;
+                        }
+                    }
+                }
+            }
+        }
+        if (threadIdx.x == 0) {
+            atomicAdd(&F.ctl->edges_done, (unsigned long long)tlen);
+            atomicAdd(&F.ctl->chunks_done, 1ull);
+            if (stolen) {
+                atomicAdd(&F.ctl->edges_stolen, (unsigned long long)tlen);
+                atomicAdd(&F.ctl->chunks_stolen, 1ull);
+                e_stolen += tlen;
+            } else {
+                e_own += tlen;
+            }
+        }
+        __syncthreads();
+    }
+    // run counters (warp-reduced) and the per-worker busy window of this iteration
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        remote += __shfl_xor_sync(0xffffffffu, remote, o);
+        acts += __shfl_xor_sync(0xffffffffu, acts, o);
+    }
+    if (lane_id() == 0 && (remote | acts)) {
+        FragCtl* hc = c.f[w % c.P].ctl;
+        if (remote) atomicAdd(&hc->remote_updates, remote);
+        if (acts) atomicAdd(&hc->activations, acts);
+    }
+    gum_iter_trace* tr = c.trace[w0];
+    if (tr && threadIdx.x == 0 && k < (unsigned)kTraceMax) {
+        const unsigned long long t1 = globaltimer();
+        gum_iter_trace* r = tr + k;
+        atomicMin((unsigned long long*)&r->t_start[w], t0);
+        atomicMax((unsigned long long*)&r->t_end[w], t1);
+        if (e_own) atomicAdd((unsigned long long*)&r->edges_own[w], e_own);
+        if (e_stolen) atomicAdd((unsigned long long*)&r->edges_stolen[w], e_stolen);
+    }
+}
+
+// ------------------------------------------------------------------------------------------ PR finalize
+__global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
+    RunCtl* rc = c.rctl[w0];
+    if (vload(&rc->done)) return;
+    const int f = blockIdx.y;
+    const unsigned o = rc->owner[f];
+    if ((int)o < w0 || (int)o >= w0 + nw) return;
+    const FragPtrs& F = c.f[f];
+    // PR's frontier queue is static: re-arm its steal-queue head for the next advance (every
+    // advance of this iteration has finished: kernel boundary / cross-device barrier)
+    if (blockIdx.x == 0 && threadIdx.x == 0) F.ctl->claim = 0;
+    const double N = (double)c.num_vertices, d = c.pr_d, D = rc->pr_D;
+    double dang = 0.0, res = 0.0;
+    for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
+        const double xo = F.x[i];
+        const double nx = (1.0 - d) / N + d * (F.acc[i] + D / N);
+        res += fabs(nx - xo);
+        if (__ldg(F.row_ptr + i + 1) == __ldg(F.row_ptr + i)) dang += nx;
+        F.x[i] = nx;
+        F.acc[i] = 0.0;
+    }
+#pragma unroll
+    for (int s = 16; s > 0; s >>= 1) {
+        dang += __shfl_xor_sync(0xffffffffu, dang, s);
+        res += __shfl_xor_sync(0xffffffffu, res, s);
+    }
+    __shared__ double s_d[kThreads / 32], s_r[kThreads / 32];
+    if (lane_id() == 0) {
+        s_d[threadIdx.x >> 5] = dang;
+        s_r[threadIdx.x >> 5] = res;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double a = 0, b = 0;
+        for (int i = 0; i < kThreads / 32; i++) {
+            a += s_d[i];
+            b += s_r[i];
+        }
+        const unsigned slot = (rc->iter - 1) & 1;
+        atomicAdd(&F.ctl->pr_dang[slot], a);
+        atomicAdd(&F.ctl->pr_resid[slot], b);
+    }
+}
+
+// ------------------------------------------------------------------------------------------ result
+template <typename T>
+__global__ void k_gather(const __grid_constant__ DevCtx c, int f, T* out, int is_pr) {
+    const FragPtrs& F = c.f[f];
+    for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
+        const unsigned ov = F.orig ? F.orig[i] : F.base + i;
+        if (is_pr)
+            ((double*)out)[ov] = F.x[i];
+        else
+            ((unsigned*)out)[ov] = F.state[i];
+    }
+}
+
+// ================================================================================ host launchers
+// Phase A / phase B of one iteration; a cross-device barrier separates them (and follows B) when
+// the workers live on different GPUs. In single-device mode both phases go into one graph body.
+//   BFS/SSSP/WCC: A = filter            B = control, advance
+//   PR:           A = control, advance  B = finalize
+// Phase A / phase B of one iteration; a cross-device barrier separates them (and follows B) when
+// the workers live on different GPUs. In single-device mode both phases go into one graph body.
+//   BFS/SSSP/WCC: A = filter            B = control, advance
+//   PR:           A = control, advance  B = finalize
+template <int ALG>
+static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
+                                   cudaGraphConditionalHandle h, int use_h) {
+    switch (kind) {
+        case KER_FILTER: k_filter<<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
+        case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
+        case KER_ADVANCE:
+            if (c.P > 1)
+                k_advance<ALG, true><<<L.adv_grid, kThreads, 0, s>>>(c, L.w0, L.nw);
+            else
+                k_advance<ALG, false><<<L.adv_grid, kThreads, 0, s>>>(c, L.w0, L.nw);
+            break;
+        case KER_FINALIZE: k_pr_finalize<<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
+                          cudaGraphConditionalHandle h, int use_h) {
+    switch (alg) {
+        case ALG_BFS: return launch_kernel_t<ALG_BFS>(kind, c, L, s, h, use_h);
+        case ALG_SSSP: return launch_kernel_t<ALG_SSSP>(kind, c, L, s, h, use_h);
+        case ALG_WCC: return launch_kernel_t<ALG_WCC>(kind, c, L, s, h, use_h);
+        default: return launch_kernel_t<ALG_PR>(kind, c, L, s, h, use_h);
+    }
+}
+
+int phase_kernels(int alg, int phase, int* kinds) {
+    if (alg != ALG_PR) {
+        if (phase == 0) {
+            kinds[0] = KER_FILTER;
+            return 1;
+        }
+        kinds[0] = KER_CONTROL;
+        kinds[1] = KER_ADVANCE;
+        return 2;
+    }
+    if (phase == 0) {
+        kinds[0] = KER_CONTROL;
+        kinds[1] = KER_ADVANCE;
+        return 2;
+    }
+    kinds[0] = KER_FINALIZE;
+    return 1;
+}
+
+cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
+                         cudaGraphConditionalHandle h, int use_h) {
+    int kinds[2];
+    const int n = phase_kernels(alg, phase, kinds);
+    for (int i = 0; i < n; i++) {
+        cudaError_t e = launch_kernel(alg, kinds[i], c, L, s, h, use_h);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
+cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream_t s, int f0, int nf, double D0,
+                        int src_frag, unsigned src_local) {
+    dim3 g(L.init_grid, nf);
+    switch (alg) {
+        case ALG_BFS: k_init<ALG_BFS><<<g, kThreads, 0, s>>>(c, f0); break;
+        case ALG_SSSP: k_init<ALG_SSSP><<<g, kThreads, 0, s>>>(c, f0); break;
+        case ALG_WCC: k_init<ALG_WCC><<<g, kThreads, 0, s>>>(c, f0); break;
+        default: k_init<ALG_PR><<<g, kThreads, 0, s>>>(c, f0); break;
+    }
+    k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, c.trace[L.w0]);
+    if (src_frag >= f0 && src_frag < f0 + nf) k_init_source<<<1, 1, 0, s>>>(c, src_frag, src_local);
+    if (alg == ALG_PR) {
+        // PR's frontier is every vertex with out-degree > 0: build its queue once (dense filter)
+        k_filter<<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid) {
+    if (is_pr)
+        k_gather<double><<<grid, kThreads, 0, s>>>(c, f, (double*)out, 1);
+    else
+        k_gather<unsigned><<<grid, kThreads, 0, s>>>(c, f, (unsigned*)out, 0);
+    return cudaGetLastError();
+}
+
+cudaError_t advance_occupancy(int* blocks_per_sm) {
+    int a = 0, b = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_advance<ALG_PR, true>, kThreads, 0);
+    if (e != cudaSuccess) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_advance<ALG_SSSP, true>, kThreads, 0);
+    if (e != cudaSuccess) return e;
+    *blocks_per_sm = a < b ? a : b;
+    return cudaSuccess;
+}
+
+}  // namespace gum

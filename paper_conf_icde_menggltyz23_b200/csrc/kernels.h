@@ -1,0 +1,53 @@
+// Host-side launchers of the sm_100a kernels (kernels.cu) and of the setup kernels (setup.cu).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "gum_internal.h"
+
+namespace gum {
+
+enum { ALG_BFS = GUM_BFS, ALG_SSSP = GUM_SSSP, ALG_WCC = GUM_WCC, ALG_PR = GUM_PR };
+
+// One launch unit = the workers [w0, w0+nw) that live on one device.
+struct LaunchCfg {
+    int w0, nw;
+    int adv_grid;     // persistent advance grid (multiple of nw)
+    int filter_grid;  // persistent filter CTAs per fragment
+    int fin_grid;     // PR finalize CTAs per fragment
+    int init_grid;
+};
+
+enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_COUNT = 5 };
+cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
+                          cudaGraphConditionalHandle h, int use_h);
+int phase_kernels(int alg, int phase, int* kinds);
+cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
+                         cudaGraphConditionalHandle h, int use_h);
+cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream_t s, int f0, int nf, double D0,
+                        int src_frag, unsigned src_local);
+cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
+cudaError_t advance_occupancy(int* blocks_per_sm);
+
+// ---- setup (setup.cu): validation, partitioning, relabelling, symmetrisation -------------------
+cudaError_t setup_validate(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                           unsigned* d_err, cudaStream_t s);
+cudaError_t setup_seg_bounds(const unsigned long long* row_ptr, unsigned V, unsigned long long E, int P,
+                             unsigned* d_bounds, cudaStream_t s);
+// RANDOM partitioner: keyed Feistel permutation pi on [0, V) (cycle walking), inverse table, and the
+// relabelled CSR (row of new id pi(v) = row of v, destinations mapped through pi).
+cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w, unsigned V,
+                          unsigned long long E, unsigned long long seed, unsigned* d_inv, unsigned long long* r_row_ptr,
+                          unsigned* r_col, unsigned* r_w, void* tmp, size_t tmp_bytes, cudaStream_t s);
+size_t setup_scan_tmp_bytes(unsigned V);
+// symmetric (out + in) CSR for WCC: sym row v = out-neighbours of v followed by in-neighbours of v.
+cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                             unsigned long long* s_row_ptr, unsigned* s_col, unsigned long long* cursor, void* tmp,
+                             size_t tmp_bytes, cudaStream_t s);
+// fragment extraction: rebased row_ptr slice; orig ids slice (or identity when inv == null)
+cudaError_t setup_rebase_rows(const unsigned long long* row_ptr, unsigned b0, unsigned b1, unsigned long long* out,
+                              cudaStream_t s);
+cudaError_t setup_count_dangling(const unsigned long long* row_ptr, unsigned V, unsigned long long* d_count,
+                                 cudaStream_t s);
+unsigned host_feistel(unsigned v, unsigned V, unsigned long long seed);
+
+}  // namespace gum

@@ -1,0 +1,982 @@
+// Host runtime behind the C ABI (include/gum.h): context, device fragments, partition, the
+// iteration driver (CUDA-graph WHILE loop, or host loop with launch batches) and result/stat
+// readback. PAPER.md lines as P:<line>; SURVEY.md §8(b) is the ABI contract.
+#include <cuda_runtime.h>
+#include <omp.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "gum.h"
+#include "gum_internal.h"
+#include "kernels.h"
+
+using namespace gum;
+
+namespace {
+
+struct Alloc {
+    void* p;
+    size_t bytes;
+    int dev;
+};
+
+struct FragBufs {
+    int dev = 0;
+    unsigned V = 0, base = 0;
+    unsigned long long E = 0, sE = 0;
+    unsigned long long* row_ptr = nullptr;
+    unsigned* col = nullptr;
+    unsigned* w = nullptr;
+    unsigned long long* s_row_ptr = nullptr;
+    unsigned* s_col = nullptr;
+    unsigned* orig = nullptr;
+    unsigned* state = nullptr;
+    double* x = nullptr;
+    double* acc = nullptr;
+    unsigned* bm = nullptr;
+    unsigned* app = nullptr;
+    unsigned* q_v = nullptr;
+    unsigned long long* q_off = nullptr;
+    long long* q_base = nullptr;
+    unsigned* tile = nullptr;
+    unsigned long long tile_cap = 0;
+    FragCtl* ctl = nullptr;
+};
+
+}  // namespace
+
+struct gum_ctx {
+    gum_config cfg{};
+    int P = 1;
+    int dev[kMaxW] = {0};
+    bool single_device = true;
+    int n_units = 1;
+    cudaStream_t stream[kMaxW] = {nullptr};
+    bool own_stream[kMaxW] = {false};
+    int nsm = 148;
+    int adv_occ = 4;
+    std::string err;
+    bool poisoned = false;
+    std::vector<Alloc> load_allocs, part_allocs, misc_allocs;
+    // loaded graph (worker 0's device)
+    bool loaded = false;
+    unsigned V = 0;
+    unsigned long long E = 0;
+    bool has_w = false;
+    unsigned long long* g_row_ptr = nullptr;
+    unsigned* g_col = nullptr;
+    unsigned* g_w = nullptr;
+    // partition
+    bool partitioned = false;
+    int part_kind = GUM_PART_SEG;
+    unsigned long long seed = 0;
+    unsigned bounds[kMaxW + 1] = {0};
+    unsigned* inv = nullptr;  // relabelled id -> original id (RANDOM)
+    unsigned long long* p_row_ptr = nullptr;  // the partitioned global CSR (relabelled or original)
+    unsigned* p_col = nullptr;
+    unsigned* p_w = nullptr;
+    bool sym_ready = false;
+    FragBufs fr[kMaxW];
+    unsigned long long n_dangling = 0;
+    RunCtl* rctl[kMaxW] = {nullptr};
+    LBSlot* lb[kMaxW] = {nullptr};
+    unsigned lb_parts = 0;
+    gum_iter_trace* trace[kMaxW] = {nullptr};
+    RunCtl* h_rctl = nullptr;  // pinned
+    void* d_res = nullptr;
+    cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    std::vector<cudaEvent_t> bar_ev;
+    std::vector<cudaEvent_t> prof_ev;  // pairs (start, end)
+    std::vector<int> prof_kind;
+    gum_kernel_times prof{};
+    int last_alg = -1;
+    bool has_result = false;
+    unsigned last_iters = 0;
+};
+
+namespace {
+
+gum_status fail(gum_ctx* c, gum_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    if (c) {
+        c->err = buf;
+        if (st == GUM_ECUDA) c->poisoned = true;
+    }
+    return st;
+}
+
+#define CK(call)                                                                                  \
+    do {                                                                                          \
+        cudaError_t e_ = (call);                                                                  \
+        if (e_ != cudaSuccess) return fail(c, GUM_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), \
+                                           __FILE__, __LINE__);                                   \
+    } while (0)
+
+void* dalloc(gum_ctx* c, int dev, size_t bytes, std::vector<Alloc>& list) {
+    bytes = std::max<size_t>(bytes, 256);
+    bytes = (bytes + 255) & ~size_t(255);
+    void* p = nullptr;
+    if (c->cfg.alloc) {
+        p = c->cfg.alloc(bytes, dev, c->cfg.alloc_user);
+    } else {
+        cudaSetDevice(dev);
+        if (cudaMalloc(&p, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+        }
+    }
+    if (p) list.push_back({p, bytes, dev});
+    return p;
+}
+
+void free_list(gum_ctx* c, std::vector<Alloc>& list) {
+    for (auto& a : list) {
+        if (c->cfg.free_fn) {
+            c->cfg.free_fn(a.p, a.bytes, a.dev, c->cfg.alloc_user);
+        } else {
+            cudaSetDevice(a.dev);
+            cudaFree(a.p);
+        }
+    }
+    list.clear();
+}
+
+void drop_graphs(gum_ctx* c) {
+    for (auto& g : c->gexec) {
+        if (g) cudaGraphExecDestroy(g);
+        g = nullptr;
+    }
+}
+
+void drop_partition(gum_ctx* c) {
+    drop_graphs(c);
+    for (int d = 0; d < c->P; d++) {
+        cudaSetDevice(c->dev[d]);
+        cudaStreamSynchronize(c->stream[d]);
+    }
+    free_list(c, c->part_allocs);
+    c->partitioned = false;
+    c->sym_ready = false;
+    c->has_result = false;
+    c->inv = nullptr;
+    c->p_row_ptr = nullptr;
+    c->p_col = nullptr;
+    c->p_w = nullptr;
+    for (auto& f : c->fr) f = FragBufs{};
+    for (int i = 0; i < kMaxW; i++) {
+        c->rctl[i] = nullptr;
+        c->lb[i] = nullptr;
+        c->trace[i] = nullptr;
+    }
+    c->d_res = nullptr;
+}
+
+// unit u covers workers [unit_w0(u), unit_w0(u)+unit_nw(u))
+int unit_w0(const gum_ctx* c, int u) { return c->single_device ? 0 : u; }
+int unit_nw(const gum_ctx* c, int u) { return c->single_device ? c->P : 1; }
+int unit_dev(const gum_ctx* c, int u) { return c->dev[unit_w0(c, u)]; }
+
+LaunchCfg make_launch(const gum_ctx* c, int u) {
+    LaunchCfg L;
+    L.w0 = unit_w0(c, u);
+    L.nw = unit_nw(c, u);
+    int grid = c->nsm * c->adv_occ;
+    grid = (grid / L.nw) * L.nw;
+    if (grid < L.nw) grid = L.nw;
+    L.adv_grid = grid;
+    L.filter_grid = std::max(1, (c->nsm * 2) / (c->single_device ? std::min(c->P, 2) : 1));
+    L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
+    L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
+    return L;
+}
+
+DevCtx make_devctx(const gum_ctx* c, int alg) {
+    DevCtx d;
+    memset(&d, 0, sizeof(d));
+    for (int f = 0; f < c->P; f++) {
+        const FragBufs& F = c->fr[f];
+        FragPtrs& p = d.f[f];
+        if (alg == GUM_WCC) {
+            p.row_ptr = F.s_row_ptr;
+            p.col = F.s_col;
+            p.E = F.sE;
+        } else {
+            p.row_ptr = F.row_ptr;
+            p.col = F.col;
+            p.E = F.E;
+        }
+        p.w = F.w;
+        p.state = F.state;
+        p.x = F.x;
+        p.acc = F.acc;
+        p.orig = F.orig;
+        p.bm = F.bm;
+        p.app = F.app;
+        p.q_v = F.q_v;
+        p.q_off = F.q_off;
+        p.q_base = F.q_base;
+        p.tile = F.tile;
+        p.ctl = F.ctl;
+        p.V = F.V;
+        p.base = F.base;
+        d.lb[f] = c->lb[f];
+    }
+    for (int w = 0; w < c->P; w++) {
+        int u = c->single_device ? 0 : w;
+        d.rctl[w] = c->rctl[unit_w0(c, u)];
+        d.trace[w] = c->trace[unit_w0(c, u)];
+    }
+    d.lb_parts = c->lb_parts;
+    for (int i = 0; i <= c->P; i++) d.bounds[i] = c->bounds[i];
+    d.P = c->P;
+    d.chunk = c->cfg.chunk_edges;
+    d.num_vertices = c->V;
+    d.fsteal = c->cfg.fsteal;
+    d.osteal = c->cfg.osteal;
+    d.t1 = c->cfg.t1_min_max_edges;
+    d.t2 = c->cfg.t2_min_spread_edges;
+    d.os_thresh = c->cfg.osteal_active_threshold;
+    d.os_epw = c->cfg.osteal_edges_per_worker;
+    d.max_iter = c->cfg.max_iterations ? c->cfg.max_iterations : 0x7FFFFFFFu;
+    d.pr_iters = c->cfg.pr_iterations;
+    d.pr_d = c->cfg.pr_damping;
+    d.force_mode = (c->cfg.flags & GUM_CFG_FORCE_DENSE) ? 2u : ((c->cfg.flags & GUM_CFG_FORCE_SPARSE) ? 1u : 0u);
+    d.dense_div = 32;
+    return d;
+}
+
+gum_status sync_all(gum_ctx* c) {
+    for (int u = 0; u < c->n_units; u++) {
+        CK(cudaSetDevice(unit_dev(c, u)));
+        CK(cudaStreamSynchronize(c->stream[unit_w0(c, u)]));
+    }
+    return GUM_OK;
+}
+
+// cross-unit barrier (multi-device, single process): every unit's stream waits for every other's.
+gum_status unit_barrier(gum_ctx* c) {
+    if (c->n_units == 1) return GUM_OK;
+    for (int u = 0; u < c->n_units; u++) {
+        CK(cudaSetDevice(unit_dev(c, u)));
+        CK(cudaEventRecord(c->bar_ev[u], c->stream[unit_w0(c, u)]));
+    }
+    for (int u = 0; u < c->n_units; u++) {
+        CK(cudaSetDevice(unit_dev(c, u)));
+        for (int v = 0; v < c->n_units; v++)
+            if (v != u) CK(cudaStreamWaitEvent(c->stream[unit_w0(c, u)], c->bar_ev[v], 0));
+    }
+    return GUM_OK;
+}
+
+gum_status ensure_fragment_state(gum_ctx* c, int f, unsigned long long max_edges) {
+    FragBufs& F = c->fr[f];
+    const unsigned long long need = max_edges / c->cfg.chunk_edges + 2;
+    if (F.tile && F.tile_cap >= need) return GUM_OK;
+    F.tile = (unsigned*)dalloc(c, F.dev, need * sizeof(unsigned), c->part_allocs);
+    if (!F.tile) return fail(c, GUM_ENOMEM, "tile table alloc failed (fragment %d)", f);
+    F.tile_cap = need;
+    return GUM_OK;
+}
+
+gum_status build_sym(gum_ctx* c) {
+    if (c->sym_ready) return GUM_OK;
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    const unsigned long long sE = 2ull * c->E;
+    std::vector<Alloc> tmp;
+    unsigned long long* srp = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, c->part_allocs);
+    unsigned* scol = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(sE, 1) * 4, c->part_allocs);
+    unsigned long long* cursor = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, tmp);
+    size_t tb = setup_scan_tmp_bytes(c->V);
+    void* t = dalloc(c, d0, tb, tmp);
+    if (!srp || !scol || !cursor || !t) {
+        free_list(c, tmp);
+        return fail(c, GUM_ENOMEM, "symmetric CSR alloc failed (%llu entries)", sE);
+    }
+    cudaError_t e = setup_symmetrize(c->p_row_ptr, c->p_col, c->V, c->E, srp, scol, cursor, t, tb, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    free_list(c, tmp);
+    if (e != cudaSuccess) return fail(c, GUM_ECUDA, "symmetrize: %s", cudaGetErrorString(e));
+    std::vector<unsigned long long> hb(c->P + 1);
+    for (int f = 0; f <= c->P; f++) CK(cudaMemcpy(&hb[f], srp + c->bounds[f], 8, cudaMemcpyDeviceToHost));
+    for (int f = 0; f < c->P; f++) {
+        FragBufs& F = c->fr[f];
+        F.sE = hb[f + 1] - hb[f];
+        if (c->P == 1 && c->single_device) {
+            F.s_row_ptr = srp;
+            F.s_col = scol;
+        } else {
+            F.s_row_ptr = (unsigned long long*)dalloc(c, F.dev, (F.V + 1ull) * 8, c->part_allocs);
+            F.s_col = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.sE, 1) * 4, c->part_allocs);
+            if (!F.s_row_ptr || !F.s_col) return fail(c, GUM_ENOMEM, "sym fragment alloc failed");
+            unsigned long long* tmp_rp = F.s_row_ptr;
+            std::vector<Alloc> t2;
+            if (F.dev != d0) tmp_rp = (unsigned long long*)dalloc(c, d0, (F.V + 1ull) * 8, t2);
+            CK(setup_rebase_rows(srp, c->bounds[f], c->bounds[f + 1], tmp_rp, s));
+            if (F.dev != d0) CK(cudaMemcpyPeerAsync(F.s_row_ptr, F.dev, tmp_rp, d0, (F.V + 1ull) * 8, s));
+            if (F.sE) CK(cudaMemcpyPeerAsync(F.s_col, F.dev, scol + hb[f], d0, F.sE * 4, s));
+            CK(cudaStreamSynchronize(s));
+            free_list(c, t2);
+        }
+        gum_status st = ensure_fragment_state(c, f, std::max(F.E, F.sE));
+        if (st != GUM_OK) return st;
+    }
+    c->sym_ready = true;
+    drop_graphs(c);
+    return GUM_OK;
+}
+
+// Launch one phase; in profile mode bracket every kernel with a pair of CUDA events.
+gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const LaunchCfg& L, cudaStream_t s) {
+    if (!(c->cfg.flags & GUM_CFG_PROFILE)) {
+        CK(launch_phase(alg, phase, d, L, s, 0, 0));
+        return GUM_OK;
+    }
+    int kinds[2];
+    const int n = phase_kernels(alg, phase, kinds);
+    for (int i = 0; i < n; i++) {
+        cudaEvent_t a, b;
+        CK(cudaEventCreate(&a));
+        CK(cudaEventCreate(&b));
+        CK(cudaEventRecord(a, s));
+        CK(launch_kernel(alg, kinds[i], d, L, s, 0, 0));
+        CK(cudaEventRecord(b, s));
+        c->prof_ev.push_back(a);
+        c->prof_ev.push_back(b);
+        c->prof_kind.push_back(kinds[i]);
+    }
+    return GUM_OK;
+}
+
+gum_status capture_graph(gum_ctx* c, int alg, const DevCtx& d, const LaunchCfg& L) {
+    if (c->gexec[alg]) return GUM_OK;
+    cudaStream_t s = c->stream[0];
+    cudaGraph_t g;
+    CK(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle h;
+    CK(cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault));
+    alignas(cudaGraphNodeParams) unsigned char pbuf[sizeof(cudaGraphNodeParams)];
+    memset(pbuf, 0, sizeof(pbuf));
+    cudaGraphNodeParams& p = *reinterpret_cast<cudaGraphNodeParams*>(pbuf);
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeWhile;
+    p.conditional.size = 1;
+    cudaGraphNode_t node;
+    CK(cudaGraphAddNode(&node, g, nullptr, 0, &p));
+    cudaGraph_t body = p.conditional.phGraph_out[0];
+    CK(cudaStreamBeginCaptureToGraph(s, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+    cudaError_t e = launch_phase(alg, 0, d, L, s, h, 1);
+    if (e == cudaSuccess) e = launch_phase(alg, 1, d, L, s, h, 1);
+    cudaGraph_t captured;
+    cudaError_t e2 = cudaStreamEndCapture(s, &captured);
+    if (e != cudaSuccess || e2 != cudaSuccess) {
+        cudaGraphDestroy(g);
+        return fail(c, GUM_ECUDA, "graph capture: %s / %s", cudaGetErrorString(e), cudaGetErrorString(e2));
+    }
+    cudaGraphExec_t ex;
+    CK(cudaGraphInstantiate(&ex, g, 0));
+    cudaGraphDestroy(g);
+    c->gexec[alg] = ex;
+    return GUM_OK;
+}
+
+}  // namespace
+
+// ================================================================================ C ABI
+extern "C" {
+
+int gum_version(void) { return 100; }
+
+void gum_config_default(gum_config* cfg) {
+    if (!cfg) return;
+    memset(cfg, 0, sizeof(*cfg));
+    cfg->num_gpus = 1;
+    cfg->fsteal = 1;
+    cfg->osteal = 1;
+    cfg->chunk_edges = 2048;
+    cfg->pr_iterations = 20;
+    cfg->pr_damping = 0.85;
+}
+
+const char* gum_last_error(const gum_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
+    if (!cfg || !out) return GUM_EINVAL;
+    *out = nullptr;
+    if (cfg->num_gpus < 1 || cfg->num_gpus > kMaxW) return GUM_EINVAL;
+    gum_ctx* c = new gum_ctx();
+    c->cfg = *cfg;
+    if (c->cfg.chunk_edges == 0) c->cfg.chunk_edges = kTileMax;
+    if (c->cfg.chunk_edges > (unsigned)kTileMax || c->cfg.chunk_edges % 32 != 0) {
+        delete c;
+        return GUM_EINVAL;
+    }
+    if (c->cfg.pr_iterations <= 0) c->cfg.pr_iterations = 20;
+    if (c->cfg.pr_damping <= 0.0) c->cfg.pr_damping = 0.85;
+    c->P = cfg->num_gpus;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        delete c;
+        return GUM_ECUDA;
+    }
+    for (int i = 0; i < c->P; i++) {
+        c->dev[i] = cfg->device_ids ? cfg->device_ids[i] : 0;
+        if (c->dev[i] < 0 || c->dev[i] >= ndev) {
+            delete c;
+            return GUM_EINVAL;
+        }
+    }
+    c->single_device = true;
+    for (int i = 1; i < c->P; i++)
+        if (c->dev[i] != c->dev[0]) c->single_device = false;
+    if (!c->single_device) {
+        for (int i = 0; i < c->P; i++)
+            for (int j = 0; j < c->P; j++)
+                if (i != j && c->dev[i] == c->dev[j]) {
+                    delete c;
+                    return GUM_EUNSUP;  // mixed: some workers share a device, others do not
+                }
+    }
+    c->n_units = c->single_device ? 1 : c->P;
+    for (int u = 0; u < c->n_units; u++) {
+        int d = unit_dev(c, u);
+        int w0 = unit_w0(c, u);
+        cudaSetDevice(d);
+        if (cfg->streams && cfg->streams[w0]) {
+            c->stream[w0] = (cudaStream_t)cfg->streams[w0];
+        } else {
+            if (cudaStreamCreateWithFlags(&c->stream[w0], cudaStreamNonBlocking) != cudaSuccess) {
+                cudaGetLastError();
+                delete c;
+                return GUM_ECUDA;
+            }
+            c->own_stream[w0] = true;
+        }
+        if (!c->single_device) {
+            for (int v = 0; v < c->P; v++) {
+                if (v == u) continue;
+                int can = 0;
+                cudaDeviceCanAccessPeer(&can, d, c->dev[v]);
+                if (!can) {
+                    delete c;
+                    return GUM_EUNSUP;
+                }
+                cudaError_t e = cudaDeviceEnablePeerAccess(c->dev[v], 0);
+                if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+                    cudaGetLastError();
+                    delete c;
+                    return GUM_ECUDA;
+                }
+                cudaGetLastError();
+            }
+        }
+        cudaEvent_t ev;
+        cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+        c->bar_ev.push_back(ev);
+    }
+    cudaSetDevice(c->dev[0]);
+    cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->dev[0]);
+    int occ = 0;
+    if (advance_occupancy(&occ) == cudaSuccess && occ > 0) c->adv_occ = occ;
+    cudaGetLastError();
+    cudaEventCreate(&c->ev0);
+    cudaEventCreate(&c->ev1);
+    if (cudaMallocHost(&c->h_rctl, sizeof(RunCtl)) != cudaSuccess) {
+        cudaGetLastError();
+        delete c;
+        return GUM_ENOMEM;
+    }
+    *out = c;
+    return GUM_OK;
+}
+
+void gum_destroy(gum_ctx* c) {
+    if (!c) return;
+    drop_partition(c);
+    free_list(c, c->load_allocs);
+    free_list(c, c->misc_allocs);
+    for (int i = 0; i < kMaxW; i++) {
+        if (c->own_stream[i]) {
+            cudaSetDevice(c->dev[i]);
+            cudaStreamDestroy(c->stream[i]);
+        }
+    }
+    for (auto e : c->bar_ev) cudaEventDestroy(e);
+    if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->h_rctl) cudaFreeHost(c->h_rctl);
+    delete c;
+}
+
+gum_status gum_build_csr(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                         uint64_t* row_ptr, uint32_t* col, uint32_t* wout) {
+    if ((!src || !dst || !col) && E) return GUM_EINVAL;
+    if (!row_ptr) return GUM_EINVAL;
+    if (w && !wout && E) return GUM_EINVAL;
+    const int T = omp_get_max_threads();
+    // per-thread histograms over contiguous edge ranges -> stable counting sort
+    std::vector<std::vector<uint64_t>> hist(T);
+    int bad = 0;
+#pragma omp parallel num_threads(T) reduction(| : bad)
+    {
+        int t = omp_get_thread_num();
+        auto& h = hist[t];
+        h.assign((size_t)V + 1, 0);
+        uint64_t lo = E * t / T, hi = E * (t + 1) / T;
+        for (uint64_t i = lo; i < hi; i++) {
+            if (src[i] >= V || dst[i] >= V) {
+                bad = 1;
+                continue;
+            }
+            h[src[i]]++;
+        }
+    }
+    if (bad) return GUM_EINVAL;
+    // row_ptr and per-thread write cursors (thread t's edges of row v follow threads < t)
+    row_ptr[0] = 0;
+    {
+        // column-wise prefix over (v, t)
+        std::vector<uint64_t> rowsum((size_t)V, 0);
+#pragma omp parallel for num_threads(T) schedule(static)
+        for (int64_t v = 0; v < (int64_t)V; v++) {
+            uint64_t s = 0;
+            for (int t = 0; t < T; t++) {
+                uint64_t x = hist[t][v];
+                hist[t][v] = s;
+                s += x;
+            }
+            rowsum[v] = s;
+        }
+        for (uint64_t v = 0; v < V; v++) row_ptr[v + 1] = row_ptr[v] + rowsum[v];
+    }
+#pragma omp parallel num_threads(T)
+    {
+        int t = omp_get_thread_num();
+        auto& h = hist[t];
+        uint64_t lo = E * t / T, hi = E * (t + 1) / T;
+        for (uint64_t i = lo; i < hi; i++) {
+            uint32_t u = src[i];
+            uint64_t pos = row_ptr[u] + h[u]++;
+            col[pos] = dst[i];
+            if (w) wout[pos] = w[i];
+        }
+    }
+    return GUM_OK;
+}
+
+gum_status gum_load_csr(gum_ctx* c, uint32_t V, uint64_t E, const uint64_t* row_ptr, const uint32_t* col_idx,
+                        const uint32_t* weights, uint32_t flags) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned by an earlier CUDA error");
+    if (!row_ptr || (!col_idx && E)) return fail(c, GUM_EINVAL, "null row_ptr/col_idx");
+    if (V == 0 || V > 0xFFFFFFFEu) return fail(c, GUM_EINVAL, "V must be in [1, 2^32-2]");
+    drop_partition(c);
+    free_list(c, c->load_allocs);
+    c->loaded = false;
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    c->g_row_ptr = (unsigned long long*)dalloc(c, d0, (V + 1ull) * 8, c->load_allocs);
+    c->g_col = (unsigned*)dalloc(c, d0, std::max<uint64_t>(E, 1) * 4, c->load_allocs);
+    c->g_w = weights ? (unsigned*)dalloc(c, d0, std::max<uint64_t>(E, 1) * 4, c->load_allocs) : nullptr;
+    unsigned* d_err = (unsigned*)dalloc(c, d0, 256, c->load_allocs);
+    if (!c->g_row_ptr || !c->g_col || (weights && !c->g_w) || !d_err) {
+        free_list(c, c->load_allocs);
+        return fail(c, GUM_ENOMEM, "graph alloc failed (V=%u E=%llu)", V, (unsigned long long)E);
+    }
+    const cudaMemcpyKind kind = (flags & GUM_LOAD_DEVICE) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+    CK(cudaMemcpyAsync(c->g_row_ptr, row_ptr, (V + 1ull) * 8, kind, s));
+    if (E) CK(cudaMemcpyAsync(c->g_col, col_idx, E * 4, kind, s));
+    if (weights && E) CK(cudaMemcpyAsync(c->g_w, weights, E * 4, kind, s));
+    CK(cudaMemsetAsync(d_err, 0, 4, s));
+    CK(setup_validate(c->g_row_ptr, c->g_col, V, E, d_err, s));
+    unsigned herr = 0;
+    CK(cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (herr) {
+        free_list(c, c->load_allocs);
+        return fail(c, GUM_EINVAL, "malformed CSR (code %u: 1=row_ptr[0]!=0 2=row_ptr[V]!=E 4=not monotone 8=col>=V)",
+                    herr);
+    }
+    c->V = V;
+    c->E = E;
+    c->has_w = weights != nullptr;
+    c->loaded = true;
+    return GUM_OK;
+}
+
+gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
+    if (!c->loaded) return fail(c, GUM_ESTATE, "gum_partition before gum_load_csr");
+    if (kind != GUM_PART_SEG && kind != GUM_PART_RANDOM) return fail(c, GUM_EINVAL, "bad partition kind");
+    drop_partition(c);
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    const unsigned V = c->V;
+    const unsigned long long E = c->E;
+    c->part_kind = kind;
+    c->seed = seed;
+    // ---- a2: relabel (RANDOM) then edge-balanced contiguous ranges (SEG)
+    if (kind == GUM_PART_RANDOM) {
+        c->inv = (unsigned*)dalloc(c, d0, (size_t)V * 4, c->part_allocs);
+        c->p_row_ptr = (unsigned long long*)dalloc(c, d0, (V + 1ull) * 8, c->part_allocs);
+        c->p_col = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs);
+        c->p_w = c->has_w ? (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs) : nullptr;
+        std::vector<Alloc> tmp;
+        size_t tb = setup_scan_tmp_bytes(V);
+        void* t = dalloc(c, d0, tb, tmp);
+        if (!c->inv || !c->p_row_ptr || !c->p_col || (c->has_w && !c->p_w) || !t) {
+            free_list(c, tmp);
+            return fail(c, GUM_ENOMEM, "relabel alloc failed");
+        }
+        cudaError_t e = setup_relabel(c->g_row_ptr, c->g_col, c->g_w, V, E, seed, c->inv, c->p_row_ptr, c->p_col,
+                                      c->p_w, t, tb, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        free_list(c, tmp);
+        if (e != cudaSuccess) return fail(c, GUM_ECUDA, "relabel: %s", cudaGetErrorString(e));
+    } else {
+        c->inv = nullptr;
+        c->p_row_ptr = c->g_row_ptr;
+        c->p_col = c->g_col;
+        c->p_w = c->g_w;
+    }
+    {
+        std::vector<Alloc> tmp;
+        unsigned* db = (unsigned*)dalloc(c, d0, 64, tmp);
+        CK(setup_seg_bounds(c->p_row_ptr, V, E, c->P, db, s));
+        CK(cudaMemcpyAsync(c->bounds, db, (c->P + 1) * 4, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        free_list(c, tmp);
+    }
+    std::vector<unsigned long long> eb(c->P + 1);
+    for (int f = 0; f <= c->P; f++) CK(cudaMemcpy(&eb[f], c->p_row_ptr + c->bounds[f], 8, cudaMemcpyDeviceToHost));
+    // ---- per-fragment device CSR + state + frontier + control
+    for (int f = 0; f < c->P; f++) {
+        FragBufs& F = c->fr[f];
+        F.dev = c->dev[f];
+        F.base = c->bounds[f];
+        F.V = c->bounds[f + 1] - c->bounds[f];
+        F.E = eb[f + 1] - eb[f];
+        const size_t Vn = std::max<size_t>(F.V, 1);
+        if (c->P == 1 && c->single_device) {
+            F.row_ptr = c->p_row_ptr;
+            F.col = c->p_col;
+            F.w = c->p_w;
+            F.orig = c->inv;
+        } else {
+            F.row_ptr = (unsigned long long*)dalloc(c, F.dev, (F.V + 1ull) * 8, c->part_allocs);
+            F.col = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.E, 1) * 4, c->part_allocs);
+            F.w = c->has_w ? (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.E, 1) * 4, c->part_allocs)
+                           : nullptr;
+            F.orig = c->inv ? (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs) : nullptr;
+            if (!F.row_ptr || !F.col || (c->has_w && !F.w) || (c->inv && !F.orig))
+                return fail(c, GUM_ENOMEM, "fragment %d CSR alloc failed", f);
+            std::vector<Alloc> t2;
+            unsigned long long* tmp_rp = F.row_ptr;
+            if (F.dev != d0) tmp_rp = (unsigned long long*)dalloc(c, d0, (F.V + 1ull) * 8, t2);
+            CK(setup_rebase_rows(c->p_row_ptr, c->bounds[f], c->bounds[f + 1], tmp_rp, s));
+            if (F.dev != d0) CK(cudaMemcpyPeerAsync(F.row_ptr, F.dev, tmp_rp, d0, (F.V + 1ull) * 8, s));
+            if (F.E) CK(cudaMemcpyPeerAsync(F.col, F.dev, c->p_col + eb[f], d0, F.E * 4, s));
+            if (F.E && F.w) CK(cudaMemcpyPeerAsync(F.w, F.dev, c->p_w + eb[f], d0, F.E * 4, s));
+            if (F.orig && F.V) CK(cudaMemcpyPeerAsync(F.orig, F.dev, c->inv + F.base, d0, (size_t)F.V * 4, s));
+            CK(cudaStreamSynchronize(s));
+            free_list(c, t2);
+        }
+        F.state = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
+        F.x = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
+        F.acc = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
+        F.bm = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
+        F.app = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
+        F.q_v = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
+        F.q_off = (unsigned long long*)dalloc(c, F.dev, (Vn + 1) * 8, c->part_allocs);
+        F.q_base = (long long*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
+        F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
+        if (!F.state || !F.x || !F.acc || !F.bm || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
+            return fail(c, GUM_ENOMEM, "fragment %d state alloc failed", f);
+        CK(cudaSetDevice(F.dev));
+        CK(cudaMemset(F.ctl, 0, sizeof(FragCtl)));
+        CK(cudaSetDevice(d0));
+        gum_status st = ensure_fragment_state(c, f, F.E);
+        if (st != GUM_OK) return st;
+    }
+    // look-back slots (per fragment, in the fragment's memory) and per-unit run control
+    unsigned parts = 1;
+    for (int f = 0; f < c->P; f++) {
+        unsigned nwords = (c->fr[f].V + 31) / 32;
+        unsigned a = (nwords + kFilterWordsPerPart - 1) / kFilterWordsPerPart;
+        unsigned b = (c->fr[f].V + kFilterAppPerPart - 1) / kFilterAppPerPart;
+        parts = std::max(parts, std::max(a, b) + 1);
+    }
+    c->lb_parts = parts;
+    for (int f = 0; f < c->P; f++) {
+        c->lb[f] = (LBSlot*)dalloc(c, c->fr[f].dev, (size_t)parts * sizeof(LBSlot), c->part_allocs);
+        if (!c->lb[f]) return fail(c, GUM_ENOMEM, "look-back alloc failed");
+        CK(cudaSetDevice(c->fr[f].dev));
+        CK(cudaMemset(c->lb[f], 0, (size_t)parts * sizeof(LBSlot)));
+    }
+    for (int u = 0; u < c->n_units; u++) {
+        int w0 = unit_w0(c, u), d = unit_dev(c, u);
+        c->rctl[w0] = (RunCtl*)dalloc(c, d, sizeof(RunCtl), c->part_allocs);
+        if (!c->rctl[w0]) return fail(c, GUM_ENOMEM, "run control alloc failed");
+        CK(cudaSetDevice(d));
+        CK(cudaMemset(c->rctl[w0], 0, sizeof(RunCtl)));
+        if (c->cfg.flags & GUM_CFG_TRACE) {
+            c->trace[w0] = (gum_iter_trace*)dalloc(c, d, (size_t)kTraceMax * sizeof(gum_iter_trace), c->part_allocs);
+            if (!c->trace[w0]) return fail(c, GUM_ENOMEM, "trace alloc failed");
+        }
+    }
+    CK(cudaSetDevice(d0));
+    {
+        std::vector<Alloc> tmp;
+        unsigned long long* dc = (unsigned long long*)dalloc(c, d0, 64, tmp);
+        CK(cudaMemsetAsync(dc, 0, 8, s));
+        CK(setup_count_dangling(c->p_row_ptr, V, dc, s));
+        CK(cudaMemcpyAsync(&c->n_dangling, dc, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        free_list(c, tmp);
+    }
+    c->d_res = dalloc(c, d0, (size_t)V * 8, c->part_allocs);
+    if (!c->d_res) return fail(c, GUM_ENOMEM, "result buffer alloc failed");
+    c->partitioned = true;
+    return GUM_OK;
+}
+
+gum_status gum_partition_bounds(const gum_ctx* c, uint32_t* bounds, int n) {
+    if (!c || !bounds) return GUM_EINVAL;
+    if (!c->partitioned) return GUM_ESTATE;
+    for (int i = 0; i <= c->P && i < n; i++) bounds[i] = c->bounds[i];
+    return GUM_OK;
+}
+
+gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
+    if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
+    if (alg == GUM_WCC) return build_sym(c);
+    if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
+    return GUM_OK;
+}
+
+gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stats) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
+    if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_run before gum_partition");
+    if (alg < GUM_BFS || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
+    if (alg == GUM_SSSP && !c->has_w) return fail(c, GUM_EINVAL, "SSSP needs edge weights");
+    if ((alg == GUM_BFS || alg == GUM_SSSP) && source >= c->V) return fail(c, GUM_ERANGE, "source %u >= V", source);
+    gum_status st = gum_prepare(c, alg);
+    if (st != GUM_OK) return st;
+    c->has_result = false;
+    const DevCtx d = make_devctx(c, alg);
+    int src_frag = -1;
+    unsigned src_local = 0;
+    if (alg == GUM_BFS || alg == GUM_SSSP) {
+        unsigned sp = c->inv ? host_feistel(source, c->V, c->seed) : source;
+        for (int f = 0; f < c->P; f++)
+            if (sp >= c->bounds[f] && sp < c->bounds[f + 1]) src_frag = f;
+        src_local = sp - c->bounds[src_frag];
+    }
+    const double D0 = (double)c->n_dangling / (double)c->V;
+    const bool profile = (c->cfg.flags & GUM_CFG_PROFILE) != 0;
+    if (profile && !c->single_device) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single device");
+    const bool graph_mode = c->single_device && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
+    for (auto e : c->prof_ev) cudaEventDestroy(e);
+    c->prof_ev.clear();
+    c->prof_kind.clear();
+    memset(&c->prof, 0, sizeof(c->prof));
+    cudaEvent_t init_a = nullptr, init_b = nullptr;
+    if (graph_mode) {
+        CK(cudaSetDevice(c->dev[0]));
+        st = capture_graph(c, alg, d, make_launch(c, 0));
+        if (st != GUM_OK) return st;
+    }
+    CK(cudaSetDevice(c->dev[0]));
+    CK(cudaEventRecord(c->ev0, c->stream[0]));
+    if (c->n_units > 1) {
+        st = unit_barrier(c);
+        if (st != GUM_OK) return st;
+    }
+    if (profile) {
+        CK(cudaEventCreate(&init_a));
+        CK(cudaEventCreate(&init_b));
+        CK(cudaEventRecord(init_a, c->stream[0]));
+    }
+    for (int u = 0; u < c->n_units; u++) {
+        const LaunchCfg L = make_launch(c, u);
+        CK(cudaSetDevice(unit_dev(c, u)));
+        CK(launch_init(alg, d, L, c->stream[L.w0], L.w0, L.nw, D0, src_frag, src_local));
+    }
+    if (profile) CK(cudaEventRecord(init_b, c->stream[0]));
+    if (graph_mode) {
+        CK(cudaGraphLaunch(c->gexec[alg], c->stream[0]));
+    } else {
+        // host-driven loop: launch batches of iterations, then poll the device-side done flag
+        const int B = profile ? 1 : 8;
+        for (;;) {
+            for (int b = 0; b < B; b++) {
+                for (int phase = 0; phase < 2; phase++) {
+                    st = unit_barrier(c);
+                    if (st != GUM_OK) return st;
+                    for (int u = 0; u < c->n_units; u++) {
+                        const LaunchCfg L = make_launch(c, u);
+                        CK(cudaSetDevice(unit_dev(c, u)));
+                        st = run_phase(c, alg, phase, d, L, c->stream[L.w0]);
+                        if (st != GUM_OK) return st;
+                    }
+                }
+            }
+            CK(cudaSetDevice(c->dev[0]));
+            CK(cudaMemcpyAsync(c->h_rctl, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost, c->stream[0]));
+            CK(cudaStreamSynchronize(c->stream[0]));
+            if (c->h_rctl->done) break;
+        }
+        st = unit_barrier(c);
+        if (st != GUM_OK) return st;
+    }
+    CK(cudaSetDevice(c->dev[0]));
+    CK(cudaEventRecord(c->ev1, c->stream[0]));
+    st = sync_all(c);
+    if (st != GUM_OK) return st;
+    CK(cudaMemcpy(c->h_rctl, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+    const RunCtl R = *c->h_rctl;
+    if (profile) {
+        float t = 0.f;
+        CK(cudaEventElapsedTime(&t, init_a, init_b));
+        c->prof.init_ms = t;
+        c->prof.init_launches = (alg == GUM_BFS || alg == GUM_SSSP) ? 3 : (alg == GUM_PR ? 3 : 2);
+        cudaEventDestroy(init_a);
+        cudaEventDestroy(init_b);
+        for (size_t i = 0; i < c->prof_kind.size(); i++) {
+            CK(cudaEventElapsedTime(&t, c->prof_ev[2 * i], c->prof_ev[2 * i + 1]));
+            switch (c->prof_kind[i]) {
+                case KER_FILTER: c->prof.filter_ms += t; c->prof.filter_launches++; break;
+                case KER_CONTROL: c->prof.control_ms += t; c->prof.control_launches++; break;
+                case KER_ADVANCE: c->prof.advance_ms += t; c->prof.advance_launches++; break;
+                default: c->prof.finalize_ms += t; c->prof.finalize_launches++; break;
+            }
+        }
+    }
+    c->last_alg = alg;
+    c->last_iters = R.iter;
+    if (R.err) return fail(c, GUM_ERANGE, "SSSP distance reached 2^32-1");
+    if (stats) {
+        memset(stats, 0, sizeof(*stats));
+        stats->iterations = R.iter;
+        stats->ms = ms;
+        stats->final_owners = R.m;
+        stats->osteal_iteration = R.osteal_iter;
+        stats->pr_last_residual = R.pr_resid;
+        unsigned long long qedges_total = 0;
+        for (int f = 0; f < c->P; f++) {
+            FragCtl fc;
+            CK(cudaSetDevice(c->fr[f].dev));
+            CK(cudaMemcpy(&fc, c->fr[f].ctl, sizeof(FragCtl), cudaMemcpyDeviceToHost));
+            stats->edges_expanded += fc.edges_done;
+            stats->edges_stolen += fc.edges_stolen;
+            stats->chunks_stolen += fc.chunks_stolen;
+            stats->chunks_total += fc.chunks_done;
+            stats->edges_frontier += fc.frontier_edges;
+            stats->remote_updates += fc.remote_updates;
+            stats->activations += fc.activations;
+            stats->vertices_frontier += fc.frontier_vertices;
+            qedges_total += fc.qedges;
+        }
+        if (alg == GUM_PR) {
+            stats->edges_frontier = qedges_total * R.iter;
+            stats->vertices_frontier *= R.iter;
+        }
+        CK(cudaSetDevice(c->dev[0]));
+    }
+    c->has_result = true;
+    return GUM_OK;
+}
+
+static gum_status gather_result(gum_ctx* c, void* dst_dev) {
+    const bool pr = c->last_alg == GUM_PR;
+    const DevCtx d = make_devctx(c, c->last_alg);
+    for (int f = 0; f < c->P; f++) {
+        CK(cudaSetDevice(c->fr[f].dev));
+        CK(launch_gather(d, f, dst_dev, pr, c->stream[c->single_device ? 0 : f], c->nsm * 4));
+    }
+    return sync_all(c);
+}
+
+gum_status gum_result(gum_ctx* c, void* out, uint64_t out_bytes) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
+    if (!c->has_result) return fail(c, GUM_ESTATE, "gum_result before a successful gum_run");
+    if (!out) return fail(c, GUM_EINVAL, "null output buffer");
+    const size_t es = c->last_alg == GUM_PR ? 8 : 4;
+    if (out_bytes < (uint64_t)c->V * es) return fail(c, GUM_EINVAL, "output buffer too small");
+    gum_status st = gather_result(c, c->d_res);
+    if (st != GUM_OK) return st;
+    CK(cudaSetDevice(c->dev[0]));
+    CK(cudaMemcpyAsync(out, c->d_res, (size_t)c->V * es, cudaMemcpyDeviceToHost, c->stream[0]));
+    CK(cudaStreamSynchronize(c->stream[0]));
+    return GUM_OK;
+}
+
+gum_status gum_result_device(gum_ctx* c, void* out, uint64_t out_bytes) {
+    if (!c) return GUM_EINVAL;
+    if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
+    if (!c->has_result) return fail(c, GUM_ESTATE, "gum_result_device before a successful gum_run");
+    if (!out) return fail(c, GUM_EINVAL, "null output buffer");
+    const size_t es = c->last_alg == GUM_PR ? 8 : 4;
+    if (out_bytes < (uint64_t)c->V * es) return fail(c, GUM_EINVAL, "output buffer too small");
+    return gather_result(c, out);
+}
+
+gum_status gum_profile(const gum_ctx* c, gum_kernel_times* out) {
+    if (!c || !out) return GUM_EINVAL;
+    if (!(c->cfg.flags & GUM_CFG_PROFILE)) return GUM_ESTATE;
+    *out = c->prof;
+    return GUM_OK;
+}
+
+gum_status gum_trace(const gum_ctx* cc, gum_iter_trace* out, uint32_t max_records, uint32_t* n_records) {
+    gum_ctx* c = const_cast<gum_ctx*>(cc);
+    if (!c || !n_records) return GUM_EINVAL;
+    *n_records = 0;
+    if (!c->has_result) return fail(c, GUM_ESTATE, "no run to trace");
+    if (!c->trace[0]) return fail(c, GUM_ESTATE, "tracing disabled (GUM_CFG_TRACE)");
+    uint32_t n = std::min<uint32_t>(std::min<uint32_t>(c->last_iters, kTraceMax), max_records);
+    if (n && out) {
+        CK(cudaSetDevice(c->dev[0]));
+        CK(cudaMemcpy(out, c->trace[0], n * sizeof(gum_iter_trace), cudaMemcpyDeviceToHost));
+        // multi-device: worker w's busy window and edge counts live in its own unit's buffer
+        if (!c->single_device) {
+            std::vector<gum_iter_trace> tmp(n);
+            for (int w = 1; w < c->P; w++) {
+                CK(cudaSetDevice(c->dev[w]));
+                CK(cudaMemcpy(tmp.data(), c->trace[w], n * sizeof(gum_iter_trace), cudaMemcpyDeviceToHost));
+                for (uint32_t i = 0; i < n; i++) {
+                    out[i].t_start[w] = tmp[i].t_start[w];
+                    out[i].t_end[w] = tmp[i].t_end[w];
+                    out[i].edges_own[w] = tmp[i].edges_own[w];
+                    out[i].edges_stolen[w] = tmp[i].edges_stolen[w];
+                }
+            }
+        }
+    }
+    *n_records = n;
+    return GUM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,215 @@
+// Setup kernels (untimed): CSR validation, seg bounds, RANDOM relabel, WCC symmetrisation.
+// SURVEY.md §8(a) rows a1/a2; PAPER.md P:55-57 (edge-cut partition), P:315/P:382 (seg, random).
+#include <cub/cub.cuh>
+#include <cuda_runtime.h>
+
+#include "kernels.h"
+
+namespace gum {
+
+__host__ __device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+// Keyed balanced Feistel network on 2h >= ceil(log2 V) bits, cycle-walked into [0, V): a bijection
+// of [0, V) (reading #17 "random partitioner = keyed Feistel relabel, then seg").
+__host__ __device__ __forceinline__ unsigned feistel(unsigned v, unsigned V, unsigned long long seed) {
+    if (V <= 2) return v;
+    int bits = 0;
+    while ((1ull << bits) < (unsigned long long)V) bits++;
+    const int h = (bits + 1) / 2;
+    const unsigned long long mask = (1ull << h) - 1;
+    const unsigned long long key = mix64(seed ^ 0x5851F42D4C957F2Dull);
+    unsigned long long x = v;
+    do {
+        unsigned long long L = x >> h, R = x & mask;
+#pragma unroll
+        for (int r = 0; r < 4; r++) {
+            unsigned long long nl = R;
+            unsigned long long nr = (L ^ mix64(R ^ key ^ ((unsigned long long)r << 56))) & mask;
+            L = nl;
+            R = nr;
+        }
+        x = (L << h) | R;
+    } while (x >= V);
+    return (unsigned)x;
+}
+
+unsigned host_feistel(unsigned v, unsigned V, unsigned long long seed) { return feistel(v, V, seed); }
+
+__global__ void k_validate(const unsigned long long* rp, const unsigned* col, unsigned V, unsigned long long E,
+                           unsigned* err) {
+    const unsigned long long tid = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    if (tid == 0) {
+        if (rp[0] != 0) atomicOr(err, 1u);
+        if (rp[V] != E) atomicOr(err, 2u);
+    }
+    for (unsigned long long i = tid; i < V; i += stride)
+        if (rp[i] > rp[i + 1]) atomicOr(err, 4u);
+    for (unsigned long long e = tid; e < E; e += stride)
+        if (col[e] >= V) atomicOr(err, 8u);
+}
+
+cudaError_t setup_validate(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                           unsigned* d_err, cudaStream_t s) {
+    k_validate<<<1184, 256, 0, s>>>(row_ptr, col, V, E, d_err);
+    return cudaGetLastError();
+}
+
+__global__ void k_seg_bounds(const unsigned long long* rp, unsigned V, unsigned long long E, int P, unsigned* b) {
+    const int g = threadIdx.x;
+    if (g > P) return;
+    if (g == 0) {
+        b[0] = 0;
+        return;
+    }
+    if (g == P) {
+        b[P] = V;
+        return;
+    }
+    const unsigned long long target = (E * (unsigned long long)g) / (unsigned long long)P;
+    unsigned lo = 0, hi = V;  // first v in [0, V] with rp[v] >= target
+    while (lo < hi) {
+        unsigned mid = lo + (hi - lo) / 2;
+        if (rp[mid] >= target)
+            hi = mid;
+        else
+            lo = mid + 1;
+    }
+    b[g] = lo;
+}
+
+cudaError_t setup_seg_bounds(const unsigned long long* row_ptr, unsigned V, unsigned long long E, int P,
+                             unsigned* d_bounds, cudaStream_t s) {
+    k_seg_bounds<<<1, 32, 0, s>>>(row_ptr, V, E, P, d_bounds);
+    return cudaGetLastError();
+}
+
+size_t setup_scan_tmp_bytes(unsigned V) {
+    size_t bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, bytes, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (int)0 + (size_t)V + 1);
+    return bytes + 256;
+}
+
+__global__ void k_inv_perm(unsigned V, unsigned long long seed, unsigned* inv) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+        inv[feistel(v, V, seed)] = v;
+}
+
+__global__ void k_new_deg(const unsigned long long* rp, const unsigned* inv, unsigned V, unsigned long long* out) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v <= V; v += gridDim.x * blockDim.x) {
+        if (v == V) {
+            out[V] = 0;
+        } else {
+            unsigned o = inv[v];
+            out[v] = rp[o + 1] - rp[o];
+        }
+    }
+}
+
+__global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
+                               unsigned V, unsigned long long seed, const unsigned long long* nrp, unsigned* ncol,
+                               unsigned* nw) {
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+    const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
+    for (unsigned long long v = warp; v < V; v += nwarps) {
+        const unsigned o = inv[v];
+        const unsigned long long s0 = rp[o], s1 = rp[o + 1], d0 = nrp[v];
+        for (unsigned long long j = lane; j < s1 - s0; j += 32) {
+            ncol[d0 + j] = feistel(col[s0 + j], V, seed);
+            if (w) nw[d0 + j] = w[s0 + j];
+        }
+    }
+}
+
+cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w, unsigned V,
+                          unsigned long long E, unsigned long long seed, unsigned* d_inv, unsigned long long* r_row_ptr,
+                          unsigned* r_col, unsigned* r_w, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    (void)E;
+    k_inv_perm<<<1184, 256, 0, s>>>(V, seed, d_inv);
+    k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
+    if (e != cudaSuccess) return e;
+    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, r_row_ptr, r_col, r_w);
+    return cudaGetLastError();
+}
+
+__global__ void k_sym_deg(const unsigned long long* rp, const unsigned* col, unsigned V, unsigned long long E,
+                          unsigned long long* srp) {
+    const unsigned long long tid = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long e = tid; e < E; e += stride) atomicAdd(srp + col[e], 1ull);
+}
+
+__global__ void k_out_deg_init(const unsigned long long* rp, unsigned V, unsigned long long* srp) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v <= V; v += gridDim.x * blockDim.x)
+        srp[v] = (v == V) ? 0 : rp[v + 1] - rp[v];
+}
+
+__global__ void k_sym_fill(const unsigned long long* rp, const unsigned* col, unsigned V,
+                           const unsigned long long* srp, unsigned* scol, unsigned long long* cursor) {
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+    const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
+    for (unsigned long long u = warp; u < V; u += nwarps) {
+        const unsigned long long s0 = rp[u], s1 = rp[u + 1], d0 = srp[u];
+        for (unsigned long long j = lane; j < s1 - s0; j += 32) {
+            const unsigned v = col[s0 + j];
+            scol[d0 + j] = v;                                  // out-neighbour
+            scol[atomicAdd(cursor + v, 1ull)] = (unsigned)u;   // u is an in-neighbour of v
+        }
+    }
+}
+
+__global__ void k_cursor_init(const unsigned long long* rp, const unsigned long long* srp, unsigned V,
+                              unsigned long long* cursor) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+        cursor[v] = srp[v] + (rp[v + 1] - rp[v]);
+}
+
+cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                             unsigned long long* s_row_ptr, unsigned* s_col, unsigned long long* cursor, void* tmp,
+                             size_t tmp_bytes, cudaStream_t s) {
+    k_out_deg_init<<<1184, 256, 0, s>>>(row_ptr, V, s_row_ptr);
+    k_sym_deg<<<1184, 256, 0, s>>>(row_ptr, col, V, E, s_row_ptr);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, s_row_ptr, s_row_ptr, (size_t)V + 1, s);
+    if (e != cudaSuccess) return e;
+    k_cursor_init<<<1184, 256, 0, s>>>(row_ptr, s_row_ptr, V, cursor);
+    k_sym_fill<<<1184, 256, 0, s>>>(row_ptr, col, V, s_row_ptr, s_col, cursor);
+    return cudaGetLastError();
+}
+
+__global__ void k_rebase(const unsigned long long* rp, unsigned b0, unsigned b1, unsigned long long* out) {
+    const unsigned long long base = rp[b0];
+    for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i <= b1 - b0; i += gridDim.x * blockDim.x)
+        out[i] = rp[b0 + i] - base;
+}
+
+cudaError_t setup_rebase_rows(const unsigned long long* row_ptr, unsigned b0, unsigned b1, unsigned long long* out,
+                              cudaStream_t s) {
+    k_rebase<<<592, 256, 0, s>>>(row_ptr, b0, b1, out);
+    return cudaGetLastError();
+}
+
+__global__ void k_count_dangling(const unsigned long long* rp, unsigned V, unsigned long long* cnt) {
+    unsigned long long c = 0;
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+        c += (rp[v + 1] == rp[v]) ? 1 : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, c);
+}
+
+cudaError_t setup_count_dangling(const unsigned long long* row_ptr, unsigned V, unsigned long long* d_count,
+                                 cudaStream_t s) {
+    k_count_dangling<<<592, 256, 0, s>>>(row_ptr, V, d_count);
+    return cudaGetLastError();
+}
+
+}  // namespace gum

@@ -1,0 +1,172 @@
+"""T2/T3 parity: the CUDA path (through the C ABI) vs the CPU oracle on the same seeded inputs.
+
+BFS/SSSP/WCC bit-exact; PR per-vertex relative error <= 1e-5 and L1 <= 1e-6.
+Results must not depend on the number of (virtual) workers, the partitioner, FSteal/OSteal or the
+frontier mode (§8(c) c-6); conservation of expanded edges is checked on every run.
+"""
+import numpy as np
+import pytest
+
+import inputs
+import oracle
+from tests.gpu_helpers import check, csr_of, gpu_run
+
+pytestmark = pytest.mark.gpu
+
+ALGS = ["bfs", "sssp", "wcc", "pr"]
+
+
+def hand_graphs():
+    n = 40
+    yield "path", inputs.from_pairs(n, [(i, i + 1) for i in range(n - 1)], np.arange(1, n)), 0
+    yield "cycle", inputs.from_pairs(n, [(i, (i + 1) % n) for i in range(n)], np.full(n, 3)), 7
+    yield "outstar", inputs.from_pairs(n, [(0, i) for i in range(1, n)], np.arange(1, n)), 0
+    yield "instar", inputs.from_pairs(n, [(i, 0) for i in range(1, n)], np.arange(1, n)), 0
+    yield "pieces", inputs.from_pairs(12, [(0, 1), (0, 1), (1, 1), (1, 2), (4, 5), (5, 4), (2, 0), (9, 10)],
+                                      [5, 1, 2, 3, 1, 1, 0, 9]), 0
+    yield "isolated", inputs.from_pairs(5, [], []), 2
+    yield "single", inputs.from_pairs(1, [(0, 0)], [4]), 0
+    yield "grid33", inputs.grid(33, seed=3), 0
+
+
+@pytest.mark.parametrize("alg", ALGS)
+def test_hand_graphs(alg):
+    for name, g, s in hand_graphs():
+        if g.w is None:
+            g.w = np.ones(g.num_edges, np.uint32)
+        for P in (1, 3):
+            check(g, alg, s, num_gpus=P)
+
+
+@pytest.mark.parametrize("alg", ALGS)
+@pytest.mark.parametrize("scale", [10, 14])
+def test_rmat_single_worker(alg, scale):
+    g = inputs.rmat(scale, 16, seed=scale)
+    s = inputs.pick_source(g, scale)
+    check(g, alg, s)
+
+
+def test_c1_bfs_sssp():
+    """BASELINE.json configs[0]: RMAT-16 EF16, BFS + SSSP, 1 GPU vs the oracle."""
+    g = inputs.make_config("C1")
+    s = inputs.pick_source(g, 1)
+    csr = csr_of(g)
+    check(g, "bfs", s, csr=csr)
+    check(g, "sssp", s, csr=csr)
+
+
+@pytest.mark.parametrize("alg", ALGS)
+@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("part", ["seg", "random"])
+def test_virtual_workers_invariance(alg, P, part):
+    g = inputs.rmat(13, 16, seed=21)
+    s = inputs.pick_source(g, 21)
+    ref = oracle.run(alg, g, s)
+    csr = csr_of(g)
+    check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P * 7)
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
+def test_forced_modes_and_stealing(alg):
+    g = inputs.rmat(13, 8, seed=5, scramble=False)  # static skew: hubs at low ids -> fragment 0 heavy
+    s = inputs.pick_source(g, 5)
+    ref = oracle.run(alg, g, s)
+    csr = csr_of(g)
+    for kw in (dict(force_mode="sparse"), dict(force_mode="dense"), dict(fsteal=False),
+               dict(chunk_edges=32, num_gpus=4), dict(num_gpus=4, osteal_threshold=1 << 30),
+               dict(num_gpus=8, osteal_threshold=1 << 30, osteal_edges_per_worker=1000),
+               dict(num_gpus=4, host_loop=True), dict(num_gpus=2, use_torch_allocator=True)):
+        kw.setdefault("num_gpus", 4)
+        out, st, _ = check(g, alg, s, csr=csr, ref=ref, **kw)
+        if kw.get("osteal_threshold"):
+            assert st.final_owners < kw["num_gpus"]
+
+
+def test_stealing_happens_and_balances():
+    g = inputs.rmat(15, 16, seed=9, scramble=False, weighted=False)
+    s = inputs.pick_source(g, 9)
+    csr = csr_of(g)
+    ref = oracle.run("bfs", g, s)
+    _, st_on, tr_on = check(g, "bfs", s, csr=csr, ref=ref, num_gpus=4, trace=True, chunk_edges=256)
+    _, st_off, tr_off = check(g, "bfs", s, csr=csr, ref=ref, num_gpus=4, trace=True, chunk_edges=256, fsteal=False)
+    assert st_on.chunks_stolen > 0 and st_off.chunks_stolen == 0
+    assert sum(r["frontier_edges"] for r in tr_on) == st_on.edges_frontier
+    for r in tr_on:
+        assert sum(r["edges_own"]) + sum(r["edges_stolen"]) == r["frontier_edges"]
+
+
+def test_sssp_unit_weights_equals_bfs():
+    g = inputs.rmat(14, 16, seed=3)
+    g.w[:] = 1
+    s = inputs.pick_source(g, 3)
+    csr = csr_of(g)
+    a, _, _ = gpu_run(g, "bfs", s, csr=csr)
+    b, _, _ = gpu_run(g, "sssp", s, csr=csr)
+    assert np.array_equal(a, b)
+
+
+def test_grid_closed_form_bfs():
+    n = 512
+    g = inputs.grid(n, unit_weights=True)
+    d, _, _ = gpu_run(g, "bfs", 0)
+    i, j = np.indices((n, n))
+    assert np.array_equal(d.reshape(n, n), (i + j).astype(np.uint32))
+
+
+def test_pr_torus_uniform():
+    g = inputs.torus(128)
+    x, st, _ = gpu_run(g, "pr", 0, num_gpus=4)
+    assert np.allclose(x, 1.0 / g.num_vertices, rtol=1e-12, atol=0)
+    assert st.iterations == 20
+
+
+def test_errors():
+    import paper_conf_icde_menggltyz23_b200 as gum
+    g = inputs.from_pairs(3, [(0, 1), (1, 2)], [0xFFFFFFF0, 0x20])
+    rp, col, w = csr_of(g)
+    with gum.Context() as ctx:
+        with pytest.raises(gum.GumError) as e:
+            ctx.run("bfs", 0)
+        assert e.value.status == gum.GUM_ESTATE
+        ctx.load_csr(rp, col, w)
+        ctx.partition()
+        with pytest.raises(gum.GumError) as e:
+            ctx.result()
+        assert e.value.status == gum.GUM_ESTATE
+        with pytest.raises(gum.GumError) as e:
+            ctx.run("bfs", 3)
+        assert e.value.status == gum.GUM_ERANGE
+        with pytest.raises(gum.GumError) as e:
+            ctx.run("sssp", 0)
+        assert e.value.status == gum.GUM_ERANGE
+        d = ctx.run("bfs", 0)
+        assert ctx.result().tolist() == [0, 1, 2]
+    with gum.Context() as ctx:
+        ctx.load_csr(rp, col, None)
+        ctx.partition()
+        with pytest.raises(gum.GumError) as e:
+            ctx.run("sssp", 0)
+        assert e.value.status == gum.GUM_EINVAL
+        with pytest.raises(gum.GumError) as e:
+            ctx.load_csr(np.array([0, 1, 3, 2], np.uint64), col, None)
+        assert e.value.status == gum.GUM_EINVAL
+        with pytest.raises(gum.GumError) as e:
+            ctx.load_csr(rp, np.array([0, 9], np.uint32), None)
+        assert e.value.status == gum.GUM_EINVAL
+
+
+def test_repeated_runs_reuse_context():
+    import paper_conf_icde_menggltyz23_b200 as gum
+    g = inputs.rmat(12, 16, seed=2)
+    rp, col, w = csr_of(g)
+    adj = oracle.Adjacency(g.num_vertices, g.src, g.dst, g.w)
+    with gum.Context(num_gpus=2) as ctx:
+        ctx.load_csr(rp, col, w)
+        ctx.partition("random", 5)
+        for s in (0, 17, 100, 4095):
+            ctx.run("sssp", s)
+            assert np.array_equal(ctx.result(), oracle.sssp(adj, s))
+            ctx.run("bfs", s)
+            assert np.array_equal(ctx.result(), oracle.bfs(adj, s))
+        ctx.run("wcc")
+        assert np.array_equal(ctx.result(), oracle.wcc(g.num_vertices, g.src, g.dst))
