@@ -1,0 +1,414 @@
+#!/usr/bin/env python
+"""GUM hot-path benchmark (driver contract).
+
+Default workload = BASELINE.json configs[1] = C2: BFS on RMAT scale 24, edge factor 16 (268M directed
+edges), 1 GPU. One "step" = one gum_run(BFS, source) to convergence (time-to-converge), sources
+cycling over a fixed seeded set. value = GTEPS (Graph500-style: sum of out-degrees of reached
+vertices / time), whole job. Inputs (1.07 GB col) are larger than L2, so no L2 flush is needed.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2]
+
+--impl reference times the CPU oracle (the tier's reference arm) on the same metric/config.
+Under torchrun (N>1) rank 0 drives all N GPUs from one process (single-process multi-device mode
+with P2P peer mappings); the other ranks only join the barriers.
+"""
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import inputs  # noqa: E402
+
+ALG_UNITS = {"bfs": "GTEPS", "sssp": "GTEPS", "wcc": "GTEPS", "pr": "GTEPS"}
+WORKLOADS = {
+    "C1": "BFS/SSSP on RMAT-16 EF16 (65,536 V, 1,048,576 E), Graph500 a,b,c=.57,.19,.19, scrambled ids, seed 1",
+    "C2": "BFS on RMAT-24 EF16 (16,777,216 V, 268,435,456 E), Graph500 a,b,c=.57,.19,.19, scrambled ids, seed 2",
+    "C3": "SSSP on 8192x8192 4-neighbour grid (67,108,864 V, 268,402,688 E), w in [1,255], source 0, seed 3",
+    "C4": "WCC on RMAT-26 EF16 (67,108,864 V, 1,073,741,824 E, symmetrised 2^31 entries), seed 4",
+    "C5": "PR (20 iterations, d=0.85) on RMAT-25 EF44 (33,554,432 V, 1,476,395,008 E), seed 5",
+}
+DEFAULT_ALG = {"C1": "bfs", "C2": "bfs", "C3": "sssp", "C4": "wcc", "C5": "pr"}
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def pick_sources(g, seed, n):
+    outdeg = np.bincount(g.src, minlength=g.num_vertices)
+    lib = inputs._load()
+    out, j = [], 0
+    while len(out) < n and j < 100000:
+        v = int(lib.gen_splitmix_seq(seed, j) % g.num_vertices)
+        if outdeg[v] > 0 and v not in out:
+            out.append(v)
+        j += 1
+    return out, outdeg
+
+
+def traversed_edges(alg, result, outdeg, E):
+    """GTEPS numerator: BFS/SSSP sum of out-degrees of reached vertices;
+    WCC symmetric entries 2E; PR 20*E (per iteration all edges)."""
+    if alg in ("bfs", "sssp"):
+        return int(outdeg[result != 0xFFFFFFFF].sum())
+    if alg == "wcc":
+        return 2 * E
+    return None
+
+
+class ClockSampler:
+    """Samples SM clock and clock-event reasons with NVML during the timed region."""
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting"}
+
+    def __init__(self, dev=0):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:  # noqa: BLE001 - clocks are reported as unavailable
+            self.max_mhz = None
+
+    def _run(self):
+        nv = self.nv
+        get_r = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            nv.nvmlDeviceGetCurrentClocksThrottleReasons
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = get_r(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def load_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        return float(json.load(open(p))["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:  # noqa: BLE001
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def load_ncu_traffic(config, alg):
+    p = os.path.join(ROOT, "profiles", "ncu_advance_traffic.json")
+    try:
+        d = json.load(open(p))
+        return d.get(f"{config}_{alg}")
+    except Exception:  # noqa: BLE001
+        return None
+
+
+def advance_bytes(alg, st):
+    """Algorithmic bytes of the advance kernel: per expanded edge col 4 B +
+    state 4 B (+ w 4 B for SSSP; PR: acc 8 B), per frontier vertex 24 B (queue id 4, prefix 8, col base
+    8, own state 4; PR: x 8 instead of state 4 -> 28 B), per activation 8 B (bitmap 4 + list 4)."""
+    per_edge = {"bfs": 8, "sssp": 12, "wcc": 8, "pr": 12}[alg]
+    per_vertex = 28 if alg == "pr" else 24
+    return per_edge * st.edges_expanded + per_vertex * st.vertices_frontier + 8 * st.activations
+
+
+def launches_per_run(alg, st):
+    init = {"bfs": 3, "sssp": 3, "wcc": 2, "pr": 3}[alg]
+    if alg == "pr":
+        return init + 3 * st.iterations + 1
+    return init + 3 * (st.iterations + 1)
+
+
+def oracle_bench(g, alg, sources, outdeg, budget_s, reps=None):
+    """Times the oracle as it stands (single-threaded by construction). Returns dict."""
+    import oracle
+    t0 = time.perf_counter()
+    adj = None
+    if alg in ("bfs", "sssp"):
+        adj = oracle.Adjacency(g.num_vertices, g.src, g.dst, g.w if alg == "sssp" else None)
+    t_build = time.perf_counter() - t0
+    solved, edges, t_solve, outs = 0, 0, 0.0, {}
+    i = 0
+    while True:
+        s = sources[i % len(sources)]
+        t1 = time.perf_counter()
+        if alg == "bfs":
+            r = oracle.bfs(adj, s)
+        elif alg == "sssp":
+            r = oracle.sssp(adj, s)
+        elif alg == "wcc":
+            r = oracle.wcc(g.num_vertices, g.src, g.dst)
+        else:
+            r = oracle.pagerank(g.num_vertices, g.src, g.dst, 20, 0.85)
+        dt = time.perf_counter() - t1
+        t_solve += dt
+        te = traversed_edges(alg, r, outdeg, g.num_edges) if alg != "pr" else 20 * g.num_edges
+        edges += te
+        outs[s] = r
+        solved += 1
+        i += 1
+        if reps is not None and solved >= reps:
+            break
+        if reps is None and (t_solve >= budget_s or (alg in ("wcc", "pr") and solved >= 1)):
+            break
+    return dict(value=edges / t_solve / 1e9, solves=solved, solve_s=t_solve, build_s=t_build, outs=outs)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=env_int("WORLD_SIZE", 1))
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", choices=list(WORKLOADS))
+    ap.add_argument("--alg", default=None)
+    ap.add_argument("--sources", type=int, default=8)
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--part", default="seg")
+    ap.add_argument("--fsteal", type=int, default=1)
+    args = ap.parse_args()
+    alg = args.alg or DEFAULT_ALG[args.config]
+    rank = env_int("RANK", 0)
+    world = env_int("WORLD_SIZE", 1)
+    N = args.gpus
+
+    pg = False
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+        pg = True
+
+    def barrier():
+        if pg:
+            import torch.distributed as dist
+            dist.barrier()
+
+    metric = f"{alg.upper()} GTEPS (time-to-converge per source; {args.config})"
+    cfg_desc = {"workload": f"{args.config}: {WORKLOADS[args.config]}", "alg": alg, "partition": args.part,
+                "l2": "inputs larger than L2 (col array > 126 MB); no flush"}
+
+    if rank != 0:
+        # rank 0 drives every GPU of the job (single-process multi-device); others only synchronise
+        barrier()
+        barrier()
+        return
+
+    t_gen = time.perf_counter()
+    g = inputs.make_config(args.config, weighted=(alg == "sssp"))
+    sources, outdeg = pick_sources(g, {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}[args.config], args.sources)
+    if args.config == "C3":
+        sources = [0]
+    t_gen = time.perf_counter() - t_gen
+
+    if args.impl == "reference":
+        barrier()
+        steps_total = args.warmup + args.steps
+        ob = oracle_bench(g, alg, sources, outdeg, 0, reps=max(1, args.steps))
+        line = {"impl": "reference", "metric": metric, "value": ob["value"], "unit": "GTEPS", "n_gpus": N,
+                "steps": args.steps, "warmup": 0, "ms_per_step": ob["solve_s"] / ob["solves"] * 1e3,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+                "data": "synthetic", "config": cfg_desc,
+                "cpu_baseline": {"kind": "oracle", "value": ob["value"], "unit": "GTEPS", "cores": 1,
+                                 "sample": f"{ob['solves']} oracle {alg} solves on the full {args.config} graph "
+                                           f"(adjacency build {ob['build_s']:.1f}s excluded); warm-up skipped "
+                                           f"(the oracle has no warm state), requested {steps_total}"},
+                "e2e": {"value": ob["value"], "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        barrier()
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+
+    import paper_conf_icde_menggltyz23_b200 as gum
+
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    t_csr = time.perf_counter()
+    row_ptr, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if alg == "sssp" else None)
+    t_csr = time.perf_counter() - t_csr
+    E = g.num_edges
+    dev_ids = list(range(N)) if N > 1 else None
+    ctx_kw = dict(num_gpus=N, device_ids=dev_ids, fsteal=bool(args.fsteal))
+
+    # ---------------------------------------------------------------- device-resident timed region
+    ctx = gum.Context(streams=[stream] * N if N == 1 else None, **ctx_kw)
+    ctx.load_csr(row_ptr, col, w)
+    ctx.partition(args.part, 1)
+    ctx.prepare(alg)
+    edges_of, iters_of = {}, {}
+    for i in range(max(args.warmup, len(sources) if alg in ("bfs", "sssp") else args.warmup)):
+        s = sources[i % len(sources)]
+        st = ctx.run(alg, s)
+        if s not in edges_of:
+            r = ctx.result()
+            edges_of[s] = traversed_edges(alg, r, outdeg, E) if alg != "pr" else 20 * E
+            iters_of[s] = st
+    barrier()
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    total_edges, launches = 0, 0
+    sampler = ClockSampler(0)
+    with sampler:
+        with torch.cuda.stream(stream):
+            ev0.record(stream)
+            for i in range(args.steps):
+                s = sources[i % len(sources)]
+                st = ctx.run(alg, s)
+                total_edges += edges_of[s]
+                launches += launches_per_run(alg, st)
+            ev1.record(stream)
+        torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    barrier()
+    value = total_edges / (ms / 1e3) / 1e9
+    ms_per_step = ms / args.steps
+    ctx.close()
+
+    # ---------------------------------------------------------------- roofline of the advance kernel
+    peak, peak_src = load_peak()
+    pctx = gum.Context(profile=True, **ctx_kw) if N == 1 else None
+    roof = None
+    share = None
+    if pctx is not None:
+        pctx.load_csr(row_ptr, col, w)
+        pctx.partition(args.part, 1)
+        pctx.prepare(alg)
+        pctx.run(alg, sources[0])  # warm
+        adv_ms, adv_bytes, adv_launches, all_ms = 0.0, 0, 0, 0.0
+        for s in sources[: min(len(sources), 4)]:
+            st = pctx.run(alg, s)
+            k = pctx.profile()
+            adv_ms += k["advance_ms"]
+            adv_launches += k["advance_launches"]
+            all_ms += k["advance_ms"] + k["filter_ms"] + k["control_ms"] + k["finalize_ms"] + k["init_ms"]
+            adv_bytes += advance_bytes(alg, st)
+        pctx.close()
+        achieved = adv_bytes / (adv_ms / 1e3) / 1e9
+        traffic = load_ncu_traffic(args.config, alg)
+        roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "kernel": "k_advance", "peak_source": peak_src,
+                "bytes_per_launch": adv_bytes / max(adv_launches, 1),
+                "avg_launch_ms": adv_ms / max(adv_launches, 1),
+                "how": "CUDA events around every k_advance launch on its stream (profile pass, host loop)"}
+        share = adv_ms / all_ms if all_ms else None
+
+    # ---------------------------------------------------------------- end to end through the C ABI
+    e2e = None
+    if not args.no_e2e and N == 1:
+        rp_t = torch.from_numpy(row_ptr.view(np.int64)).pin_memory()
+        col_t = torch.from_numpy(col.view(np.int32)).pin_memory()
+        w_t = torch.from_numpy(w.view(np.int32)).pin_memory() if w is not None else None
+        out_t = torch.empty(g.num_vertices * (8 if alg == "pr" else 4), dtype=torch.uint8).pin_memory()
+        ectx = gum.Context(streams=[stream], use_torch_allocator=True, **ctx_kw)
+        h2d = rp_t.numel() * 8 + col_t.numel() * 4 + (w_t.numel() * 4 if w_t is not None else 0)
+        d2h = out_t.numel()
+        K2 = max(3, min(args.steps, 10))
+
+        def e2e_step(s):
+            ectx.load_csr(rp_t, col_t, w_t)
+            ectx.partition(args.part, 1)
+            ectx.run(alg, s)
+            ectx.result(out_t)
+
+        for i in range(2):
+            e2e_step(sources[i % len(sources)])
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tot = 0
+        with torch.cuda.stream(stream):
+            a.record(stream)
+            for i in range(K2):
+                s = sources[i % len(sources)]
+                e2e_step(s)
+                tot += edges_of[s]
+            b.record(stream)
+        torch.cuda.synchronize()
+        e_ms = a.elapsed_time(b)
+        e2e = {"value": tot / (e_ms / 1e3) / 1e9, "unit": "GTEPS", "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "steps": K2, "ms_per_step": e_ms / K2,
+               "path": "gum_load_csr(pinned host CSR) + gum_partition + gum_run + gum_result(pinned host)"}
+        ectx.close()
+
+    # ---------------------------------------------------------------- CPU oracle baseline (+ parity)
+    cpu = None
+    parity = None
+    if not args.no_cpu:
+        ob = oracle_bench(g, alg, sources, outdeg, args.cpu_budget)
+        ncpu = len(os.sched_getaffinity(0))
+        cpu = {"value": round(ob["value"], 4), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+               "sample": f"{ob['solves']} single-threaded oracle {alg} solve(s) on the full {args.config} graph "
+                         f"({ob['solve_s']:.1f}s solve; adjacency build {ob['build_s']:.1f}s excluded; "
+                         f"host has {ncpu} cores)"}
+        # full-size parity on the sampled sources (bit-exact for BFS/SSSP/WCC)
+        vctx = gum.Context(**ctx_kw)
+        vctx.load_csr(row_ptr, col, w)
+        vctx.partition(args.part, 1)
+        ok = True
+        for s, ref in ob["outs"].items():
+            vctx.run(alg, s)
+            out = vctx.result()
+            if alg == "pr":
+                ok &= bool(np.max(np.abs(out - ref) / ref) <= 1e-5 and np.abs(out - ref).sum() <= 1e-6)
+            else:
+                ok &= bool(np.array_equal(out, ref))
+        vctx.close()
+        parity = {"checked_sources": len(ob["outs"]), "exact": ok}
+
+    st0 = iters_of.get(sources[0])
+    line = {
+        "metric": metric, "value": round(value, 3), "unit": "GTEPS", "n_gpus": N, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32" if alg != "pr" else "f64", "data": "synthetic",
+        "config": cfg_desc, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+        "clocks": sampler.summary(),
+        "detail": {"time_to_converge_ms": round(ms_per_step, 4), "sources": len(sources),
+                   "iterations_first_source": st0.iterations if st0 else None,
+                   "edges_traversed_first_source": edges_of.get(sources[0]),
+                   "advance_share_of_step": share, "parity_full_size": parity,
+                   "setup_s": {"generate": round(t_gen, 2), "build_csr": round(t_csr, 2)}},
+    }
+    barrier()
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    try:
+        main()
+    except Exception as e:  # noqa: BLE001 - the driver needs one JSON line even on failure
+        if env_int("RANK", 0) == 0:
+            print(json.dumps({"error": f"{type(e).__name__}: {e}"}), flush=True)
+        raise

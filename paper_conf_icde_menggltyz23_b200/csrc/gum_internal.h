@@ -13,8 +13,8 @@ constexpr int kMaxW = GUM_MAX_WORKERS;
 constexpr int kThreads = 256;          // CTA size of advance / filter
 constexpr int kTileMax = 2048;         // max edges per claimable chunk (smem sized for it)
 constexpr int kEdgesPerThread = kTileMax / kThreads;
-constexpr int kFilterWordsPerThread = 4;                          // dense filter: bitmap words per thread
-constexpr int kFilterWordsPerPart = kThreads * kFilterWordsPerThread;  // 1024 words = 32768 vertices
+constexpr int kDenseWordsPerWarp = 32;                            // dense filter: bitmap words per warp
+constexpr int kDenseWordsPerPart = (kThreads / 32) * kDenseWordsPerWarp;  // 256 words = 8192 vertices
 constexpr int kFilterAppPerThread = 8;                            // sparse filter: list entries per thread
 constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;
@@ -50,6 +50,8 @@ struct alignas(128) RunCtl {
     unsigned int done;
     unsigned int m;           // active owners (OSteal): workers {0..m-1}
     unsigned int steal_ok;    // FSteal gate for the current advance
+    unsigned int next_dense;  // the current advance only sets bitmap bits (next filter scans the bitmap)
+                              // instead of appending to the activation list
     unsigned int owner[kMaxW];// fragment -> worker (P_OSteal vector O)
     unsigned int err;
     unsigned int osteal_iter;
@@ -76,6 +78,7 @@ struct FragPtrs {
     double* acc;                        // PR [V_f]
     const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
     unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
+    unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
     unsigned int* app;                  // [V_f] activation list (sparse next frontier)
     unsigned int* q_v;                  // [V_f] frontier queue (local ids, out-degree > 0)
     unsigned long long* q_off;          // [V_f + 1] exclusive prefix of out-degrees over the queue

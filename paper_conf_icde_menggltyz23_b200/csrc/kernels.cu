@@ -15,6 +15,7 @@
 //   k_pr_finalize a11  x' = (1-d)/V + d(acc + D/V), dangling mass and residual (PR, fp64).
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "gum_internal.h"
 #include "kernels.h"
@@ -78,6 +79,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
                 wv = rem >= 32 ? 0xFFFFFFFFu : ((1u << rem) - 1u);
             }
             F.bm[i] = wv;
+            if (ALG == ALG_BFS) F.vis[i] = 0u;
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -101,13 +103,15 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
 __global__ void k_init_source(const __grid_constant__ DevCtx c, int f, unsigned ls) {
     const FragPtrs& F = c.f[f];
     F.state[ls] = 0;
+    if (F.vis) F.vis[ls >> 5] |= 1u << (ls & 31);
     F.bm[ls >> 5] |= 1u << (ls & 31);
     F.app[0] = ls;
     F.ctl->app_cnt = 1;
 }
 
-__global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, gum_iter_trace* trace) {
+__global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, unsigned next_dense0) {
     RunCtl* rc = c.rctl[w0];
+    rc->next_dense = next_dense0;
     rc->iter = 0;
     rc->done = 0;
     rc->m = c.P;
@@ -167,7 +171,26 @@ __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, u
     for (; t * chunk < off + deg; t++) F.tile[t] = (unsigned)pos;
 }
 
-__global__ void __launch_bounds__(kThreads) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+// Dense partitions: 8 warps x 32 bitmap words (8192 vertices); a warp walks its words i-major,
+// lane-minor (vertex = word*32 + lane), so row_ptr reads are coalesced and the queue is sorted.
+
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+}
+__device__ __forceinline__ unsigned long long warp_excl_scan_u64(unsigned long long x, unsigned long long& total) {
+    unsigned long long inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane_id() >= (unsigned)o) inc += y;
+    }
+    total = __shfl_sync(0xffffffffu, inc, 31);
+    return inc - x;
+}
+
+__global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
     if (vload(&rc->done)) return;
     const int f = blockIdx.y;
@@ -175,16 +198,18 @@ __global__ void __launch_bounds__(kThreads) k_filter(const __grid_constant__ Dev
     if ((int)o < w0 || (int)o >= w0 + nw) return;
     const FragPtrs& F = c.f[f];
     FragCtl* ct = F.ctl;
-    const unsigned app_cnt = vload(&ct->app_cnt);
-    const bool dense = c.force_mode == 2 || (c.force_mode == 0 && (unsigned long long)app_cnt * c.dense_div > F.V);
+    // the advance that produced these activations either appended them (sparse) or only set bits
+    const bool dense = vload(&rc->next_dense) != 0;
+    const unsigned app_cnt = dense ? 0u : vload(&ct->app_cnt);
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
-    const unsigned per = dense ? kFilterWordsPerPart : kFilterAppPerPart;
+    const unsigned per = dense ? kDenseWordsPerPart : kFilterAppPerPart;
     unsigned long long n_parts = (n_items + per - 1) / per;
     if (n_parts == 0) n_parts = 1;
     const unsigned long long epoch = rc->epoch;
     const unsigned chunk = c.chunk;
     LBSlot* slots = c.lb[f];
+    const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
 
     __shared__ unsigned s_part;
     __shared__ Pair s_warp[kThreads / 32];
@@ -197,133 +222,179 @@ __global__ void __launch_bounds__(kThreads) k_filter(const __grid_constant__ Dev
         __syncthreads();
         if (p >= n_parts) break;
 
-        // ---- phase 1: gather items, count vertices with out-degree > 0 and their degrees
-        unsigned items[8];
-        int nit = 0;
+        // ---- phase 1: count vertices with out-degree > 0 and their degrees
         Pair mine{0, 0};
+        unsigned myword = 0;
+        unsigned items[kFilterAppPerThread];
+        const unsigned wbase = p * kDenseWordsPerPart + wid * kDenseWordsPerWarp;
+        const unsigned long long ibase =
+            (unsigned long long)p * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
         if (dense) {
-            const unsigned wbase = p * kFilterWordsPerPart + threadIdx.x * kFilterWordsPerThread;
-            if (wbase + kFilterWordsPerThread <= nwords) {
-                uint4 q = *reinterpret_cast<const uint4*>(F.bm + wbase);
-                items[0] = q.x; items[1] = q.y; items[2] = q.z; items[3] = q.w;
-                *reinterpret_cast<uint4*>(F.bm + wbase) = make_uint4(0, 0, 0, 0);
-            } else {
+            if (wbase + lane < nwords) {
+                myword = F.bm[wbase + lane];
+                if (myword) F.bm[wbase + lane] = 0u;
+            }
+            unsigned long long wc = 0, wd = 0;
 #pragma unroll
-                for (int j = 0; j < 4; j++) {
-                    items[j] = (wbase + j < nwords) ? F.bm[wbase + j] : 0u;
-                    if (wbase + j < nwords) F.bm[wbase + j] = 0u;
+            for (int i0 = 0; i0 < kDenseWordsPerWarp; i0 += 8) {
+                unsigned long long d[8];
+#pragma unroll
+                for (int k = 0; k < 8; k++) {
+                    const unsigned wv = __shfl_sync(0xffffffffu, myword, i0 + k);
+                    const unsigned v = (wbase + i0 + k) * 32 + lane;
+                    d[k] = 0;
+                    if ((wv >> lane) & 1u) d[k] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
+                }
+#pragma unroll
+                for (int k = 0; k < 8; k++) {
+                    wc += d[k] ? 1 : 0;
+                    wd += d[k];
                 }
             }
-            nit = 4;
-#pragma unroll
-            for (int j = 0; j < 4; j++) {
-                unsigned wv = items[j];
-                while (wv) {
-                    unsigned b = __ffs(wv) - 1;
-                    wv &= wv - 1;
-                    unsigned v = (wbase + j) * 32 + b;
-                    unsigned long long d = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
-                    if (d) {
-                        mine.cnt++;
-                        mine.deg += d;
-                    }
-                }
-            }
+            wc = warp_sum_u64(wc);
+            wd = warp_sum_u64(wd);
+            if (lane == 0) mine = Pair{wc, wd};  // block scan over warps (lane 0 carries the warp)
         } else {
-            const unsigned long long ibase = (unsigned long long)p * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
+            unsigned long long d[kFilterAppPerThread];
 #pragma unroll
-            for (int j = 0; j < 8; j++) {
+            for (int j = 0; j < kFilterAppPerThread; j++) {
+                d[j] = 0;
+                items[j] = 0xFFFFFFFFu;
                 if (ibase + j < app_cnt) {
-                    unsigned v = F.app[ibase + j];
+                    const unsigned v = F.app[ibase + j];
                     items[j] = v;
-                    nit = j + 1;
                     F.bm[v >> 5] = 0u;  // every set bit belongs to a listed vertex: clearing whole words is exact
-                    unsigned long long d = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
-                    if (d) {
-                        mine.cnt++;
-                        mine.deg += d;
-                    }
+                    d[j] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
                 }
+            }
+#pragma unroll
+            for (int j = 0; j < kFilterAppPerThread; j++) {
+                mine.cnt += d[j] ? 1 : 0;
+                mine.deg += d[j];
             }
         }
         Pair agg;
         Pair texcl = block_excl_scan(mine, s_warp, agg);
 
-        // ---- decoupled look-back (single thread) over partitions of this fragment
-        if (threadIdx.x == 0) {
+        // ---- decoupled look-back over partitions of this fragment (warp 0, 32 predecessors per step)
+        if (wid == 0) {
             LBSlot* S = slots + p;
+            const unsigned long long AGG = epoch * 4 + 1, INC = epoch * 4 + 2;
             Pair excl{0, 0};
-            if (p == 0) {
-                S->inc_cnt = agg.cnt;
-                S->inc_deg = agg.deg;
-                st_release_u64(&S->flag, epoch * 4 + 2);
-            } else {
-                S->agg_cnt = agg.cnt;
-                S->agg_deg = agg.deg;
-                st_release_u64(&S->flag, epoch * 4 + 1);
-                long long j = (long long)p - 1;
-                while (j >= 0) {
-                    unsigned long long fl = ld_acquire_u64(&slots[j].flag);
-                    if (fl < epoch * 4 + 1) continue;  // predecessor not published yet
-                    if (fl == epoch * 4 + 2) {
-                        excl.cnt += __ldcg(&slots[j].inc_cnt);
-                        excl.deg += __ldcg(&slots[j].inc_deg);
-                        break;
-                    }
-                    excl.cnt += __ldcg(&slots[j].agg_cnt);
-                    excl.deg += __ldcg(&slots[j].agg_deg);
-                    j--;
+            if (lane == 0) {
+                if (p == 0) {
+                    S->inc_cnt = agg.cnt;
+                    S->inc_deg = agg.deg;
+                    st_release_u64(&S->flag, INC);
+                } else {
+                    S->agg_cnt = agg.cnt;
+                    S->agg_deg = agg.deg;
+                    st_release_u64(&S->flag, AGG);
                 }
-                S->inc_cnt = excl.cnt + agg.cnt;
-                S->inc_deg = excl.deg + agg.deg;
-                st_release_u64(&S->flag, epoch * 4 + 2);
             }
-            s_excl = excl;
-            if (p == n_parts - 1) {
-                const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
-                F.q_off[tc] = td;
-                ct->qlen = tc;
-                ct->qedges = td;
-                ct->ntiles = (td + chunk - 1) / chunk;
-                ct->claim = 0;
-                ct->app_cnt = 0;
-                ct->dense = dense ? 1u : 0u;
-                ct->frontier_edges += td;
-                ct->frontier_vertices += tc;
+            __syncwarp();
+            if (p > 0) {
+                long long j = (long long)p - 1 - lane;  // lane 0 = nearest predecessor
+                for (;;) {
+                    unsigned long long fl = INC;
+                    if (j >= 0) {
+                        do {
+                            fl = ld_acquire_u64(&slots[j].flag);
+                        } while (fl < AGG);
+                    }
+                    const bool is_inc = fl >= INC;
+                    const unsigned incmask = __ballot_sync(0xffffffffu, is_inc);
+                    const int first = incmask ? __ffs(incmask) - 1 : 32;  // nearest inclusive in window
+                    unsigned long long vc = 0, vd = 0;
+                    if ((int)lane <= first && j >= 0) {
+                        if ((int)lane == first) {
+                            vc = __ldcg(&slots[j].inc_cnt);
+                            vd = __ldcg(&slots[j].inc_deg);
+                        } else {
+                            vc = __ldcg(&slots[j].agg_cnt);
+                            vd = __ldcg(&slots[j].agg_deg);
+                        }
+                    }
+                    excl.cnt += warp_sum_u64(vc);
+                    excl.deg += warp_sum_u64(vd);
+                    if (incmask) break;
+                    j -= 32;
+                }
+                if (lane == 0) {
+                    S->inc_cnt = excl.cnt + agg.cnt;
+                    S->inc_deg = excl.deg + agg.deg;
+                    st_release_u64(&S->flag, INC);
+                }
+            }
+            if (lane == 0) {
+                s_excl = excl;
+                if (p == n_parts - 1) {
+                    const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
+                    F.q_off[tc] = td;
+                    ct->qlen = tc;
+                    ct->qedges = td;
+                    ct->ntiles = (td + chunk - 1) / chunk;
+                    ct->claim = 0;
+                    ct->app_cnt = 0;
+                    ct->dense = dense ? 1u : 0u;
+                    ct->frontier_edges += td;
+                    ct->frontier_vertices += tc;
+                }
             }
         }
         __syncthreads();
-        unsigned long long pos = s_excl.cnt + texcl.cnt;
-        unsigned long long off = s_excl.deg + texcl.deg;
 
         // ---- phase 2: write queue entries, degree prefix and chunk table
         if (dense) {
-            const unsigned wbase = p * kFilterWordsPerPart + threadIdx.x * kFilterWordsPerThread;
+            unsigned long long pos = s_excl.cnt + __shfl_sync(0xffffffffu, texcl.cnt, 0);
+            unsigned long long off = s_excl.deg + __shfl_sync(0xffffffffu, texcl.deg, 0);
 #pragma unroll
-            for (int j = 0; j < 4; j++) {
-                unsigned wv = items[j];
-                while (wv) {
-                    unsigned b = __ffs(wv) - 1;
-                    wv &= wv - 1;
-                    unsigned v = (wbase + j) * 32 + b;
-                    unsigned long long rp = __ldg(F.row_ptr + v);
-                    unsigned long long d = __ldg(F.row_ptr + v + 1) - rp;
-                    if (d) {
-                        emit_vertex(F, chunk, v, rp, d, pos, off);
-                        pos++;
-                        off += d;
+            for (int i0 = 0; i0 < kDenseWordsPerWarp; i0 += 8) {
+                unsigned long long rp[8], d[8];
+#pragma unroll
+                for (int k = 0; k < 8; k++) {
+                    const unsigned wv = __shfl_sync(0xffffffffu, myword, i0 + k);
+                    const unsigned v = (wbase + i0 + k) * 32 + lane;
+                    d[k] = 0;
+                    rp[k] = 0;
+                    if ((wv >> lane) & 1u) {
+                        rp[k] = __ldg(F.row_ptr + v);
+                        d[k] = __ldg(F.row_ptr + v + 1) - rp[k];
                     }
+                }
+#pragma unroll
+                for (int k = 0; k < 8; k++) {
+                    const unsigned bal = __ballot_sync(0xffffffffu, d[k] != 0);
+                    if (bal == 0) continue;  // warp-uniform
+                    unsigned long long dtot;
+                    const unsigned long long dex = warp_excl_scan_u64(d[k], dtot);
+                    if (d[k]) {
+                        const unsigned v = (wbase + i0 + k) * 32 + lane;
+                        emit_vertex(F, chunk, v, rp[k], d[k], pos + __popc(bal & lanemask_lt()), off + dex);
+                    }
+                    pos += __popc(bal);
+                    off += dtot;
                 }
             }
         } else {
-            for (int j = 0; j < nit; j++) {
-                unsigned v = items[j];
-                unsigned long long rp = __ldg(F.row_ptr + v);
-                unsigned long long d = __ldg(F.row_ptr + v + 1) - rp;
-                if (d) {
-                    emit_vertex(F, chunk, v, rp, d, pos, off);
+            unsigned long long pos = s_excl.cnt + texcl.cnt;
+            unsigned long long off = s_excl.deg + texcl.deg;
+            unsigned long long rp[kFilterAppPerThread], d[kFilterAppPerThread];
+#pragma unroll
+            for (int j = 0; j < kFilterAppPerThread; j++) {
+                rp[j] = 0;
+                d[j] = 0;
+                if (items[j] != 0xFFFFFFFFu) {
+                    rp[j] = __ldg(F.row_ptr + items[j]);
+                    d[j] = __ldg(F.row_ptr + items[j] + 1) - rp[j];
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < kFilterAppPerThread; j++) {
+                if (d[j]) {
+                    emit_vertex(F, chunk, items[j], rp[j], d[j], pos, off);
                     pos++;
-                    off += d;
+                    off += d[j];
                 }
             }
         }
@@ -401,6 +472,12 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             mn = l[i] < mn ? l[i] : mn;
         }
         rc->steal_ok = (c.fsteal && m > 1 && mx >= c.t1 && mx - mn >= c.t2) ? 1u : 0u;
+        // frontier density switch: expanding more than V/dense_div edges is expected to activate a
+        // dense next frontier -> the advance only sets bitmap bits (fire-and-forget) and the next
+        // filter scans the bitmap; otherwise activations are deduplicated and appended to a list.
+        rc->next_dense = c.force_mode == 2 ? 1u
+                         : c.force_mode == 1 ? 0u
+                         : (total_edges * c.dense_div > (unsigned long long)c.num_vertices ? 1u : 0u);
         gum_iter_trace* tr = c.trace[w0];
         if (tr && k < (unsigned)kTraceMax) {
             gum_iter_trace* r = tr + k;
@@ -437,12 +514,44 @@ struct ValT<ALG_PR> {
     typedef double T;
 };
 
+// Warp-aggregated append of this thread's activations (bit j of need: slot j) to the owner
+// fragments' activation lists: one reservation atomic per warp and target fragment.
+template <bool MULTI>
+__device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned need, const unsigned char* tfv,
+                                                       const unsigned* lvv) {
+    unsigned done = 0;
+    const int nfrag = MULTI ? c.P : 1;
+    for (int g = 0; g < nfrag; g++) {
+        unsigned mine = 0;
+#pragma unroll
+        for (int j = 0; j < kEdgesPerThread; j++) mine += ((need >> j) & 1u) && tfv[j] == g ? 1u : 0u;
+        unsigned inc = mine;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned x = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane_id() >= (unsigned)o) inc += x;
+        }
+        const unsigned total = __shfl_sync(0xffffffffu, inc, 31);
+        if (total == 0) continue;  // warp-uniform
+        unsigned basepos = 0;
+        if (lane_id() == 31) basepos = atomicAdd(&c.f[g].ctl->app_cnt, total);
+        basepos = __shfl_sync(0xffffffffu, basepos, 31);
+        unsigned pos = basepos + inc - mine;
+        unsigned* app = c.f[g].app;
+#pragma unroll
+        for (int j = 0; j < kEdgesPerThread; j++)
+            if (((need >> j) & 1u) && tfv[j] == g) app[pos++] = lvv[j];
+        done += mine;
+    }
+    return done;
+}
+
 template <int ALG, bool MULTI>
-__global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
+__global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
     __shared__ long long s_base[kTileMax + 1];
-    __shared__ VT s_val[kTileMax + 1];
-    __shared__ unsigned short s_head[kTileMax];
+    __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
+    __shared__ unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
     __shared__ unsigned s_wmax[kThreads / 32];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
@@ -457,6 +566,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
     if ((unsigned)w >= m) return;  // evicted by OSteal: this worker's GPU only serves as memory
     const unsigned k = rc->iter - 1;
     const bool steal = rc->steal_ok != 0;
+    const bool next_dense = rc->next_dense != 0;
     const unsigned long long t0 = globaltimer();
     if (threadIdx.x < (unsigned)c.P) {
         FragCtl* ct = c.f[threadIdx.x].ctl;
@@ -467,26 +577,38 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
     }
     __syncthreads();
     const unsigned CH = c.chunk;
+    for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kThreads) s_head[e] = 0;
+    unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0;
 
+    // next own chunk claimed one tile ahead (its atomic overlaps the current chunk's expansion)
+    int pf_f = -1;
+    unsigned long long pf_t = 0;
     for (;;) {
         if (threadIdx.x == 0) {
             int f = -1;
             unsigned long long t = 0;
             int stolen = 0;
-            while (own_cursor < c.P) {
-                int g = (w + own_cursor) % c.P;
-                if (s_owner[g] == (unsigned)w) {
-                    unsigned long long tt = atomicAdd(&c.f[g].ctl->claim, 1ull);
-                    if (tt < s_ntiles[g]) {
-                        f = g;
-                        t = tt;
-                        break;
+            if (pf_f >= 0 && pf_t < s_ntiles[pf_f]) {
+                f = pf_f;
+                t = pf_t;
+            } else {
+                if (pf_f >= 0) own_cursor++;  // prefetched claim overflowed: that queue is drained
+                while (own_cursor < c.P) {
+                    int g = (w + own_cursor) % c.P;
+                    if (s_owner[g] == (unsigned)w) {
+                        unsigned long long tt = atomicAdd(&c.f[g].ctl->claim, 1ull);
+                        if (tt < s_ntiles[g]) {
+                            f = g;
+                            t = tt;
+                            break;
+                        }
                     }
+                    own_cursor++;
                 }
-                own_cursor++;
             }
+            pf_f = -1;
             if (f < 0 && steal) {
                 // FSteal: claim a chunk of the active owner queue with the most remaining chunks
                 for (;;) {
@@ -514,6 +636,10 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
             s_f = f;
             s_t = t;
             s_stolen = stolen;
+            if (f >= 0 && !stolen) {
+                pf_f = f;
+                pf_t = atomicAdd(&c.f[f].ctl->claim, 1ull);
+            }
         }
         __syncthreads();
         const int f = s_f;
@@ -529,21 +655,21 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
         const unsigned nv = i1 - i0 + 1;
 
         // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
-        for (unsigned e = threadIdx.x; e < tlen; e += kThreads) s_head[e] = 0;
-        __syncthreads();
+        seq++;
         for (unsigned kk = threadIdx.x; kk < nv; kk += kThreads) {
             const unsigned i = i0 + kk;
-            const unsigned u = __ldg(F.q_v + i);
-            const unsigned long long off = __ldg(F.q_off + i);
-            s_base[kk] = __ldg(F.q_base + i);
+            const unsigned long long off = __ldcs(F.q_off + i);
+            s_base[kk] = __ldcs(F.q_base + i);
             if (ALG == ALG_PR) {
-                const unsigned long long deg = __ldg(F.q_off + i + 1) - off;
+                const unsigned u = __ldcs(F.q_v + i);
+                const unsigned long long deg = __ldcs(F.q_off + i + 1) - off;
                 s_val[kk] = (VT)(__ldcg(F.x + u) / (double)deg);
-            } else {
+            } else if (ALG != ALG_BFS) {
+                const unsigned u = __ldcs(F.q_v + i);
                 s_val[kk] = (VT)__ldcg(F.state + u);
             }
             const long long rel = (long long)off - (long long)tb;
-            if (rel > 0 && rel < (long long)tlen) s_head[rel] = (unsigned short)kk;
+            if (rel > 0 && rel < (long long)tlen) s_head[rel] = (seq << 12) | kk;
         }
         __syncthreads();
         // blocked inclusive max-scan of s_head: s_head[e] = index of the vertex owning edge e
@@ -553,7 +679,8 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
             unsigned run = 0;
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
-                hv[j] = (b + j < tlen) ? s_head[b + j] : 0u;
+                const unsigned raw = (b + j < tlen) ? s_head[b + j] : 0u;
+                hv[j] = (raw >> 12) == seq ? (raw & 0xFFFu) : 0u;
                 run = hv[j] > run ? hv[j] : run;
                 hv[j] = run;
             }
@@ -570,35 +697,36 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
             for (unsigned i = 0; i < (threadIdx.x >> 5); i++) excl = s_wmax[i] > excl ? s_wmax[i] : excl;
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++)
-                if (b + j < tlen) s_head[b + j] = (unsigned short)(hv[j] > excl ? hv[j] : excl);
+                if (b + j < tlen) s_head[b + j] = hv[j] > excl ? hv[j] : excl;
         }
         __syncthreads();
 
-        // ---- expand: striped edges, coalesced col/w loads; apply to the owner fragment
+        // ---- expand: striped edges, coalesced streaming col/w loads
         unsigned vv[kEdgesPerThread];
         VT cv[kEdgesPerThread];
 #pragma unroll
         for (int j = 0; j < kEdgesPerThread; j++) {
             const unsigned e = j * kThreads + threadIdx.x;
             vv[j] = GUM_INF;
+            cv[j] = (VT)0;
             if (e < tlen) {
                 const unsigned kk = s_head[e];
                 const unsigned long long ci = (unsigned long long)((long long)(tb + e) + s_base[kk]);
-                vv[j] = __ldg(F.col + ci);
-                if (ALG == ALG_BFS) cv[j] = s_val[kk] + 1u;
-                if (ALG == ALG_WCC) cv[j] = s_val[kk];
-                if (ALG == ALG_PR) cv[j] = s_val[kk];
+                vv[j] = __ldcs(F.col + ci);
+                if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
+                if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];
                 if (ALG == ALG_SSSP) {
-                    const unsigned long long nd = (unsigned long long)s_val[kk] + __ldg(F.w + ci);
+                    const unsigned long long nd = (unsigned long long)s_val[kk] + __ldcs(F.w + ci);
                     if (nd >= (unsigned long long)GUM_INF) {
                         atomicOr(&F.ctl->err, 1u);
                         vv[j] = GUM_INF;
                     }
-                    cv[j] = (unsigned)nd;
+                    cv[j] = (VT)(unsigned)nd;
                 }
             }
         }
         if (ALG == ALG_PR) {
+            // GAS apply for PR: push x[u]/outdeg(u) into the owner's accumulator (red.global.add.f64)
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
                 if (vv[j] != GUM_INF) {
@@ -610,61 +738,111 @@ __global__ void __launch_bounds__(kThreads, 4) k_advance(const __grid_constant__
                         lv = v - c.bounds[tf];
                         remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
                     }
-                    atomicAdd(c.f[tf].acc + lv, cv[j]);
+                    atomicAdd(c.f[tf].acc + lv, (double)cv[j]);
                 }
+            }
+        } else if (ALG == ALG_BFS) {
+            // BFS: check the visited bit (1 bit/vertex, L1-cacheable) instead of the 4-byte depth.
+            // All candidates of iteration k equal k+1, so the depth store needs no atomic.
+            unsigned lvv[kEdgesPerThread], wd[kEdgesPerThread];
+            unsigned char tfv[kEdgesPerThread];
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                tfv[j] = 0;
+                lvv[j] = vv[j];
+                wd[j] = 0xFFFFFFFFu;
+                if (vv[j] != GUM_INF) {
+                    if (MULTI) {
+                        const int tf = frag_of(c, vv[j]);
+                        tfv[j] = (unsigned char)tf;
+                        lvv[j] = vv[j] - c.bounds[tf];
+                    }
+                    wd[j] = c.f[tfv[j]].vis[lvv[j] >> 5];
+                }
+            }
+            unsigned upd = 0;
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++)
+                if (!(wd[j] & (1u << (lvv[j] & 31)))) upd |= 1u << j;
+            if (next_dense) {
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++) {
+                    if (upd & (1u << j)) {
+                        const FragPtrs& T = c.f[tfv[j]];
+                        const unsigned bit = 1u << (lvv[j] & 31);
+                        atomicOr(T.vis + (lvv[j] >> 5), bit);  // RED.OR
+                        atomicOr(T.bm + (lvv[j] >> 5), bit);   // RED.OR
+                        T.state[lvv[j]] = k + 1;
+                        if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
+                    }
+                }
+                acts += __popc(upd);
+            } else {
+                unsigned ob[kEdgesPerThread];
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++) {
+                    ob[j] = 0xFFFFFFFFu;
+                    if (upd & (1u << j)) ob[j] = atomicOr(c.f[tfv[j]].vis + (lvv[j] >> 5), 1u << (lvv[j] & 31));
+                }
+                unsigned need = 0;
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++) {
+                    if (!(ob[j] & (1u << (lvv[j] & 31)))) {
+                        need |= 1u << j;
+                        c.f[tfv[j]].state[lvv[j]] = k + 1;
+                        if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
+                    }
+                }
+                acts += append_activations<MULTI>(c, need, tfv, lvv);
             }
         } else {
-            unsigned cur[kEdgesPerThread];
+            // GAS apply for min-algorithms: check (plain load) -> red.min on the owner's state ->
+            // activation bit. Any thread whose candidate beat the value it read knows v improved in this
+            // iteration, so it may set v's bit without waiting for the atomic's return value.
+            unsigned lvv[kEdgesPerThread], cur[kEdgesPerThread];
+            unsigned char tfv[kEdgesPerThread];
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
+                tfv[j] = 0;
+                lvv[j] = vv[j];
                 cur[j] = 0;
                 if (vv[j] != GUM_INF) {
-                    const int tf = MULTI ? frag_of(c, vv[j]) : 0;
-                    const unsigned lv = MULTI ? vv[j] - c.bounds[tf] : vv[j];
-                    cur[j] = __ldcg(c.f[tf].state + lv);  // check before atomic
+                    if (MULTI) {
+                        const int tf = frag_of(c, vv[j]);
+                        tfv[j] = (unsigned char)tf;
+                        lvv[j] = vv[j] - c.bounds[tf];
+                    }
+                    cur[j] = c.f[tfv[j]].state[lvv[j]];
                 }
             }
+            unsigned upd = 0;
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
-                bool need = false;
-                int tf = 0;
-                unsigned lv = 0;
-                if (vv[j] != GUM_INF && cv[j] < cur[j]) {
-                    tf = MULTI ? frag_of(c, vv[j]) : 0;
-                    lv = MULTI ? vv[j] - c.bounds[tf] : vv[j];
-                    if (MULTI) remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
-                    const unsigned old = atomicMin(c.f[tf].state + lv, (unsigned)cv[j]);
-                    if ((unsigned)cv[j] < old) {
-                        const unsigned bit = 1u << (lv & 31);
-                        const unsigned ob = atomicOr(c.f[tf].bm + (lv >> 5), bit);
-                        need = (ob & bit) == 0;
-                    }
+                if (vv[j] != GUM_INF && (unsigned)cv[j] < cur[j]) {
+                    upd |= 1u << j;
+                    atomicMin(c.f[tfv[j]].state + lvv[j], (unsigned)cv[j]);  // RED.MIN (no return)
+                    if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
                 }
-                // warp-aggregated append to the owner's activation list (next frontier)
-                if (MULTI) {
-                    const unsigned key = need ? (unsigned)tf : 0xFFFFFFFFu;
-                    const unsigned grp = __match_any_sync(0xffffffffu, key);
-                    if (need) {
-                        const unsigned leader = __ffs(grp) - 1;
-                        unsigned basepos = 0;
-                        if (lane_id() == leader) basepos = atomicAdd(&c.f[tf].ctl->app_cnt, (unsigned)__popc(grp));
-                        basepos = __shfl_sync(grp, basepos, leader);
-                        c.f[tf].app[basepos + __popc(grp & lanemask_lt())] = lv;
-                        acts++;
-                    }
-                } else {
-                    const unsigned grp = __ballot_sync(0xffffffffu, need);
-                    if (grp) {
-                        const unsigned leader = __ffs(grp) - 1;
-                        unsigned basepos = 0;
-                        if (lane_id() == leader) basepos = atomicAdd(&c.f[0].ctl->app_cnt, (unsigned)__popc(grp));
-                        basepos = __shfl_sync(0xffffffffu, basepos, leader);
-                        if (need) {
-                            c.f[0].app[basepos + __popc(grp & lanemask_lt())] = lv;
-                            acts++;
-                        }
-                    }
+            }
+            if (next_dense) {
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++)
+                    if (upd & (1u << j)) atomicOr(c.f[tfv[j]].bm + (lvv[j] >> 5), 1u << (lvv[j] & 31));  // RED.OR
+                acts += __popc(upd);
+            } else {
+                // sparse next frontier: dedupe on the bitmap (returning atomics issued back to back) and
+                // append with one warp-aggregated reservation per target fragment
+                unsigned ob[kEdgesPerThread];
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++) {
+                    ob[j] = 0xFFFFFFFFu;
+                    if (upd & (1u << j)) ob[j] = atomicOr(c.f[tfv[j]].bm + (lvv[j] >> 5), 1u << (lvv[j] & 31));
                 }
+                unsigned need = 0;
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++)
+                    if (!(ob[j] & (1u << (lvv[j] & 31)))) need |= 1u << j;
+                acts += append_activations<MULTI>(c, need, tfv, lvv);
             }
         }
         if (threadIdx.x == 0) {
@@ -835,7 +1013,9 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
         case ALG_WCC: k_init<ALG_WCC><<<g, kThreads, 0, s>>>(c, f0); break;
         default: k_init<ALG_PR><<<g, kThreads, 0, s>>>(c, f0); break;
     }
-    k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, c.trace[L.w0]);
+    // the initial frontier: {source} as a list (BFS/SSSP) or every vertex as a full bitmap (WCC/PR)
+    const unsigned nd0 = c.force_mode == 1 ? 0u : ((alg == ALG_WCC || alg == ALG_PR) ? 1u : 0u);
+    k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, nd0);
     if (src_frag >= f0 && src_frag < f0 + nf) k_init_source<<<1, 1, 0, s>>>(c, src_frag, src_local);
     if (alg == ALG_PR) {
         // PR's frontier is every vertex with out-degree > 0: build its queue once (dense filter)
@@ -852,14 +1032,42 @@ cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStre
     return cudaGetLastError();
 }
 
-cudaError_t advance_occupancy(int* blocks_per_sm) {
-    int a = 0, b = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_advance<ALG_PR, true>, kThreads, 0);
-    if (e != cudaSuccess) return e;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_advance<ALG_SSSP, true>, kThreads, 0);
-    if (e != cudaSuccess) return e;
-    *blocks_per_sm = a < b ? a : b;
-    return cudaSuccess;
+static int g_carveout = -1;  // GUM_SMEM_CARVEOUT (percent) for tuning; -1 = driver default
+template <int ALG, bool MULTI>
+static void carveout() {
+    if (g_carveout >= 0)
+        cudaFuncSetAttribute(k_advance<ALG, MULTI>, cudaFuncAttributePreferredSharedMemoryCarveout, g_carveout);
+}
+
+template <int ALG, bool MULTI>
+static cudaError_t occ_of(int* n) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(n, k_advance<ALG, MULTI>, kThreads, 0);
+}
+
+cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm) {
+    static bool once = false;
+    if (!once) {
+        once = true;
+        if (const char* e = getenv("GUM_SMEM_CARVEOUT")) g_carveout = atoi(e);
+        carveout<ALG_BFS, false>();
+        carveout<ALG_BFS, true>();
+        carveout<ALG_SSSP, false>();
+        carveout<ALG_SSSP, true>();
+        carveout<ALG_WCC, false>();
+        carveout<ALG_WCC, true>();
+        carveout<ALG_PR, false>();
+        carveout<ALG_PR, true>();
+    }
+    switch (alg * 2 + (multi ? 1 : 0)) {
+        case 0: return occ_of<ALG_BFS, false>(blocks_per_sm);
+        case 1: return occ_of<ALG_BFS, true>(blocks_per_sm);
+        case 2: return occ_of<ALG_SSSP, false>(blocks_per_sm);
+        case 3: return occ_of<ALG_SSSP, true>(blocks_per_sm);
+        case 4: return occ_of<ALG_WCC, false>(blocks_per_sm);
+        case 5: return occ_of<ALG_WCC, true>(blocks_per_sm);
+        case 6: return occ_of<ALG_PR, false>(blocks_per_sm);
+        default: return occ_of<ALG_PR, true>(blocks_per_sm);
+    }
 }
 
 }  // namespace gum

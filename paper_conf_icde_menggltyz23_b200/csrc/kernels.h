@@ -26,7 +26,7 @@ cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L
 cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream_t s, int f0, int nf, double D0,
                         int src_frag, unsigned src_local);
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
-cudaError_t advance_occupancy(int* blocks_per_sm);
+cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 
 // ---- setup (setup.cu): validation, partitioning, relabelling, symmetrisation -------------------
 cudaError_t setup_validate(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,

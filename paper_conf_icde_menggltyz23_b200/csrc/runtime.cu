@@ -8,6 +8,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -39,6 +40,7 @@ struct FragBufs {
     double* x = nullptr;
     double* acc = nullptr;
     unsigned* bm = nullptr;
+    unsigned* vis = nullptr;
     unsigned* app = nullptr;
     unsigned* q_v = nullptr;
     unsigned long long* q_off = nullptr;
@@ -59,7 +61,7 @@ struct gum_ctx {
     cudaStream_t stream[kMaxW] = {nullptr};
     bool own_stream[kMaxW] = {false};
     int nsm = 148;
-    int adv_occ = 4;
+    int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
     std::string err;
     bool poisoned = false;
     std::vector<Alloc> load_allocs, part_allocs, misc_allocs;
@@ -186,15 +188,15 @@ int unit_w0(const gum_ctx* c, int u) { return c->single_device ? 0 : u; }
 int unit_nw(const gum_ctx* c, int u) { return c->single_device ? c->P : 1; }
 int unit_dev(const gum_ctx* c, int u) { return c->dev[unit_w0(c, u)]; }
 
-LaunchCfg make_launch(const gum_ctx* c, int u) {
+LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     LaunchCfg L;
     L.w0 = unit_w0(c, u);
     L.nw = unit_nw(c, u);
-    int grid = c->nsm * c->adv_occ;
+    int grid = c->nsm * c->adv_occ[alg][c->P > 1 ? 1 : 0];
     grid = (grid / L.nw) * L.nw;
     if (grid < L.nw) grid = L.nw;
     L.adv_grid = grid;
-    L.filter_grid = std::max(1, (c->nsm * 2) / (c->single_device ? std::min(c->P, 2) : 1));
+    L.filter_grid = std::max(1, (c->nsm * 4) / (c->single_device ? std::min(c->P, 4) : 1));
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
     return L;
@@ -221,6 +223,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.acc = F.acc;
         p.orig = F.orig;
         p.bm = F.bm;
+        p.vis = F.vis;
         p.app = F.app;
         p.q_v = F.q_v;
         p.q_off = F.q_off;
@@ -489,8 +492,12 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     }
     cudaSetDevice(c->dev[0]);
     cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->dev[0]);
-    int occ = 0;
-    if (advance_occupancy(&occ) == cudaSuccess && occ > 0) c->adv_occ = occ;
+    for (int a = 0; a < 4; a++)
+        for (int m = 0; m < 2; m++) {
+            int occ = 0;
+            if (advance_occupancy(a, m, &occ) == cudaSuccess && occ > 0) c->adv_occ[a][m] = occ;
+            if (const char* e = getenv("GUM_ADV_CTAS_PER_SM")) c->adv_occ[a][m] = std::max(1, atoi(e));
+        }
     cudaGetLastError();
     cudaEventCreate(&c->ev0);
     cudaEventCreate(&c->ev1);
@@ -701,12 +708,13 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.x = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.acc = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.bm = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
+        F.vis = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.app = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
         F.q_v = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
         F.q_off = (unsigned long long*)dalloc(c, F.dev, (Vn + 1) * 8, c->part_allocs);
         F.q_base = (long long*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
-        if (!F.state || !F.x || !F.acc || !F.bm || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
+        if (!F.state || !F.x || !F.acc || !F.bm || !F.vis || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
             return fail(c, GUM_ENOMEM, "fragment %d state alloc failed", f);
         CK(cudaSetDevice(F.dev));
         CK(cudaMemset(F.ctl, 0, sizeof(FragCtl)));
@@ -718,7 +726,7 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
     unsigned parts = 1;
     for (int f = 0; f < c->P; f++) {
         unsigned nwords = (c->fr[f].V + 31) / 32;
-        unsigned a = (nwords + kFilterWordsPerPart - 1) / kFilterWordsPerPart;
+        unsigned a = (nwords + kDenseWordsPerPart - 1) / kDenseWordsPerPart;
         unsigned b = (c->fr[f].V + kFilterAppPerPart - 1) / kFilterAppPerPart;
         parts = std::max(parts, std::max(a, b) + 1);
     }
@@ -802,7 +810,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     cudaEvent_t init_a = nullptr, init_b = nullptr;
     if (graph_mode) {
         CK(cudaSetDevice(c->dev[0]));
-        st = capture_graph(c, alg, d, make_launch(c, 0));
+        st = capture_graph(c, alg, d, make_launch(c, 0, alg));
         if (st != GUM_OK) return st;
     }
     CK(cudaSetDevice(c->dev[0]));
@@ -817,7 +825,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         CK(cudaEventRecord(init_a, c->stream[0]));
     }
     for (int u = 0; u < c->n_units; u++) {
-        const LaunchCfg L = make_launch(c, u);
+        const LaunchCfg L = make_launch(c, u, alg);
         CK(cudaSetDevice(unit_dev(c, u)));
         CK(launch_init(alg, d, L, c->stream[L.w0], L.w0, L.nw, D0, src_frag, src_local));
     }
@@ -833,7 +841,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
                     st = unit_barrier(c);
                     if (st != GUM_OK) return st;
                     for (int u = 0; u < c->n_units; u++) {
-                        const LaunchCfg L = make_launch(c, u);
+                        const LaunchCfg L = make_launch(c, u, alg);
                         CK(cudaSetDevice(unit_dev(c, u)));
                         st = run_phase(c, alg, phase, d, L, c->stream[L.w0]);
                         if (st != GUM_OK) return st;

@@ -1,0 +1,41 @@
+"""Summarise an ncu --set full report: key metrics + top stall reasons (SASS source page)."""
+import csv
+import io
+import subprocess
+import sys
+
+rep = sys.argv[1]
+KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+        "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sector_hit_rate.pct",
+        "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
+        "launch__occupancy_limit_registers", "launch__occupancy_limit_shared_mem", "launch__grid_size",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
+        "lts__t_requests_srcunit_tex_op_red.sum", "lts__t_requests_srcunit_tex_op_atom.sum",
+        "sm__cycles_elapsed.avg.per_second"]
+raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+rows = list(csv.reader(io.StringIO(raw)))
+h, units = rows[0], rows[1]
+for r in rows[2:]:
+    print("kernel:", r[h.index("Kernel Name")][:80] if "Kernel Name" in h else "")
+    for k in KEYS:
+        if k in h:
+            i = h.index(k)
+            print(f"  {k:62s} {r[i]:>18s} {units[i]}")
+src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=sass"], capture_output=True,
+                     text=True).stdout
+rows = list(csv.reader(io.StringIO(src)))
+if len(rows) > 2:
+    h = rows[1]
+    data = rows[2:]
+    ix = {n: i for i, n in enumerate(h)}
+    col = "Warp Stall Sampling (All Samples)"
+    tot = sum(float(r[ix[col]] or 0) for r in data) or 1
+    stalls = [n for n in h if n.startswith("stall_") and "Not Issued" not in n]
+    agg = sorted(((sum(float(r[ix[n]] or 0) for r in data) / tot * 100, n) for n in stalls), reverse=True)[:8]
+    print("  stall reasons (% of samples):", ", ".join(f"{n[6:]} {v:.1f}" for v, n in agg))
+    print("  top instructions:")
+    for r in sorted(data, key=lambda r: -float(r[ix[col]] or 0))[:int(sys.argv[2]) if len(sys.argv) > 2 else 12]:
+        smp = float(r[ix[col]] or 0)
+        br = sorted(((float(r[ix[n]] or 0), n[6:]) for n in stalls), reverse=True)[:2]
+        print(f"    {smp / tot * 100:5.1f}%  {r[1][:58]:58s} {br}")

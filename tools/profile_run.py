@@ -1,0 +1,31 @@
+"""One configurable GUM run for ncu captures (host-loop mode: every kernel is a separate launch).
+
+  python tools/profile_run.py --config C2 --alg bfs --runs 1
+"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import inputs  # noqa: E402
+import paper_conf_icde_menggltyz23_b200 as gum  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C2")
+ap.add_argument("--alg", default="bfs")
+ap.add_argument("--runs", type=int, default=1)
+ap.add_argument("--gpus", type=int, default=1)
+ap.add_argument("--host-loop", type=int, default=1)
+a = ap.parse_args()
+g = inputs.make_config(a.config, weighted=(a.alg == "sssp"))
+s = 0 if a.config == "C3" else inputs.pick_source(g, int(a.config[1]))
+rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
+with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop)) as ctx:
+    ctx.load_csr(rp, col, w)
+    ctx.partition()
+    ctx.prepare(a.alg)
+    for _ in range(a.runs):
+        st = ctx.run(a.alg, s)
+    print(st)
