@@ -140,7 +140,7 @@ def advance_bytes(alg, st):
     state 4 B (+ w 4 B for SSSP; PR: acc 8 B), per frontier vertex 24 B (queue id 4, prefix 8, col base
     8, own state 4; PR: x 8 instead of state 4 -> 28 B), per activation 8 B (bitmap 4 + list 4)."""
     per_edge = {"bfs": 8, "sssp": 12, "wcc": 8, "pr": 12}[alg]
-    per_vertex = 28 if alg == "pr" else 24
+    per_vertex = 20 if alg == "pr" else 24  # PR queue entry: q_v 4 + q_off 8 + x/outdeg 8
     return per_edge * st.edges_expanded + per_vertex * st.vertices_frontier + 8 * st.activations
 
 

@@ -76,6 +76,7 @@ struct FragPtrs {
     unsigned int* state;                // [V_f] depth / dist / label
     double* x;                          // PR [V_f]
     double* acc;                        // PR [V_f]
+    double* cx;                         // PR [V_f] x[u]/outdeg(u): the value pushed along out-edges
     const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
     unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
     unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
@@ -88,6 +89,7 @@ struct FragPtrs {
     unsigned int V;                     // |V_f|
     unsigned int base;                  // global id of local vertex 0
     unsigned long long E;
+    unsigned long long pr_qlen, pr_qedges;  // PR's static destination-blocked queue (gum_prepare)
 };
 
 struct DevCtx {

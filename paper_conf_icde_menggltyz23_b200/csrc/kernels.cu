@@ -68,8 +68,11 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
             if (ALG == ALG_WCC) F.state[i] = F.orig ? F.orig[i] : F.base + i;
             if (ALG == ALG_WCC || ALG == ALG_PR) F.app[i] = i;  // all-active frontier as a list too
             if (ALG == ALG_PR) {
-                F.x[i] = 1.0 / (double)c.num_vertices;
+                const double x0 = 1.0 / (double)c.num_vertices;
+                const unsigned long long od = F.row_ptr[i + 1] - F.row_ptr[i];
+                F.x[i] = x0;
                 F.acc[i] = 0.0;
+                F.cx[i] = od ? x0 / (double)od : 0.0;  // the contribution x/outdeg pushed along out-edges
             }
         }
         if (i < nwords) {
@@ -85,10 +88,11 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         FragCtl* ct = F.ctl;
         ct->claim = 0;
-        ct->ntiles = 0;
-        ct->qlen = 0;
-        ct->qedges = 0;
-        ct->app_cnt = (ALG == ALG_WCC || ALG == ALG_PR) ? F.V : 0;
+        // PR: the frontier is the static destination-blocked queue built by gum_prepare(PR)
+        ct->ntiles = (ALG == ALG_PR) ? (F.pr_qedges + c.chunk - 1) / c.chunk : 0;
+        ct->qlen = (ALG == ALG_PR) ? F.pr_qlen : 0;
+        ct->qedges = (ALG == ALG_PR) ? F.pr_qedges : 0;
+        ct->app_cnt = (ALG == ALG_WCC) ? F.V : 0;
         ct->err = 0;
         ct->dense = 0;
         ct->pr_dang[0] = ct->pr_dang[1] = 0.0;
@@ -659,11 +663,11 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
         for (unsigned kk = threadIdx.x; kk < nv; kk += kThreads) {
             const unsigned i = i0 + kk;
             const unsigned long long off = __ldcs(F.q_off + i);
-            s_base[kk] = __ldcs(F.q_base + i);
+            // PR's blocked queue stores edges contiguously in queue order: col index == q_off + j
+            s_base[kk] = (ALG == ALG_PR) ? 0ll : __ldcs(F.q_base + i);
             if (ALG == ALG_PR) {
                 const unsigned u = __ldcs(F.q_v + i);
-                const unsigned long long deg = __ldcs(F.q_off + i + 1) - off;
-                s_val[kk] = (VT)(__ldcg(F.x + u) / (double)deg);
+                s_val[kk] = (VT)__ldcg(F.cx + u);
             } else if (ALG != ALG_BFS) {
                 const unsigned u = __ldcs(F.q_v + i);
                 s_val[kk] = (VT)__ldcg(F.state + u);
@@ -897,8 +901,10 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
         const double xo = F.x[i];
         const double nx = (1.0 - d) / N + d * (F.acc[i] + D / N);
         res += fabs(nx - xo);
-        if (__ldg(F.row_ptr + i + 1) == __ldg(F.row_ptr + i)) dang += nx;
+        const unsigned long long od = __ldg(F.row_ptr + i + 1) - __ldg(F.row_ptr + i);
+        if (od == 0) dang += nx;
         F.x[i] = nx;
+        F.cx[i] = od ? nx / (double)od : 0.0;  // next iteration's push value x'/outdeg
         F.acc[i] = 0.0;
     }
 #pragma unroll
@@ -1017,10 +1023,6 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
     const unsigned nd0 = c.force_mode == 1 ? 0u : ((alg == ALG_WCC || alg == ALG_PR) ? 1u : 0u);
     k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, nd0);
     if (src_frag >= f0 && src_frag < f0 + nf) k_init_source<<<1, 1, 0, s>>>(c, src_frag, src_local);
-    if (alg == ALG_PR) {
-        // PR's frontier is every vertex with out-degree > 0: build its queue once (dense filter)
-        k_filter<<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
-    }
     return cudaGetLastError();
 }
 

@@ -46,6 +46,11 @@ cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* 
 // fragment extraction: rebased row_ptr slice; orig ids slice (or identity when inv == null)
 cudaError_t setup_rebase_rows(const unsigned long long* row_ptr, unsigned b0, unsigned b1, unsigned long long* out,
                               cudaStream_t s);
+// PR destination-blocked static queue: pcol may be null when B == 1 (then the fragment col is used as is)
+size_t setup_pr_tmp_bytes(unsigned Vf, int B);
+cudaError_t setup_pr_blocked(const unsigned long long* rp, const unsigned* col, unsigned Vf, unsigned long long Ef,
+                             unsigned S, int B, unsigned chunk, unsigned* pcol, unsigned* q_v, unsigned long long* q_off,
+                             unsigned* tile, unsigned long long* h_Q, void* tmp, size_t tmp_bytes, cudaStream_t s);
 cudaError_t setup_count_dangling(const unsigned long long* row_ptr, unsigned V, unsigned long long* d_count,
                                  cudaStream_t s);
 unsigned host_feistel(unsigned v, unsigned V, unsigned long long seed);

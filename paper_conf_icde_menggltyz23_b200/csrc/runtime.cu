@@ -48,6 +48,13 @@ struct FragBufs {
     unsigned* tile = nullptr;
     unsigned long long tile_cap = 0;
     FragCtl* ctl = nullptr;
+    double* cx = nullptr;
+    // PR static destination-blocked queue (gum_prepare(PR))
+    unsigned* pr_col = nullptr;
+    unsigned* pr_q_v = nullptr;
+    unsigned long long* pr_q_off = nullptr;
+    unsigned* pr_tile = nullptr;
+    unsigned long long pr_qlen = 0, pr_qedges = 0;
 };
 
 }  // namespace
@@ -83,6 +90,8 @@ struct gum_ctx {
     unsigned* p_col = nullptr;
     unsigned* p_w = nullptr;
     bool sym_ready = false;
+    bool pr_ready = false;
+    int pr_blocks = 1;
     FragBufs fr[kMaxW];
     unsigned long long n_dangling = 0;
     RunCtl* rctl[kMaxW] = {nullptr};
@@ -169,6 +178,7 @@ void drop_partition(gum_ctx* c) {
     free_list(c, c->part_allocs);
     c->partitioned = false;
     c->sym_ready = false;
+    c->pr_ready = false;
     c->has_result = false;
     c->inv = nullptr;
     c->p_row_ptr = nullptr;
@@ -221,6 +231,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.state = F.state;
         p.x = F.x;
         p.acc = F.acc;
+        p.cx = F.cx;
         p.orig = F.orig;
         p.bm = F.bm;
         p.vis = F.vis;
@@ -229,6 +240,15 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.q_off = F.q_off;
         p.q_base = F.q_base;
         p.tile = F.tile;
+        if (alg == GUM_PR) {
+            p.col = F.pr_col;
+            p.q_v = F.pr_q_v;
+            p.q_off = F.pr_q_off;
+            p.q_base = nullptr;
+            p.tile = F.pr_tile;
+            p.pr_qlen = F.pr_qlen;
+            p.pr_qedges = F.pr_qedges;
+        }
         p.ctl = F.ctl;
         p.V = F.V;
         p.base = F.base;
@@ -359,6 +379,52 @@ gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const Laun
         c->prof_ev.push_back(b);
         c->prof_kind.push_back(kinds[i]);
     }
+    return GUM_OK;
+}
+
+// PR's frontier is every vertex with out-degree > 0 in every iteration: build it once, regrouped by
+// destination block so that consecutive chunks push into one L2-resident slice of acc.
+gum_status build_pr(gum_ctx* c) {
+    if (c->pr_ready) return GUM_OK;
+    const unsigned long long block_bytes = getenv("GUM_PR_BLOCK_BYTES") ? strtoull(getenv("GUM_PR_BLOCK_BYTES"), 0, 10)
+                                                                       : (48ull << 20);
+    unsigned long long S = std::max<unsigned long long>(1024, block_bytes / 8);
+    int B = 1;
+    if ((unsigned long long)c->V * 8 > block_bytes + (block_bytes >> 1)) B = (int)((c->V + S - 1) / S);
+    if (B > 64) {
+        B = 64;
+        S = (c->V + 63) / 64;
+    }
+    if (B == 1) S = (unsigned long long)c->V + 1;
+    c->pr_blocks = B;
+    for (int f = 0; f < c->P; f++) {
+        FragBufs& F = c->fr[f];
+        CK(cudaSetDevice(F.dev));
+        cudaStream_t s = c->stream[c->single_device ? 0 : f];
+        const unsigned long long cap = std::min<unsigned long long>((unsigned long long)B * F.V, F.E) + 1;
+        F.pr_col = B > 1 ? (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.E, 1) * 4, c->part_allocs) : F.col;
+        F.pr_q_v = (unsigned*)dalloc(c, F.dev, cap * 4, c->part_allocs);
+        F.pr_q_off = (unsigned long long*)dalloc(c, F.dev, (cap + 1) * 8, c->part_allocs);
+        F.pr_tile = (unsigned*)dalloc(c, F.dev, (F.E / c->cfg.chunk_edges + 2) * 4, c->part_allocs);
+        std::vector<Alloc> tmp;
+        const size_t tb = setup_pr_tmp_bytes(F.V, B);
+        void* t = dalloc(c, F.dev, tb, tmp);
+        if (!F.pr_col || !F.pr_q_v || !F.pr_q_off || !F.pr_tile || !t) {
+            free_list(c, tmp);
+            return fail(c, GUM_ENOMEM, "PR blocked queue alloc failed (fragment %d, %d blocks)", f, B);
+        }
+        unsigned long long Q = 0;
+        cudaError_t e = setup_pr_blocked(F.row_ptr, F.col, F.V, F.E, (unsigned)S, B, c->cfg.chunk_edges,
+                                         B > 1 ? F.pr_col : nullptr, F.pr_q_v, F.pr_q_off, F.pr_tile, &Q, t, tb, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        free_list(c, tmp);
+        if (e != cudaSuccess) return fail(c, GUM_ECUDA, "PR blocked queue: %s", cudaGetErrorString(e));
+        F.pr_qlen = Q;
+        F.pr_qedges = F.E;
+    }
+    CK(cudaSetDevice(c->dev[0]));
+    c->pr_ready = true;
+    drop_graphs(c);
     return GUM_OK;
 }
 
@@ -707,6 +773,7 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.state = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
         F.x = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.acc = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
+        F.cx = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.bm = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.vis = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.app = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
@@ -714,7 +781,7 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.q_off = (unsigned long long*)dalloc(c, F.dev, (Vn + 1) * 8, c->part_allocs);
         F.q_base = (long long*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
-        if (!F.state || !F.x || !F.acc || !F.bm || !F.vis || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
+        if (!F.state || !F.x || !F.acc || !F.cx || !F.bm || !F.vis || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
             return fail(c, GUM_ENOMEM, "fragment %d state alloc failed", f);
         CK(cudaSetDevice(F.dev));
         CK(cudaMemset(F.ctl, 0, sizeof(FragCtl)));
@@ -776,6 +843,7 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
     if (alg == GUM_WCC) return build_sym(c);
+    if (alg == GUM_PR) return build_pr(c);
     if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
     return GUM_OK;
 }

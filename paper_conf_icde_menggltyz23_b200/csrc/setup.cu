@@ -197,6 +197,122 @@ cudaError_t setup_rebase_rows(const unsigned long long* row_ptr, unsigned b0, un
     return cudaGetLastError();
 }
 
+// ---- PR destination-blocked static queue (gum_prepare(PR)) ---------------------------------------
+// Destination ids are split into blocks of S ids (an acc block of 8*S bytes sized to stay L2-resident);
+// edges are regrouped block-major (rows ascending inside a block, edge order kept inside a row) and the
+// static PR frontier becomes the queue of (block, row) pairs with edges, in that order. Consecutive
+// chunks then push into one block of acc at a time.
+__global__ void k_pr_count(const unsigned long long* rp, const unsigned* col, unsigned Vf, unsigned S, int B,
+                           unsigned long long* cnt /* [B*Vf + 1] */) {
+    extern __shared__ unsigned s_hist[];  // B counters per warp
+    const unsigned lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    unsigned* h = s_hist + wib * B;
+    const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+    const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
+    for (unsigned long long u = warp; u < Vf; u += nwarps) {
+        for (int b = lane; b < B; b += 32) h[b] = 0;
+        __syncwarp();
+        for (unsigned long long e = rp[u] + lane; e < rp[u + 1]; e += 32) atomicAdd(h + col[e] / S, 1u);
+        __syncwarp();
+        for (int b = lane; b < B; b += 32) cnt[(unsigned long long)b * Vf + u] = h[b];
+        __syncwarp();
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) cnt[(unsigned long long)B * Vf] = 0;
+}
+
+__global__ void k_pr_scatter(const unsigned long long* rp, const unsigned* col, unsigned Vf, unsigned S, int B,
+                             const unsigned long long* off, unsigned* pcol) {
+    extern __shared__ unsigned long long s_cur[];  // B cursors per warp
+    const unsigned lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    unsigned long long* cur = s_cur + wib * B;
+    const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+    const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
+    for (unsigned long long u = warp; u < Vf; u += nwarps) {
+        for (int b = lane; b < B; b += 32) cur[b] = off[(unsigned long long)b * Vf + u];
+        __syncwarp();
+        const unsigned long long e0 = rp[u], e1 = rp[u + 1];
+        for (unsigned long long eb = e0; eb < e1; eb += 32) {
+            const unsigned long long e = eb + lane;
+            const bool ok = e < e1;
+            const unsigned v = ok ? col[e] : 0u;
+            const unsigned b = ok ? v / S : 0xFFFFFFFFu;
+            const unsigned grp = __match_any_sync(0xffffffffu, b);
+            const unsigned leader = __ffs(grp) - 1;
+            unsigned long long base = 0;
+            if (ok) base = cur[b];  // stable: ranks follow the row's edge order
+            if (ok) pcol[base + __popc(grp & ((1u << lane) - 1u))] = v;
+            __syncwarp();
+            if (ok && lane == leader) cur[b] = base + __popc(grp);
+            __syncwarp();
+        }
+    }
+}
+
+__global__ void k_pr_flags(const unsigned long long* off, unsigned long long n, unsigned* flag) {
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i <= n;
+         i += (unsigned long long)gridDim.x * blockDim.x)
+        flag[i] = (i < n && off[i + 1] > off[i]) ? 1u : 0u;
+}
+
+__global__ void k_pr_emit(const unsigned long long* off, const unsigned* pos, unsigned long long n, unsigned Vf,
+                          unsigned chunk, unsigned* q_v, unsigned long long* q_off, unsigned* tile) {
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+        const unsigned long long o = off[i], d = off[i + 1] - o;
+        if (!d) continue;
+        const unsigned p = pos[i];
+        q_v[p] = (unsigned)(i % Vf);
+        q_off[p] = o;
+        for (unsigned long long t = (o + chunk - 1) / chunk; t * chunk < o + d; t++) tile[t] = p;
+    }
+}
+
+size_t setup_pr_tmp_bytes(unsigned Vf, int B) {
+    const unsigned long long n = (unsigned long long)B * Vf + 1;
+    size_t a = 0, b = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, a, (unsigned long long*)nullptr, (unsigned long long*)nullptr, (size_t)n);
+    cub::DeviceScan::ExclusiveSum(nullptr, b, (unsigned*)nullptr, (unsigned*)nullptr, (size_t)n);
+    return std::max(a, b) + 256 + n * 8 + n * 4 * 2 + 1024;
+}
+
+cudaError_t setup_pr_blocked(const unsigned long long* rp, const unsigned* col, unsigned Vf, unsigned long long Ef,
+                             unsigned S, int B, unsigned chunk, unsigned* pcol, unsigned* q_v, unsigned long long* q_off,
+                             unsigned* tile, unsigned long long* h_Q, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    const unsigned long long n = (unsigned long long)B * Vf;
+    char* t = (char*)tmp;
+    unsigned long long* off = (unsigned long long*)t;
+    t += ((n + 1) * 8 + 255) / 256 * 256;
+    unsigned* flag = (unsigned*)t;
+    t += ((n + 1) * 4 + 255) / 256 * 256;
+    unsigned* pos = (unsigned*)t;
+    t += ((n + 1) * 4 + 255) / 256 * 256;
+    void* cub_tmp = t;
+    size_t cub_bytes = tmp_bytes - (size_t)(t - (char*)tmp);
+    const int warps_per_cta = 8;
+    k_pr_count<<<1184, 32 * warps_per_cta, warps_per_cta * B * sizeof(unsigned), s>>>(rp, col, Vf, S, B, off);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, off, off, (size_t)n + 1, s);
+    if (e != cudaSuccess) return e;
+    if (pcol) {
+        k_pr_scatter<<<1184, 32 * warps_per_cta, warps_per_cta * B * sizeof(unsigned long long), s>>>(rp, col, Vf, S, B,
+                                                                                                      off, pcol);
+    }
+    k_pr_flags<<<1184, 256, 0, s>>>(off, n, flag);
+    e = cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, flag, pos, (size_t)n + 1, s);
+    if (e != cudaSuccess) return e;
+    k_pr_emit<<<1184, 256, 0, s>>>(off, pos, n, Vf, chunk, q_v, q_off, tile);
+    unsigned Q = 0;
+    e = cudaMemcpyAsync(&Q, pos + n, 4, cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) return e;
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return e;
+    *h_Q = Q;
+    e = cudaMemcpyAsync(q_off + Q, &Ef, 8, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return e;
+    e = cudaStreamSynchronize(s);  // Ef is a by-value host local
+    (void)e;
+    return cudaGetLastError();
+}
+
 __global__ void k_count_dangling(const unsigned long long* rp, unsigned V, unsigned long long* cnt) {
     unsigned long long c = 0;
     for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)

@@ -83,7 +83,7 @@ def test_forced_modes_and_stealing(alg):
 
 
 def test_stealing_happens_and_balances():
-    g = inputs.rmat(15, 16, seed=9, scramble=False, weighted=False)
+    g = inputs.rmat(18, 16, seed=9, scramble=False, weighted=False)  # enough chunks to outlast a worker's CTAs
     s = inputs.pick_source(g, 9)
     csr = csr_of(g)
     ref = oracle.run("bfs", g, s)
@@ -170,3 +170,13 @@ def test_repeated_runs_reuse_context():
             assert np.array_equal(ctx.result(), oracle.bfs(adj, s))
         ctx.run("wcc")
         assert np.array_equal(ctx.result(), oracle.wcc(g.num_vertices, g.src, g.dst))
+
+
+@pytest.mark.parametrize("P", [1, 3])
+def test_pr_destination_blocked_queue(monkeypatch, P):
+    """Force the PR destination blocking (8 KiB acc blocks -> many blocks) and check parity."""
+    monkeypatch.setenv("GUM_PR_BLOCK_BYTES", "8192")
+    g = inputs.rmat(13, 16, seed=31, weighted=False)
+    ref = oracle.run("pr", g)
+    out, st, _ = check(g, "pr", 0, ref=ref, num_gpus=P, part="random" if P > 1 else "seg", seed=3)
+    assert st.vertices_frontier > 20 * np.count_nonzero(np.bincount(g.src, minlength=g.num_vertices))
