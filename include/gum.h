@@ -57,6 +57,9 @@ typedef enum { GUM_PART_SEG = 0, GUM_PART_RANDOM = 1 } gum_part;
 #define GUM_CFG_HOST_LOOP 0x2u    /* drive iterations from the host instead of a CUDA-graph WHILE node */
 #define GUM_CFG_FORCE_SPARSE 0x4u /* filter always compacts the activation list (never the bitmap) */
 #define GUM_CFG_FORCE_DENSE 0x8u  /* filter always scans the bitmap */
+#define GUM_CFG_SPLIT_UNITS 0x20u /* one launch unit (stream, control replica, kernels) per worker even
+                                     when workers share a device: runs the multi-device code path
+                                     (per-unit decisions, cross-unit barriers) on one GPU */
 #define GUM_CFG_PROFILE 0x10u     /* host loop, one iteration per poll, CUDA events around every kernel
                                      launch (read back with gum_profile); for measurement only */
 

@@ -28,7 +28,7 @@ PARTS = {"seg": 0, "random": 1}
 INF = 0xFFFFFFFF
 MAX_WORKERS = 8
 
-CFG_TRACE, CFG_HOST_LOOP, CFG_FORCE_SPARSE, CFG_FORCE_DENSE, CFG_PROFILE = 0x1, 0x2, 0x4, 0x8, 0x10
+CFG_TRACE, CFG_HOST_LOOP, CFG_FORCE_SPARSE, CFG_FORCE_DENSE, CFG_PROFILE, CFG_SPLIT_UNITS = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20
 LOAD_DEVICE = 0x1
 
 # exported symbols of include/gum.h (tests check the .so exports exactly these)
@@ -170,7 +170,7 @@ class Context:
 
     def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                  osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, force_mode=None, use_torch_allocator=False, streams=None):
+                 trace=False, host_loop=False, profile=False, split_units=False, force_mode=None, use_torch_allocator=False, streams=None):
         lib = load_library()
         cfg = gum_config()
         lib.gum_config_default(ctypes.byref(cfg))
@@ -196,6 +196,8 @@ class Context:
             flags |= CFG_HOST_LOOP
         if profile:
             flags |= CFG_PROFILE
+        if split_units:
+            flags |= CFG_SPLIT_UNITS
         if force_mode == "sparse":
             flags |= CFG_FORCE_SPARSE
         elif force_mode == "dense":

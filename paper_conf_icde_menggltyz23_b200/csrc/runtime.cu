@@ -64,6 +64,7 @@ struct gum_ctx {
     int P = 1;
     int dev[kMaxW] = {0};
     bool single_device = true;
+    bool split = false;  // one launch unit per worker (multi-device, or GUM_CFG_SPLIT_UNITS on one device)
     int n_units = 1;
     cudaStream_t stream[kMaxW] = {nullptr};
     bool own_stream[kMaxW] = {false};
@@ -194,8 +195,8 @@ void drop_partition(gum_ctx* c) {
 }
 
 // unit u covers workers [unit_w0(u), unit_w0(u)+unit_nw(u))
-int unit_w0(const gum_ctx* c, int u) { return c->single_device ? 0 : u; }
-int unit_nw(const gum_ctx* c, int u) { return c->single_device ? c->P : 1; }
+int unit_w0(const gum_ctx* c, int u) { return c->split ? u : 0; }
+int unit_nw(const gum_ctx* c, int u) { return c->split ? 1 : c->P; }
 int unit_dev(const gum_ctx* c, int u) { return c->dev[unit_w0(c, u)]; }
 
 LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
@@ -207,6 +208,7 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     if (grid < L.nw) grid = L.nw;
     L.adv_grid = grid;
     L.filter_grid = std::max(1, (c->nsm * 4) / (c->single_device ? std::min(c->P, 4) : 1));
+    if (c->split && c->single_device) L.adv_grid = std::max(1, L.adv_grid / c->P);
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
     return L;
@@ -255,7 +257,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         d.lb[f] = c->lb[f];
     }
     for (int w = 0; w < c->P; w++) {
-        int u = c->single_device ? 0 : w;
+        int u = c->split ? w : 0;
         d.rctl[w] = c->rctl[unit_w0(c, u)];
         d.trace[w] = c->trace[unit_w0(c, u)];
     }
@@ -400,7 +402,7 @@ gum_status build_pr(gum_ctx* c) {
     for (int f = 0; f < c->P; f++) {
         FragBufs& F = c->fr[f];
         CK(cudaSetDevice(F.dev));
-        cudaStream_t s = c->stream[c->single_device ? 0 : f];
+        cudaStream_t s = c->stream[c->split ? f : 0];
         const unsigned long long cap = std::min<unsigned long long>((unsigned long long)B * F.V, F.E) + 1;
         F.pr_col = B > 1 ? (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.E, 1) * 4, c->part_allocs) : F.col;
         F.pr_q_v = (unsigned*)dalloc(c, F.dev, cap * 4, c->part_allocs);
@@ -519,7 +521,8 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
                     return GUM_EUNSUP;  // mixed: some workers share a device, others do not
                 }
     }
-    c->n_units = c->single_device ? 1 : c->P;
+    c->split = !c->single_device || ((cfg->flags & GUM_CFG_SPLIT_UNITS) && c->P > 1);
+    c->n_units = c->split ? c->P : 1;
     for (int u = 0; u < c->n_units; u++) {
         int d = unit_dev(c, u);
         int w0 = unit_w0(c, u);
@@ -869,8 +872,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     }
     const double D0 = (double)c->n_dangling / (double)c->V;
     const bool profile = (c->cfg.flags & GUM_CFG_PROFILE) != 0;
-    if (profile && !c->single_device) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single device");
-    const bool graph_mode = c->single_device && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
+    if (profile && c->n_units > 1) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single launch unit");
+    const bool graph_mode = c->n_units == 1 && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
     for (auto e : c->prof_ev) cudaEventDestroy(e);
     c->prof_ev.clear();
     c->prof_kind.clear();
@@ -976,7 +979,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         }
         if (alg == GUM_PR) {
             stats->edges_frontier = qedges_total * R.iter;
-            stats->vertices_frontier *= R.iter;
+            stats->vertices_frontier = 0;
+            for (int f = 0; f < c->P; f++) stats->vertices_frontier += c->fr[f].pr_qlen * R.iter;
         }
         CK(cudaSetDevice(c->dev[0]));
     }
@@ -989,7 +993,7 @@ static gum_status gather_result(gum_ctx* c, void* dst_dev) {
     const DevCtx d = make_devctx(c, c->last_alg);
     for (int f = 0; f < c->P; f++) {
         CK(cudaSetDevice(c->fr[f].dev));
-        CK(launch_gather(d, f, dst_dev, pr, c->stream[c->single_device ? 0 : f], c->nsm * 4));
+        CK(launch_gather(d, f, dst_dev, pr, c->stream[c->split ? f : 0], c->nsm * 4));
     }
     return sync_all(c);
 }
@@ -1037,7 +1041,7 @@ gum_status gum_trace(const gum_ctx* cc, gum_iter_trace* out, uint32_t max_record
         CK(cudaSetDevice(c->dev[0]));
         CK(cudaMemcpy(out, c->trace[0], n * sizeof(gum_iter_trace), cudaMemcpyDeviceToHost));
         // multi-device: worker w's busy window and edge counts live in its own unit's buffer
-        if (!c->single_device) {
+        if (c->split) {
             std::vector<gum_iter_trace> tmp(n);
             for (int w = 1; w < c->P; w++) {
                 CK(cudaSetDevice(c->dev[w]));

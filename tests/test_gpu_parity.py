@@ -172,6 +172,25 @@ def test_repeated_runs_reuse_context():
         assert np.array_equal(ctx.result(), oracle.wcc(g.num_vertices, g.src, g.dst))
 
 
+@pytest.mark.parametrize("alg", ALGS)
+def test_split_units_multi_device_path(alg, monkeypatch):
+    """GUM_CFG_SPLIT_UNITS: one launch unit (stream + control replica) per worker on one GPU, i.e. the
+    multi-device driver (host loop, cross-unit event barriers, redundant per-unit decisions, per-unit
+    filter ownership after OSteal) with local instead of P2P pointers."""
+    monkeypatch.setenv("GUM_PR_BLOCK_BYTES", "16384")
+    g = inputs.rmat(13, 16, seed=41, scramble=False)
+    s = inputs.pick_source(g, 41)
+    ref = oracle.run(alg, g, s)
+    csr = csr_of(g)
+    for kw in (dict(num_gpus=2), dict(num_gpus=4, part="random", seed=9),
+               dict(num_gpus=4, osteal_threshold=1 << 30, osteal_edges_per_worker=20000),
+               dict(num_gpus=3, chunk_edges=64, trace=True)):
+        out, st, tr = check(g, alg, s, csr=csr, ref=ref, split_units=True, **kw)
+        if tr:
+            for r in tr:
+                assert sum(r["edges_own"]) + sum(r["edges_stolen"]) == r["frontier_edges"]
+
+
 @pytest.mark.parametrize("P", [1, 3])
 def test_pr_destination_blocked_queue(monkeypatch, P):
     """Force the PR destination blocking (8 KiB acc blocks -> many blocks) and check parity."""
