@@ -75,10 +75,11 @@ typedef struct {
     int fsteal;
     uint64_t t1_min_max_edges;
     uint64_t t2_min_spread_edges;
-    /* OSteal (§IV): when the global number of active vertices drops below osteal_active_threshold
-     * the active owner set shrinks to m' = clamp(ceil(active_edges / osteal_edges_per_worker), 1, m)
-     * survivors {0..m'-1} (uniform NVSwitch reduction tree, reading #13); shrink-only.
-     * osteal_edges_per_worker = 0 => m' = 1. */
+    /* OSteal (§IV): re-decided every iteration from the global counts. While the number of active
+     * vertices is below osteal_active_threshold the active owners are the survivors {0..m'-1}
+     * (uniform NVSwitch reduction tree, reading #13), m' = clamp(ceil(active_edges /
+     * osteal_edges_per_worker), 1, num_gpus) (0 => m' = 1); above it ownership is given back.
+     * Fragment f is owned by worker f if f < m', else by f mod m'. */
     int osteal;
     uint64_t osteal_active_threshold;
     uint64_t osteal_edges_per_worker;
@@ -89,6 +90,17 @@ typedef struct {
     double pr_damping;   /* 0 => 0.85 */
     uint32_t max_iterations; /* safety cap on BSP iterations, 0 => 2^31 */
     uint32_t flags;      /* GUM_CFG_* */
+    /* SSSP frontier split (near-far, Davidson et al. = the paper's ref [46]): activated vertices
+     * with dist >= T are parked in a far set; when the near frontier empties T moves to
+     * min(far dist) + sssp_delta and the far set is swept. 0 = plain BSP frontier (the paper's GUM).
+     * Results are identical either way (unique fixpoint); only the amount of re-relaxation changes. */
+    uint32_t sssp_delta;
+    /* Long-tail engine = OSteal's m'=1 mode (needs osteal=1 and a single launch unit):
+     * when the global frontier has <= tail_vertices vertices, worker 0 takes ownership of every
+     * fragment and one cooperative persistent kernel runs iterations back to back with one grid
+     * barrier each, until the frontier exceeds 4*tail_vertices or converges; ownership is then given
+     * back. 0 = off; gum_config_default sets 8192. */
+    uint32_t tail_vertices;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);
@@ -113,7 +125,9 @@ typedef struct {
     uint64_t activations;     /* vertices appended to next frontiers */
     uint64_t vertices_frontier; /* sum over iterations of |f_k| (queue entries expanded) */
     uint32_t final_owners;    /* active owners at the end (OSteal) */
-    uint32_t osteal_iteration;/* iteration of the last owner-set shrink (0 = never) */
+    uint32_t osteal_iteration;/* iteration of the last owner-set change (0 = never) */
+    uint32_t tail_iterations; /* of `iterations`, run inside the tail engine */
+    uint32_t bodies;          /* iteration bodies (filter/control/advance/tail launches) executed */
     double pr_last_residual;  /* PR: sum_v |x_K - x_{K-1}| */
 } gum_run_stats;
 
@@ -183,8 +197,8 @@ gum_status gum_trace(const gum_ctx* ctx, gum_iter_trace* out, uint32_t max_recor
 /* Per-kernel device time of the last run, from CUDA events recorded on the launching stream around
  * every launch (only with GUM_CFG_PROFILE; single-device). */
 typedef struct {
-    double filter_ms, control_ms, advance_ms, finalize_ms, init_ms;
-    uint32_t filter_launches, control_launches, advance_launches, finalize_launches, init_launches;
+    double filter_ms, control_ms, advance_ms, finalize_ms, init_ms, tail_ms;
+    uint32_t filter_launches, control_launches, advance_launches, finalize_launches, init_launches, tail_launches;
 } gum_kernel_times;
 gum_status gum_profile(const gum_ctx* ctx, gum_kernel_times* out);
 

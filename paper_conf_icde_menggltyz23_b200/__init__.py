@@ -53,7 +53,9 @@ class gum_config(ctypes.Structure):
                 ("t2_min_spread_edges", ctypes.c_uint64), ("osteal", ctypes.c_int),
                 ("osteal_active_threshold", ctypes.c_uint64), ("osteal_edges_per_worker", ctypes.c_uint64),
                 ("chunk_edges", ctypes.c_uint32), ("pr_iterations", ctypes.c_int), ("pr_damping", ctypes.c_double),
-                ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("alloc", ALLOC_FN),
+                ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("sssp_delta", ctypes.c_uint32),
+                ("tail_vertices", ctypes.c_uint32),
+                ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
 
@@ -63,15 +65,16 @@ class gum_run_stats(ctypes.Structure):
                 ("chunks_stolen", ctypes.c_uint64), ("chunks_total", ctypes.c_uint64),
                 ("remote_updates", ctypes.c_uint64), ("activations", ctypes.c_uint64),
                 ("vertices_frontier", ctypes.c_uint64), ("final_owners", ctypes.c_uint32), ("osteal_iteration", ctypes.c_uint32),
+                ("tail_iterations", ctypes.c_uint32), ("bodies", ctypes.c_uint32),
                 ("pr_last_residual", ctypes.c_double)]
 
 
 class gum_kernel_times(ctypes.Structure):
     _fields_ = [("filter_ms", ctypes.c_double), ("control_ms", ctypes.c_double), ("advance_ms", ctypes.c_double),
-                ("finalize_ms", ctypes.c_double), ("init_ms", ctypes.c_double),
+                ("finalize_ms", ctypes.c_double), ("init_ms", ctypes.c_double), ("tail_ms", ctypes.c_double),
                 ("filter_launches", ctypes.c_uint32), ("control_launches", ctypes.c_uint32),
                 ("advance_launches", ctypes.c_uint32), ("finalize_launches", ctypes.c_uint32),
-                ("init_launches", ctypes.c_uint32)]
+                ("init_launches", ctypes.c_uint32), ("tail_launches", ctypes.c_uint32)]
 
 
 class gum_iter_trace(ctypes.Structure):
@@ -162,6 +165,8 @@ class RunStats:
     vertices_frontier: int
     final_owners: int
     osteal_iteration: int
+    tail_iterations: int
+    bodies: int
     pr_last_residual: float
 
 
@@ -170,7 +175,7 @@ class Context:
 
     def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                  osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, split_units=False, force_mode=None, use_torch_allocator=False, streams=None):
+                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, force_mode=None, use_torch_allocator=False, streams=None):
         lib = load_library()
         cfg = gum_config()
         lib.gum_config_default(ctypes.byref(cfg))
@@ -189,6 +194,8 @@ class Context:
         cfg.pr_iterations = int(pr_iterations)
         cfg.pr_damping = float(pr_damping)
         cfg.max_iterations = int(max_iterations)
+        cfg.sssp_delta = int(sssp_delta)
+        cfg.tail_vertices = int(tail_vertices)
         flags = 0
         if trace:
             flags |= CFG_TRACE

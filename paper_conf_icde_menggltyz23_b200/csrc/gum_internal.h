@@ -41,6 +41,10 @@ struct alignas(128) FragCtl {
     unsigned long long remote_updates; // updates issued by this fragment's owner to other fragments
     unsigned long long activations;
     unsigned long long frontier_vertices; // sum over iterations of qlen
+    unsigned long long far_cnt;        // SSSP near-far: vertices currently parked in the far set
+    unsigned int far_min[2];           // SSSP near-far: min distance of far vertices, by sweep parity
+    unsigned int tcnt[3];              // tail engine: list counters (current / next / next-but-one)
+    unsigned long long tedges[3];      // tail engine: out-edges of the listed vertices
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
@@ -50,6 +54,14 @@ struct alignas(128) RunCtl {
     unsigned int done;
     unsigned int m;           // active owners (OSteal): workers {0..m-1}
     unsigned int steal_ok;    // FSteal gate for the current advance
+    unsigned int tail;        // tail engine active for the current iteration (k_tail runs it)
+    unsigned int tbar_cnt, tbar_gen;  // tail engine grid barrier
+    unsigned int tsplit_cnt[2];       // tail engine: high-degree vertices deferred to the split phase
+    unsigned int tail_iters;  // iterations run by the tail engine (stats)
+    unsigned int bodies;      // iteration bodies executed (control launches that did work)
+    unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
+    unsigned int nf_sweeps;   // number of threshold bumps so far (far_min slot parity)
+    unsigned long long nf_T;  // SSSP near-far: current split distance (near iff dist < nf_T)
     unsigned int next_dense;  // the current advance only sets bitmap bits (next filter scans the bitmap)
                               // instead of appending to the activation list
     unsigned int owner[kMaxW];// fragment -> worker (P_OSteal vector O)
@@ -69,6 +81,12 @@ struct alignas(64) LBSlot {
     unsigned long long inc_cnt, inc_deg;
 };
 
+// Tail engine split-list entry: a high-degree vertex expanded by all warps in segments.
+struct TailSplit {
+    unsigned f, v, sval, pad;
+    unsigned long long s0, s1;
+};
+
 struct FragPtrs {
     const unsigned long long* row_ptr;  // [V_f + 1], rebased to 0
     const unsigned int* col;            // [E_f] global (relabelled) destination ids
@@ -80,6 +98,8 @@ struct FragPtrs {
     const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
     unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
     unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
+    unsigned int* bm2;                  // [ceil(V_f/32)] tail engine: dedupe bits of odd-iteration lists
+    unsigned int* far;                  // [ceil(V_f/32)] SSSP near-far: parked (far) vertices
     unsigned int* app;                  // [V_f] activation list (sparse next frontier)
     unsigned int* q_v;                  // [V_f] frontier queue (local ids, out-degree > 0)
     unsigned long long* q_off;          // [V_f + 1] exclusive prefix of out-degrees over the queue
@@ -98,6 +118,7 @@ struct DevCtx {
     LBSlot* lb[kMaxW];          // per fragment: look-back slots in the filtering unit's memory
     unsigned int lb_parts;      // slots per fragment
     gum_iter_trace* trace[kMaxW];  // per worker's unit (nullable)
+    TailSplit* tsplit[kMaxW];      // per unit: tail engine split list (kTailSplitCap entries)
     unsigned int bounds[kMaxW + 1];
     int P;                      // fragments == workers
     unsigned int chunk;         // edges per chunk
@@ -109,6 +130,9 @@ struct DevCtx {
     double pr_d;
     unsigned int force_mode;    // 0 auto, 1 sparse, 2 dense
     unsigned int dense_div;     // dense filter iff app_cnt > V_f / dense_div
+    unsigned int nf_delta;      // SSSP near-far split increment (0 = plain BSP frontier, the paper's)
+    unsigned int tail_enter;    // tail engine: enter when the frontier has <= tail_enter vertices (0 = off)
+    unsigned int tail_exit;     // tail engine: hand back when the next frontier exceeds tail_exit vertices
 };
 
 }  // namespace gum

@@ -83,6 +83,8 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
             }
             F.bm[i] = wv;
             if (ALG == ALG_BFS) F.vis[i] = 0u;
+            F.bm2[i] = 0u;
+            if (ALG == ALG_SSSP) F.far[i] = 0u;
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -100,6 +102,8 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->edges_done = ct->edges_stolen = ct->chunks_stolen = ct->chunks_done = 0;
         ct->frontier_edges = ct->remote_updates = ct->activations = 0;
         ct->frontier_vertices = 0;
+        ct->far_cnt = 0;
+        ct->far_min[0] = ct->far_min[1] = GUM_INF;
     }
 }
 
@@ -130,6 +134,14 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     rc->epoch = rc->epoch + 1;
     rc->pr_D = D0;
     rc->pr_resid = 0.0;
+    rc->nf_sweep = 0;
+    rc->nf_sweeps = 0;
+    rc->tail = 0;
+    rc->tbar_cnt = 0;
+    rc->tail_iters = 0;
+    rc->bodies = 0;
+    rc->tsplit_cnt[0] = rc->tsplit_cnt[1] = 0;
+    rc->nf_T = c.nf_delta ? (unsigned long long)c.nf_delta : 0xFFFFFFFFull;
 }
 
 // ------------------------------------------------------------------------------------------ filter
@@ -194,6 +206,25 @@ __device__ __forceinline__ unsigned long long warp_excl_scan_u64(unsigned long l
     return inc - x;
 }
 
+// SSSP near-far classification of an activated vertex with out-degree > 0 (phase 1 of the filter):
+// near (dist < T) -> returns true and leaves the far set; far -> parked (bit set), counted, and its
+// distance folded into this sweep epoch's far minimum.
+__device__ __forceinline__ bool nf_classify(const FragPtrs& F, FragCtl* ct, unsigned v, unsigned T, unsigned slot) {
+    const unsigned dist = F.state[v];
+    const unsigned bit = 1u << (v & 31);
+    if (dist >= T) {
+        const unsigned ob = atomicOr(F.far + (v >> 5), bit);
+        if (!(ob & bit)) atomicAdd(&ct->far_cnt, 1ull);
+        atomicMin(&ct->far_min[slot], dist);
+        return false;
+    }
+    if (F.far[v >> 5] & bit) {
+        const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
+        if (ob & bit) atomicAdd(&ct->far_cnt, ~0ull);  // -1
+    }
+    return true;
+}
+
 __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
     if (vload(&rc->done)) return;
@@ -203,7 +234,12 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
     const FragPtrs& F = c.f[f];
     FragCtl* ct = F.ctl;
     // the advance that produced these activations either appended them (sparse) or only set bits
-    const bool dense = vload(&rc->next_dense) != 0;
+    // SSSP near-far: only vertices with dist < T enter the queue; the rest are parked in F.far
+    const bool nf = c.nf_delta != 0;
+    const bool sweep = nf && vload(&rc->nf_sweep) != 0;
+    const unsigned nfT = nf ? (unsigned)(rc->nf_T < 0xFFFFFFFFull ? rc->nf_T : 0xFFFFFFFFull) : GUM_INF;
+    const unsigned fslot = rc->nf_sweeps & 1u;
+    const bool dense = sweep || vload(&rc->next_dense) != 0;
     const unsigned app_cnt = dense ? 0u : vload(&ct->app_cnt);
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
@@ -237,6 +273,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
             if (wbase + lane < nwords) {
                 myword = F.bm[wbase + lane];
                 if (myword) F.bm[wbase + lane] = 0u;
+                if (sweep) myword |= F.far[wbase + lane];
             }
             unsigned long long wc = 0, wd = 0;
 #pragma unroll
@@ -248,6 +285,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
                     const unsigned v = (wbase + i0 + k) * 32 + lane;
                     d[k] = 0;
                     if ((wv >> lane) & 1u) d[k] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
+                    if (nf && d[k] && !nf_classify(F, ct, v, nfT, fslot)) d[k] = 0;
                 }
 #pragma unroll
                 for (int k = 0; k < 8; k++) {
@@ -269,6 +307,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
                     items[j] = v;
                     F.bm[v >> 5] = 0u;  // every set bit belongs to a listed vertex: clearing whole words is exact
                     d[j] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
+                    if (nf && d[j] && !nf_classify(F, ct, v, nfT, fslot)) d[j] = 0;
                 }
             }
 #pragma unroll
@@ -364,6 +403,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
                     if ((wv >> lane) & 1u) {
                         rp[k] = __ldg(F.row_ptr + v);
                         d[k] = __ldg(F.row_ptr + v + 1) - rp[k];
+                        if (nf && d[k] && F.state[v] >= nfT) d[k] = 0;  // parked in phase 1
                     }
                 }
 #pragma unroll
@@ -391,6 +431,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
                 if (items[j] != 0xFFFFFFFFu) {
                     rp[j] = __ldg(F.row_ptr + items[j]);
                     d[j] = __ldg(F.row_ptr + items[j] + 1) - rp[j];
+                    if (nf && d[j] && F.state[items[j]] >= nfT) d[j] = 0;  // parked in phase 1
                 }
             }
 #pragma unroll
@@ -432,6 +473,32 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             R += vload(&ct->pr_resid[(k - 1) & 1]);
         }
     }
+    // SSSP near-far: when the near frontier is empty but vertices are parked, move the split to the
+    // smallest parked distance + delta and sweep the far set in the next filter (this iteration's
+    // advance has an empty queue).
+    bool nf_bump = false;
+    if (ALG == ALG_SSSP && c.nf_delta) {
+        unsigned long long far_total = 0;
+        unsigned fmin = GUM_INF;
+        const unsigned slot = rc->nf_sweeps & 1u;
+        for (int f = 0; f < c.P; f++) {
+            far_total += vload(&c.f[f].ctl->far_cnt);
+            const unsigned fm = vload(&c.f[f].ctl->far_min[slot]);
+            fmin = fm < fmin ? fm : fmin;
+        }
+        rc->nf_sweep = 0;
+        if (active == 0 && far_total > 0 && err == 0) {
+            nf_bump = true;
+            unsigned long long T = rc->nf_T + c.nf_delta;
+            const unsigned long long T2 = (unsigned long long)fmin + c.nf_delta;
+            rc->nf_T = T2 > T ? T2 : T;
+            rc->nf_sweep = 1;
+            rc->nf_sweeps = rc->nf_sweeps + 1;
+            // the next epoch's minimum slot starts empty (only the owner resets; others read `slot`)
+            for (int f = 0; f < c.P; f++)
+                if ((int)rc->owner[f] >= w0 && (int)rc->owner[f] < w0 + nw) c.f[f].ctl->far_min[slot ^ 1u] = GUM_INF;
+        }
+    }
     bool done;
     if (ALG == ALG_PR) {
         if (k > 0) {
@@ -448,20 +515,25 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         }
         done = (int)k >= c.pr_iters;
     } else {
-        done = err != 0 || active == 0 || k >= c.max_iter;
+        done = err != 0 || (active == 0 && !nf_bump) || k >= c.max_iter;
     }
     unsigned m = rc->m;
     if (!done) {
-        // a6 OSteal: shrink the active owner set in the long tail (threshold trigger)
-        if (c.osteal && m > 1 && active < c.os_thresh) {
-            unsigned mp = 1;
-            if (c.os_epw) {
-                unsigned long long want = (total_edges + c.os_epw - 1) / c.os_epw;
-                mp = want < 1 ? 1 : (want > m ? m : (unsigned)want);
+        // a6 OSteal: the active owner set is re-decided every iteration from the global
+        // counts. Below the active-vertex threshold the survivors are {0..m'-1} (uniform-fabric
+        // reduction tree) with m' = clamp(ceil(active edges / edges-per-worker), 1, P); above it
+        // ownership is given back. Fragment f is owned by f when f < m', else by f mod m'.
+        if (c.osteal && c.P > 1) {
+            unsigned mp = (unsigned)c.P;
+            if (active < c.os_thresh) {
+                mp = 1;
+                if (c.os_epw) {
+                    const unsigned long long want = (total_edges + c.os_epw - 1) / c.os_epw;
+                    mp = want < 1 ? 1u : (want > (unsigned long long)c.P ? (unsigned)c.P : (unsigned)want);
+                }
             }
-            if (mp < m) {
-                for (int f = 0; f < c.P; f++)
-                    if (rc->owner[f] >= mp) rc->owner[f] = rc->owner[f] % mp;
+            if (mp != m) {
+                for (int f = 0; f < c.P; f++) rc->owner[f] = (unsigned)f < mp ? (unsigned)f : (unsigned)f % mp;
                 m = mp;
                 rc->m = mp;
                 rc->osteal_iter = k;
@@ -496,8 +568,26 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             r->owners = m;
             r->steal_ok = rc->steal_ok;
         }
+        // long tail: hand small frontiers to the cooperative tail engine (OSteal m'=1 engine)
+        // (OSteal's m'=1 mode: worker 0 owns every fragment while the engine runs)
+        rc->tail = 0;
+        if (ALG != ALG_PR && c.osteal && c.tail_enter && !nf_bump && active <= c.tail_enter &&
+            total_edges <= 8ull * c.tail_enter) {
+            rc->tail = 1;
+            for (int f = 0; f < c.P; f++) {
+                c.f[f].ctl->tcnt[1] = 0;
+                c.f[f].ctl->tedges[1] = 0;
+                rc->owner[f] = 0;
+            }
+            if (m != 1) rc->osteal_iter = k;
+            m = 1;
+            rc->m = 1;
+            rc->steal_ok = 0;
+            if (tr && k < (unsigned)kTraceMax) tr[k].owners = 1;
+        }
         rc->iter = k + 1;
     }
+    rc->bodies = rc->bodies + 1;
     for (int f = 0; f < kMaxW; f++) rc->ticket[f] = 0;
     rc->epoch = rc->epoch + 1;
     if (done) {
@@ -564,7 +654,7 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
     __shared__ int s_stolen;
 
     RunCtl* rc = c.rctl[w0];
-    if (vload(&rc->done)) return;
+    if (vload(&rc->done) || vload(&rc->tail)) return;  // tail engine runs this iteration
     const int w = w0 + (int)(blockIdx.x % (unsigned)nw);
     const unsigned m = rc->m;
     if ((unsigned)w >= m) return;  // evicted by OSteal: this worker's GPU only serves as memory
@@ -884,6 +974,308 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
     }
 }
 
+// ------------------------------------------------------------------------------------------ tail engine
+// The OSteal m'=1 engine of SURVEY §3: when the global frontier is small, one cooperative persistent
+// kernel runs whole BSP iterations back to back (expand -> one grid barrier -> next), so a long tail of
+// latency-bound iterations costs a barrier per iteration instead of three kernel
+// launches. Lists alternate between q_v (iteration parity 0; the filter's queue seeds it) and app;
+// three per-fragment counters rotate (current / next / reset). Semantics are the regular advance's:
+// check -> red.min -> (fence) -> bitmap test-and-set dedupe -> warp-aggregated append; a vertex's bit is
+// released (acq) before its value is read, so an improvement after the read re-activates it.
+constexpr int kTailThreads = 256;
+
+__device__ __forceinline__ void tail_barrier(RunCtl* rc, unsigned nblocks, unsigned& gen) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&rc->tbar_cnt, 1u) == nblocks - 1) {
+            rc->tbar_cnt = 0;
+            __threadfence();
+            atomicExch(&rc->tbar_gen, gen + 1);
+        } else {
+            while (vload(&rc->tbar_gen) == gen) __nanosleep(20);
+        }
+        __threadfence();
+    }
+    gen++;
+    __syncthreads();
+}
+
+constexpr unsigned kTailSplit = 256;   // vertices with more out-edges are expanded by all warps
+constexpr unsigned kTailSplitCap = 8192;
+
+// Expands edges [e_lo, e_hi) of vertex v (fragment F, value sval) with one warp: check -> red.min ->
+// dedupe on this iteration's next-list bitmap -> warp-aggregated append (+ its out-degree).
+template <int ALG, bool MULTI>
+__device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs& F, unsigned sval,
+                                                unsigned long long e_lo, unsigned long long e_hi, unsigned k,
+                                                unsigned it, unsigned ns) {
+    const unsigned lane = lane_id();
+    unsigned acts = 0;
+    for (unsigned long long eb = e_lo; eb < e_hi; eb += 32) {
+        const unsigned long long e = eb + lane;
+        bool need = false;
+        int tf = 0;
+        unsigned lu = 0;
+        if (e < e_hi) {
+            const unsigned u = __ldg(F.col + e);
+            tf = MULTI ? frag_of(c, u) : 0;
+            lu = MULTI ? u - c.bounds[tf] : u;
+            const FragPtrs& T = c.f[tf];
+            const unsigned bit = 1u << (lu & 31);
+            if (ALG == ALG_BFS) {
+                if (!(vload(T.vis + (lu >> 5)) & bit)) {
+                    const unsigned ob = atomicOr(T.vis + (lu >> 5), bit);
+                    if (!(ob & bit)) {
+                        T.state[lu] = k + 1;
+                        need = true;
+                    }
+                }
+            } else {
+                unsigned cand = sval;
+                bool ok = true;
+                if (ALG == ALG_SSSP) {
+                    const unsigned long long nd = (unsigned long long)sval + __ldg(F.w + e);
+                    if (nd >= (unsigned long long)GUM_INF) {
+                        atomicOr(&F.ctl->err, 1u);
+                        ok = false;
+                    }
+                    cand = (unsigned)nd;
+                }
+                if (ok && cand < vload(T.state + lu)) {
+                    atomicMin(T.state + lu, cand);
+                    // the next list of iteration `it` dedupes on bm (it even) / bm2 (it odd)
+                    const unsigned ob = atomicOr(((it & 1) ? T.bm2 : T.bm) + (lu >> 5), bit);
+                    need = !(ob & bit);
+                }
+            }
+        }
+        const unsigned key = need ? (unsigned)tf : 0xFFFFFFFFu;
+        const unsigned grp = MULTI ? __match_any_sync(0xffffffffu, key) : __ballot_sync(0xffffffffu, need);
+        if (need) {
+            const FragPtrs& T = c.f[tf];
+            const unsigned leader = __ffs(grp) - 1;
+            unsigned base = 0;
+            if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
+            base = __shfl_sync(grp, base, leader);
+            unsigned* nxt = (it & 1) ? T.q_v : T.app;
+            nxt[base + __popc(grp & lanemask_lt())] = lu;
+            atomicAdd(&T.ctl->tedges[ns], __ldg(T.row_ptr + lu + 1) - __ldg(T.row_ptr + lu));
+            acts++;
+        }
+    }
+    return acts;
+}
+
+template <int ALG, bool MULTI>
+__global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
+    RunCtl* rc = c.rctl[w0];
+    if (!vload(&rc->tail) || vload(&rc->done)) return;
+    const unsigned lane = lane_id();
+    const unsigned nwarps = gridDim.x * (kTailThreads / 32);
+    const unsigned gw = blockIdx.x * (kTailThreads / 32) + (threadIdx.x >> 5);
+    unsigned gen = vload(&rc->tbar_gen);
+    const unsigned k0 = rc->iter - 1;  // control already counted the first tail iteration
+    const bool nf = (ALG == ALG_SSSP) && c.nf_delta != 0;
+    const unsigned nfT = nf ? (unsigned)(rc->nf_T < 0xFFFFFFFFull ? rc->nf_T : 0xFFFFFFFFull) : GUM_INF;
+    const unsigned fslot = rc->nf_sweeps & 1u;
+    const int nfrag = MULTI ? c.P : 1;
+    gum_iter_trace* tr = c.trace[w0];
+    TailSplit* split = c.tsplit[w0];
+    // accounting: iteration k0's queue was already counted by the filter (frontier_*); later tail
+    // iterations count their own lists. edges_done counts every expanded edge (conservation).
+    unsigned long long e_done[kMaxW], e_front[kMaxW], v_front[kMaxW], a_sum = 0;
+    for (int i = 0; i < kMaxW; i++) e_done[i] = e_front[i] = v_front[i] = 0;
+    unsigned it = 0;
+    for (;; it++) {
+        const unsigned cs = it % 3, ns = (it + 1) % 3, zs = (it + 2) % 3;
+        const unsigned k = k0 + it;
+        unsigned long long it_edges = 0;
+        unsigned long long n_all = 0;
+        // ---- phase 1: one warp per listed vertex; high-degree vertices go to the split list
+        for (int f = 0; f < nfrag; f++) {
+            const FragPtrs& F = c.f[f];
+            const unsigned* cur = (it & 1) ? F.app : F.q_v;
+            const unsigned n = it == 0 ? (unsigned)vload(&F.ctl->qlen) : vload(&F.ctl->tcnt[cs]);
+            n_all += n;
+            if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
+            for (unsigned i = gw; i < n; i += nwarps) {
+                const unsigned v = cur[i];
+                const unsigned long long s0 = __ldg(F.row_ptr + v), s1 = __ldg(F.row_ptr + v + 1);
+                unsigned sval = (ALG == ALG_BFS) ? k : 0u;
+                unsigned slot = 0xFFFFFFFFu;
+                bool park = false;
+                if (lane == 0) {
+                    if (ALG != ALG_BFS) {
+                        // release the cur list's dedupe bit (reused two iterations later); any
+                        // improvement of v from now on appends it to the NEXT list (other parity)
+                        if (it > 0) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
+                        sval = vload(F.state + v);
+                        if (nf && s1 > s0) {  // like the filter, only vertices with out-edges are parked
+                            const unsigned bit = 1u << (v & 31);
+                            if (sval >= nfT) {
+                                park = true;
+                                const unsigned ob = atomicOr(F.far + (v >> 5), bit);
+                                if (!(ob & bit)) atomicAdd(&F.ctl->far_cnt, 1ull);
+                                atomicMin(&F.ctl->far_min[fslot], sval);
+                            } else if (F.far[v >> 5] & bit) {
+                                const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
+                                if (ob & bit) atomicAdd(&F.ctl->far_cnt, ~0ull);
+                            }
+                        }
+                    }
+                    if (!park) {
+                        it_edges += s1 - s0;
+                        e_done[f] += s1 - s0;
+                        if (it > 0) e_front[f] += s1 - s0;
+                        if (s1 - s0 > kTailSplit) {
+                            slot = atomicAdd(&rc->tsplit_cnt[it & 1], 1u);
+                            if (slot < kTailSplitCap) split[slot] = TailSplit{(unsigned)f, v, sval, 0u, s0, s1};
+                        }
+                    }
+                }
+                park = __shfl_sync(0xffffffffu, park ? 1u : 0u, 0) != 0;
+                if (park) continue;
+                slot = __shfl_sync(0xffffffffu, slot, 0);
+                if (slot < kTailSplitCap) continue;  // expanded cooperatively in phase 2
+                sval = __shfl_sync(0xffffffffu, sval, 0);
+                a_sum += tail_expand<ALG, MULTI>(c, F, sval, s0, s1, k, it, ns);
+            }
+        }
+        if (tr && k < (unsigned)kTraceMax) {
+            if (lane == 0 && it_edges) {
+                if (it > 0) atomicAdd((unsigned long long*)&tr[k].frontier_edges, it_edges);
+                atomicAdd((unsigned long long*)&tr[k].edges_own[0], it_edges);  // the tail's single owner
+            }
+            if (it > 0 && blockIdx.x == 0 && threadIdx.x == 0) tr[k].frontier_vertices = n_all;
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            // counters of iteration it+1's next list and split list start empty (nobody touches them
+            // before the barrier; their previous users finished before the previous barrier)
+            for (int f = 0; f < nfrag; f++) {
+                c.f[f].ctl->tcnt[zs] = 0;
+                c.f[f].ctl->tedges[zs] = 0;
+            }
+            rc->tsplit_cnt[(it + 1) & 1] = 0;
+        }
+        tail_barrier(rc, gridDim.x, gen);
+        // ---- phase 2: split vertices, 256-edge segments dealt round-robin over every warp
+        const unsigned nsplit = min(vload(&rc->tsplit_cnt[it & 1]), kTailSplitCap);
+        if (nsplit) {
+            for (unsigned sid = gw;; sid += nwarps) {
+                // locate segment sid: prefix of segment counts over the split list (warp-parallel)
+                unsigned base = 0, j = 0xFFFFFFFFu, seg = 0;
+                for (unsigned j0 = 0; j0 < nsplit && j == 0xFFFFFFFFu; j0 += 32) {
+                    unsigned cnt = 0;
+                    if (j0 + lane < nsplit) {
+                        const TailSplit& t = split[j0 + lane];
+                        cnt = (unsigned)((t.s1 - t.s0 + kTailSplit - 1) / kTailSplit);
+                    }
+                    unsigned inc = cnt;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const unsigned x = __shfl_up_sync(0xffffffffu, inc, o);
+                        if (lane >= (unsigned)o) inc += x;
+                    }
+                    const unsigned hit = __ballot_sync(0xffffffffu, cnt && sid < base + inc && sid >= base + inc - cnt);
+                    if (hit) {
+                        const unsigned l = __ffs(hit) - 1;
+                        j = j0 + l;
+                        seg = sid - (base + __shfl_sync(0xffffffffu, inc - cnt, l));
+                    }
+                    base += __shfl_sync(0xffffffffu, inc, 31);
+                }
+                if (j == 0xFFFFFFFFu) break;  // past the last segment
+                const TailSplit t = split[j];
+                const unsigned long long lo = t.s0 + (unsigned long long)seg * kTailSplit;
+                const unsigned long long hi = lo + kTailSplit < t.s1 ? lo + kTailSplit : t.s1;
+                a_sum += tail_expand<ALG, MULTI>(c, c.f[t.f], t.sval, lo, hi, k, it, ns);
+            }
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            if (tr && k + 1 < (unsigned)kTraceMax) {  // row of iteration k+1 (accumulated after the barrier)
+                gum_iter_trace* r = tr + k + 1;
+                for (int i = 0; i < kMaxW; i++) r->t_start[i] = r->t_end[i] = r->edges_own[i] = r->edges_stolen[i] = 0;
+                r->frontier_edges = 0;
+                r->frontier_vertices = 0;
+                r->owners = 1;
+                r->steal_ok = 0;
+            }
+        }
+        // appends of phase 2 (and the trace row) must be complete before the counts are read
+        if (nsplit || tr) tail_barrier(rc, gridDim.x, gen);
+        unsigned long long total_next = 0, next_edges = 0;
+        for (int f = 0; f < nfrag; f++) {
+            total_next += vload(&c.f[f].ctl->tcnt[ns]);
+            next_edges += vload(&c.f[f].ctl->tedges[ns]);
+        }
+        if (total_next == 0 || total_next > c.tail_exit || next_edges > 4ull * c.tail_exit ||
+            k + 1 >= c.max_iter || vload(&c.f[0].ctl->err))
+            break;
+    }
+    for (int f = 0; f < nfrag; f++) {
+        if (lane == 0 && e_done[f]) {
+            atomicAdd(&c.f[f].ctl->edges_done, e_done[f]);
+            if (e_front[f]) atomicAdd(&c.f[f].ctl->frontier_edges, e_front[f]);
+        }
+        if (gw == 0 && lane == 0 && v_front[f]) atomicAdd(&c.f[f].ctl->frontier_vertices, v_front[f]);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) a_sum += __shfl_xor_sync(0xffffffffu, a_sum, o);
+    if (lane == 0 && a_sum) atomicAdd(&c.f[0].ctl->activations, a_sum);
+    // hand the last produced list back to the regular path as the sparse activation list
+    if (blockIdx.x == 0) {
+        const unsigned ns = (it + 1) % 3;
+        for (int f = 0; f < nfrag; f++) {
+            const unsigned n = vload(&c.f[f].ctl->tcnt[ns]);
+            if (it & 1) {  // the last next list lives in q_v with its dedupe bits in bm2: move both
+                for (unsigned i = threadIdx.x; i < n; i += kTailThreads) {
+                    const unsigned v = c.f[f].q_v[i];
+                    c.f[f].app[i] = v;
+                    if (ALG != ALG_BFS) {
+                        atomicAnd(c.f[f].bm2 + (v >> 5), ~(1u << (v & 31)));
+                        atomicOr(c.f[f].bm + (v >> 5), 1u << (v & 31));
+                    }
+                }
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) c.f[f].ctl->app_cnt = n;
+        }
+        if (threadIdx.x == 0) {
+            rc->iter = k0 + it + 1;
+            rc->tail_iters += it + 1;
+            rc->next_dense = 0;
+            rc->tail = 0;
+            __threadfence();
+        }
+    }
+}
+
+cudaError_t tail_occupancy(int* blocks_per_sm) {
+    int a = 0, b = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_tail<ALG_SSSP, true>, kTailThreads, 0);
+    if (e != cudaSuccess) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_tail<ALG_BFS, true>, kTailThreads, 0);
+    *blocks_per_sm = a < b ? a : b;
+    return e;
+}
+
+template <int ALG>
+static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t s) {
+    if (ALG == ALG_PR || L.tail_grid <= 0) return cudaSuccess;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(L.tail_grid);
+    cfg.blockDim = dim3(kTailThreads);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;  // co-residency guaranteed (grid barrier inside)
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (c.P > 1) return cudaLaunchKernelEx(&cfg, k_tail<ALG, true>, c, L.w0);
+    return cudaLaunchKernelEx(&cfg, k_tail<ALG, false>, c, L.w0);
+}
+
 // ------------------------------------------------------------------------------------------ PR finalize
 __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
@@ -965,6 +1357,7 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
                 k_advance<ALG, false><<<L.adv_grid, kThreads, 0, s>>>(c, L.w0, L.nw);
             break;
         case KER_FINALIZE: k_pr_finalize<<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
+        case KER_TAIL: return launch_tail<ALG>(c, L, s);
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
@@ -988,7 +1381,8 @@ int phase_kernels(int alg, int phase, int* kinds) {
         }
         kinds[0] = KER_CONTROL;
         kinds[1] = KER_ADVANCE;
-        return 2;
+        kinds[2] = KER_TAIL;
+        return 3;
     }
     if (phase == 0) {
         kinds[0] = KER_CONTROL;
@@ -1001,9 +1395,10 @@ int phase_kernels(int alg, int phase, int* kinds) {
 
 cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                          cudaGraphConditionalHandle h, int use_h) {
-    int kinds[2];
+    int kinds[3];
     const int n = phase_kernels(alg, phase, kinds);
     for (int i = 0; i < n; i++) {
+        if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
         cudaError_t e = launch_kernel(alg, kinds[i], c, L, s, h, use_h);
         if (e != cudaSuccess) return e;
     }

@@ -15,9 +15,10 @@ struct LaunchCfg {
     int filter_grid;  // persistent filter CTAs per fragment
     int fin_grid;     // PR finalize CTAs per fragment
     int init_grid;
+    int tail_grid;    // tail engine CTAs (cooperative; 0 = engine disabled)
 };
 
-enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_COUNT = 5 };
+enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_COUNT = 6 };
 cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                           cudaGraphConditionalHandle h, int use_h);
 int phase_kernels(int alg, int phase, int* kinds);
@@ -27,6 +28,7 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
                         int src_frag, unsigned src_local);
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
+cudaError_t tail_occupancy(int* blocks_per_sm);
 
 // ---- setup (setup.cu): validation, partitioning, relabelling, symmetrisation -------------------
 cudaError_t setup_validate(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,

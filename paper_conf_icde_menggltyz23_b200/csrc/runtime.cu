@@ -41,6 +41,8 @@ struct FragBufs {
     double* acc = nullptr;
     unsigned* bm = nullptr;
     unsigned* vis = nullptr;
+    unsigned* bm2 = nullptr;
+    unsigned* far = nullptr;
     unsigned* app = nullptr;
     unsigned* q_v = nullptr;
     unsigned long long* q_off = nullptr;
@@ -69,6 +71,7 @@ struct gum_ctx {
     cudaStream_t stream[kMaxW] = {nullptr};
     bool own_stream[kMaxW] = {false};
     int nsm = 148;
+    int tail_occ = 1;
     int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
     std::string err;
     bool poisoned = false;
@@ -99,6 +102,7 @@ struct gum_ctx {
     LBSlot* lb[kMaxW] = {nullptr};
     unsigned lb_parts = 0;
     gum_iter_trace* trace[kMaxW] = {nullptr};
+    TailSplit* tsplit[kMaxW] = {nullptr};
     RunCtl* h_rctl = nullptr;  // pinned
     void* d_res = nullptr;
     cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -190,6 +194,7 @@ void drop_partition(gum_ctx* c) {
         c->rctl[i] = nullptr;
         c->lb[i] = nullptr;
         c->trace[i] = nullptr;
+        c->tsplit[i] = nullptr;
     }
     c->d_res = nullptr;
 }
@@ -211,6 +216,7 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     if (c->split && c->single_device) L.adv_grid = std::max(1, L.adv_grid / c->P);
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
+    L.tail_grid = (c->n_units == 1 && c->cfg.tail_vertices && alg != GUM_PR) ? c->nsm * c->tail_occ : 0;
     return L;
 }
 
@@ -237,6 +243,8 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.orig = F.orig;
         p.bm = F.bm;
         p.vis = F.vis;
+        p.bm2 = F.bm2;
+        p.far = F.far;
         p.app = F.app;
         p.q_v = F.q_v;
         p.q_off = F.q_off;
@@ -260,6 +268,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         int u = c->split ? w : 0;
         d.rctl[w] = c->rctl[unit_w0(c, u)];
         d.trace[w] = c->trace[unit_w0(c, u)];
+        d.tsplit[w] = c->tsplit[unit_w0(c, u)];
     }
     d.lb_parts = c->lb_parts;
     for (int i = 0; i <= c->P; i++) d.bounds[i] = c->bounds[i];
@@ -277,6 +286,9 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.pr_d = c->cfg.pr_damping;
     d.force_mode = (c->cfg.flags & GUM_CFG_FORCE_DENSE) ? 2u : ((c->cfg.flags & GUM_CFG_FORCE_SPARSE) ? 1u : 0u);
     d.dense_div = 32;
+    d.nf_delta = alg == GUM_SSSP ? c->cfg.sssp_delta : 0u;
+    d.tail_enter = (c->n_units == 1 && alg != GUM_PR) ? c->cfg.tail_vertices : 0u;
+    d.tail_exit = 4u * c->cfg.tail_vertices;
     return d;
 }
 
@@ -368,9 +380,10 @@ gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const Laun
         CK(launch_phase(alg, phase, d, L, s, 0, 0));
         return GUM_OK;
     }
-    int kinds[2];
+    int kinds[3];
     const int n = phase_kernels(alg, phase, kinds);
     for (int i = 0; i < n; i++) {
+        if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
         cudaEvent_t a, b;
         CK(cudaEventCreate(&a));
         CK(cudaEventCreate(&b));
@@ -479,6 +492,7 @@ void gum_config_default(gum_config* cfg) {
     cfg->chunk_edges = 2048;
     cfg->pr_iterations = 20;
     cfg->pr_damping = 0.85;
+    cfg->tail_vertices = 8192;
 }
 
 const char* gum_last_error(const gum_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
@@ -568,6 +582,11 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
             if (const char* e = getenv("GUM_ADV_CTAS_PER_SM")) c->adv_occ[a][m] = std::max(1, atoi(e));
         }
     cudaGetLastError();
+    {
+        int occ = 0;
+        if (tail_occupancy(&occ) == cudaSuccess && occ > 0) c->tail_occ = std::min(occ, 2);
+        cudaGetLastError();
+    }
     cudaEventCreate(&c->ev0);
     cudaEventCreate(&c->ev1);
     if (cudaMallocHost(&c->h_rctl, sizeof(RunCtl)) != cudaSuccess) {
@@ -779,12 +798,14 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.cx = (double*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.bm = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.vis = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
+        F.bm2 = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
+        F.far = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.app = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
         F.q_v = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
         F.q_off = (unsigned long long*)dalloc(c, F.dev, (Vn + 1) * 8, c->part_allocs);
         F.q_base = (long long*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
-        if (!F.state || !F.x || !F.acc || !F.cx || !F.bm || !F.vis || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
+        if (!F.state || !F.x || !F.acc || !F.cx || !F.bm || !F.vis || !F.bm2 || !F.far || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
             return fail(c, GUM_ENOMEM, "fragment %d state alloc failed", f);
         CK(cudaSetDevice(F.dev));
         CK(cudaMemset(F.ctl, 0, sizeof(FragCtl)));
@@ -810,7 +831,8 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
     for (int u = 0; u < c->n_units; u++) {
         int w0 = unit_w0(c, u), d = unit_dev(c, u);
         c->rctl[w0] = (RunCtl*)dalloc(c, d, sizeof(RunCtl), c->part_allocs);
-        if (!c->rctl[w0]) return fail(c, GUM_ENOMEM, "run control alloc failed");
+        c->tsplit[w0] = (TailSplit*)dalloc(c, d, 8192 * sizeof(TailSplit), c->part_allocs);
+        if (!c->rctl[w0] || !c->tsplit[w0]) return fail(c, GUM_ENOMEM, "run control alloc failed");
         CK(cudaSetDevice(d));
         CK(cudaMemset(c->rctl[w0], 0, sizeof(RunCtl)));
         if (c->cfg.flags & GUM_CFG_TRACE) {
@@ -948,6 +970,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
                 case KER_FILTER: c->prof.filter_ms += t; c->prof.filter_launches++; break;
                 case KER_CONTROL: c->prof.control_ms += t; c->prof.control_launches++; break;
                 case KER_ADVANCE: c->prof.advance_ms += t; c->prof.advance_launches++; break;
+                case KER_TAIL: c->prof.tail_ms += t; c->prof.tail_launches++; break;
                 default: c->prof.finalize_ms += t; c->prof.finalize_launches++; break;
             }
         }
@@ -962,6 +985,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         stats->final_owners = R.m;
         stats->osteal_iteration = R.osteal_iter;
         stats->pr_last_residual = R.pr_resid;
+        stats->tail_iterations = R.tail_iters;
+        stats->bodies = R.bodies;
         unsigned long long qedges_total = 0;
         for (int f = 0; f < c->P; f++) {
             FragCtl fc;
@@ -975,6 +1000,10 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->remote_updates += fc.remote_updates;
             stats->activations += fc.activations;
             stats->vertices_frontier += fc.frontier_vertices;
+            if (getenv("GUM_DEBUG"))
+                fprintf(stderr, "[gum] frag %d: V=%u E=%llu qlen=%llu edges_done=%llu frontier_edges=%llu frontier_vertices=%llu app_cnt=%u tcnt=%u,%u,%u\n",
+                        f, c->fr[f].V, (unsigned long long)(alg == GUM_WCC ? c->fr[f].sE : c->fr[f].E), fc.qlen,
+                        fc.edges_done, fc.frontier_edges, fc.frontier_vertices, fc.app_cnt, fc.tcnt[0], fc.tcnt[1], fc.tcnt[2]);
             qedges_total += fc.qedges;
         }
         if (alg == GUM_PR) {

@@ -58,12 +58,13 @@ def test_c1_bfs_sssp():
 @pytest.mark.parametrize("alg", ALGS)
 @pytest.mark.parametrize("P", [2, 4, 8])
 @pytest.mark.parametrize("part", ["seg", "random"])
-def test_virtual_workers_invariance(alg, P, part):
+@pytest.mark.parametrize("tail", [0, 8192])
+def test_virtual_workers_invariance(alg, P, part, tail):
     g = inputs.rmat(13, 16, seed=21)
     s = inputs.pick_source(g, 21)
     ref = oracle.run(alg, g, s)
     csr = csr_of(g)
-    check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P * 7)
+    check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P * 7, tail_vertices=tail)
 
 
 @pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
@@ -75,7 +76,9 @@ def test_forced_modes_and_stealing(alg):
     for kw in (dict(force_mode="sparse"), dict(force_mode="dense"), dict(fsteal=False),
                dict(chunk_edges=32, num_gpus=4), dict(num_gpus=4, osteal_threshold=1 << 30),
                dict(num_gpus=8, osteal_threshold=1 << 30, osteal_edges_per_worker=1000),
-               dict(num_gpus=4, host_loop=True), dict(num_gpus=2, use_torch_allocator=True)):
+               dict(num_gpus=4, host_loop=True), dict(num_gpus=2, use_torch_allocator=True),
+               dict(num_gpus=1, tail_vertices=0), dict(num_gpus=3, tail_vertices=16),
+               dict(num_gpus=1, tail_vertices=1 << 20), dict(num_gpus=2, profile=True, tail_vertices=64)):
         kw.setdefault("num_gpus", 4)
         out, st, _ = check(g, alg, s, csr=csr, ref=ref, **kw)
         if kw.get("osteal_threshold"):
@@ -199,3 +202,43 @@ def test_pr_destination_blocked_queue(monkeypatch, P):
     ref = oracle.run("pr", g)
     out, st, _ = check(g, "pr", 0, ref=ref, num_gpus=P, part="random" if P > 1 else "seg", seed=3)
     assert st.vertices_frontier > 20 * np.count_nonzero(np.bincount(g.src, minlength=g.num_vertices))
+
+
+@pytest.mark.parametrize("delta", [1, 37, 600, 100000])
+def test_sssp_near_far_split(delta):
+    """Near-far frontier split (sssp_delta > 0): identical distances, fewer re-relaxations on a grid."""
+    for g, s in ((inputs.rmat(13, 16, seed=51), None), (inputs.grid(96, seed=3), 0)):
+        s = inputs.pick_source(g, 51) if s is None else s
+        ref = oracle.run("sssp", g, s)
+        csr = csr_of(g)
+        base = None
+        for kw in (dict(), dict(num_gpus=4, part="random", seed=2), dict(num_gpus=3, split_units=True),
+                   dict(force_mode="sparse"), dict(num_gpus=2, osteal_threshold=500)):
+            out, st, _ = check(g, "sssp", s, csr=csr, ref=ref, sssp_delta=delta, **kw)
+            base = base or st
+        if g.name.startswith("grid") and delta <= 600:
+            _, st_plain, _ = check(g, "sssp", s, csr=csr, ref=ref)
+            assert base.edges_expanded < st_plain.edges_expanded
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
+@pytest.mark.parametrize("tail", [0, 1, 64, 8192])
+def test_tail_engine_long_chains(alg, tail):
+    """High-diameter inputs (the long-tail regime): a 3000-vertex path with shortcuts and a grid; the
+    cooperative tail engine must give the oracle's answer whether it never runs, enters/leaves every
+    iteration, or runs the whole traversal."""
+    n = 3000
+    pairs = [(i, i + 1) for i in range(n - 1)] + [(i, i + 37) for i in range(0, n - 37, 97)] + [(n - 1, 5)]
+    rng = np.random.default_rng(7)
+    w = rng.integers(1, 50, len(pairs))
+    for g, s in ((inputs.from_pairs(n, pairs, w), 0), (inputs.grid(80, seed=5), 0)):
+        ref = oracle.run(alg, g, s)
+        csr = csr_of(g)
+        for kw in (dict(), dict(num_gpus=3), dict(num_gpus=2, part="random", seed=4)):
+            _, st, _ = check(g, alg, s, csr=csr, ref=ref, tail_vertices=tail, **kw)
+            if tail == 8192 and alg != "wcc":
+                assert st.tail_iterations > 0
+            if tail == 0:
+                assert st.tail_iterations == 0
+        if alg == "sssp":
+            check(g, alg, s, csr=csr, ref=ref, tail_vertices=tail, sssp_delta=20)

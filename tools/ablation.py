@@ -1,0 +1,140 @@
+"""FSteal / OSteal ablations from the device-side per-iteration trace.
+
+FSteal: per iteration, worker w's advance busy window [t_start[w], t_end[w]] (%globaltimer, min start /
+max end over its CTAs); spread = slowest / fastest worker, starvation = sum_w (max busy - busy_w).
+Run with stealing on vs off on a statically skewed partition (unscrambled RMAT, seg ranges).
+
+OSteal: SSSP on a high-diameter grid; total time and the time spent after the active vertex count
+drops below the OSteal threshold ("long tail"), OSteal on vs off.
+
+  python tools/ablation.py --fsteal --scale 22 --workers 8 [--split]
+  python tools/ablation.py --osteal --grid 2048 --workers 8 [--split]
+"""
+import argparse
+import json
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import inputs  # noqa: E402
+import paper_conf_icde_menggltyz23_b200 as gum  # noqa: E402
+
+
+def run(csr, alg, src, reps=3, **kw):
+    rp, col, w = csr
+    with gum.Context(trace=True, **kw) as ctx:
+        ctx.load_csr(rp, col, w if alg == "sssp" else None)
+        ctx.partition("seg")
+        ctx.run(alg, src)  # warm
+        best = None
+        for _ in range(reps):
+            st = ctx.run(alg, src)
+            tr = ctx.trace()
+            if best is None or st.ms < best[0].ms:
+                best = (st, tr)
+        out = ctx.result()
+    return best[0], best[1], out
+
+
+def spread_stats(tr, P):
+    rows = []
+    for k, r in enumerate(tr):
+        busy = [(r["t_end"][w] - r["t_start"][w]) / 1e3 if r["t_end"][w] else 0.0 for w in range(P)]
+        active = [b for b in busy if b > 0]
+        if not active:
+            continue
+        mx, mn = max(active), min(active)
+        dur = (max(r["t_end"][w] for w in range(P) if r["t_end"][w]) -
+               min(r["t_start"][w] for w in range(P) if r["t_end"][w])) / 1e3
+        rows.append(dict(iter=k, frontier_edges=r["frontier_edges"], steal_ok=r["steal_ok"], owners=r["owners"],
+                         busy_us=[round(b, 1) for b in busy], spread=round(mx / mn, 3) if mn > 0 else None,
+                         starvation_us=round(sum(mx - b for b in busy), 1), advance_us=round(dur, 1),
+                         stolen_edges=sum(r["edges_stolen"])))
+    return rows
+
+
+def fsteal(args):
+    g = inputs.rmat(args.scale, 16, seed=9, scramble=False, weighted=False)
+    src = inputs.pick_source(g, 9)
+    csr = gum.build_csr(g.num_vertices, g.src, g.dst)
+    res = {}
+    for on in (True, False):
+        st, tr, out = run(csr, "bfs", src, num_gpus=args.workers, fsteal=on, split_units=args.split,
+                          chunk_edges=args.chunk)
+        rows = spread_stats(tr, args.workers)
+        big = [r for r in rows if r["frontier_edges"] >= 0.05 * max(x["frontier_edges"] for x in rows)]
+        res["on" if on else "off"] = dict(
+            run_ms=st.ms, iterations=st.iterations, chunks_stolen=st.chunks_stolen, edges_stolen=st.edges_stolen,
+            advance_us_total=round(sum(r["advance_us"] for r in rows), 1),
+            max_spread_big_iters=max((r["spread"] or 1) for r in big),
+            starvation_us_total=round(sum(r["starvation_us"] for r in rows), 1), per_iteration=rows)
+        res.setdefault("outputs", []).append(out)
+    same = bool(np.array_equal(res["outputs"][0], res["outputs"][1]))
+    del res["outputs"]
+    res["identical_outputs"] = same
+    res["workload"] = (f"BFS RMAT-{args.scale} EF16 unscrambled (hubs at low ids), seg partition, "
+                       f"{args.workers} {'split-unit' if args.split else 'virtual'} workers on 1 B200, "
+                       f"chunk {args.chunk} edges, source {src}")
+    return res
+
+
+def osteal(args):
+    g = inputs.grid(args.grid, seed=3)
+    csr = gum.build_csr(g.num_vertices, g.src, g.dst, g.w)
+    res = {}
+    thr = args.threshold
+    for on in (True, False):
+        st, tr, out = run(csr, "sssp", 0, reps=2, num_gpus=args.workers, osteal=on, osteal_threshold=thr,
+                          split_units=args.split)
+        rows = spread_stats(tr, args.workers)
+        tail = [r for r in rows if tr[r["iter"]]["frontier_vertices"] < thr]
+        res["on" if on else "off"] = dict(run_ms=st.ms, iterations=st.iterations, final_owners=st.final_owners,
+                                          osteal_iteration=st.osteal_iteration,
+                                          tail_iterations=len(tail),
+                                          tail_advance_us=round(sum(r["advance_us"] for r in tail), 1))
+        res.setdefault("outputs", []).append(out)
+    res["identical_outputs"] = bool(np.array_equal(res["outputs"][0], res["outputs"][1]))
+    del res["outputs"]
+    res["workload"] = (f"SSSP on a {args.grid}x{args.grid} grid (w in [1,255]), source 0, {args.workers} "
+                       f"{'split-unit' if args.split else 'virtual'} workers on 1 B200, OSteal threshold {thr} "
+                       f"active vertices -> m'=1")
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--fsteal", action="store_true")
+    ap.add_argument("--osteal", action="store_true")
+    ap.add_argument("--scale", type=int, default=22)
+    ap.add_argument("--grid", type=int, default=2048)
+    ap.add_argument("--workers", type=int, default=8)
+    ap.add_argument("--chunk", type=int, default=2048)
+    ap.add_argument("--threshold", type=int, default=4096)
+    ap.add_argument("--split", action="store_true")
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    out = {}
+    if args.fsteal:
+        out["fsteal"] = fsteal(args)
+        f = out["fsteal"]
+        print(f"FSteal on : {f['on']['run_ms']:.3f} ms, advance {f['on']['advance_us_total']} us, "
+              f"max spread {f['on']['max_spread_big_iters']}, starvation {f['on']['starvation_us_total']} us, "
+              f"stolen chunks {f['on']['chunks_stolen']}")
+        print(f"FSteal off: {f['off']['run_ms']:.3f} ms, advance {f['off']['advance_us_total']} us, "
+              f"max spread {f['off']['max_spread_big_iters']}, starvation {f['off']['starvation_us_total']} us")
+    if args.osteal:
+        out["osteal"] = osteal(args)
+        o = out["osteal"]
+        for k in ("on", "off"):
+            print(f"OSteal {k}: {o[k]['run_ms']:.2f} ms, {o[k]['iterations']} iterations, owners {o[k]['final_owners']}, "
+                  f"tail iterations {o[k]['tail_iterations']}, tail advance {o[k]['tail_advance_us']} us")
+    if args.out:
+        json.dump(out, open(args.out, "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()
