@@ -201,6 +201,10 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--part", default="seg")
     ap.add_argument("--fsteal", type=int, default=1)
+    ap.add_argument("--osteal", type=int, default=1)
+    ap.add_argument("--sssp-delta", type=int, default=None,
+                    help="near-far split for SSSP (default: 4096 on the C3 grid, 0 = plain BSP frontier otherwise)")
+    ap.add_argument("--tail", type=int, default=8192, help="tail engine threshold (vertices; 0 = off)")
     args = ap.parse_args()
     alg = args.alg or DEFAULT_ALG[args.config]
     rank = env_int("RANK", 0)
@@ -219,7 +223,10 @@ def main():
             dist.barrier()
 
     metric = f"{alg.upper()} GTEPS (time-to-converge per source; {args.config})"
+    sssp_delta = args.sssp_delta if args.sssp_delta is not None else (4096 if args.config == "C3" else 0)
     cfg_desc = {"workload": f"{args.config}: {WORKLOADS[args.config]}", "alg": alg, "partition": args.part,
+                "fsteal": args.fsteal, "osteal": args.osteal, "tail_engine_vertices": args.tail,
+                "sssp_near_far_delta": sssp_delta if alg == "sssp" else None,
                 "l2": "inputs larger than L2 (col array > 126 MB); no flush"}
 
     if rank != 0:
@@ -267,7 +274,8 @@ def main():
     t_csr = time.perf_counter() - t_csr
     E = g.num_edges
     dev_ids = list(range(N)) if N > 1 else None
-    ctx_kw = dict(num_gpus=N, device_ids=dev_ids, fsteal=bool(args.fsteal))
+    ctx_kw = dict(num_gpus=N, device_ids=dev_ids, fsteal=bool(args.fsteal), osteal=bool(args.osteal),
+                  sssp_delta=sssp_delta, tail_vertices=args.tail)
 
     # ---------------------------------------------------------------- device-resident timed region
     ctx = gum.Context(streams=[stream] * N if N == 1 else None, **ctx_kw)

@@ -89,7 +89,7 @@ def osteal(args):
     thr = args.threshold
     for on in (True, False):
         st, tr, out = run(csr, "sssp", 0, reps=2, num_gpus=args.workers, osteal=on, osteal_threshold=thr,
-                          split_units=args.split)
+                          split_units=args.split, sssp_delta=args.delta)
         rows = spread_stats(tr, args.workers)
         tail = [r for r in rows if tr[r["iter"]]["frontier_vertices"] < thr]
         res["on" if on else "off"] = dict(run_ms=st.ms, iterations=st.iterations, final_owners=st.final_owners,
@@ -101,7 +101,8 @@ def osteal(args):
     del res["outputs"]
     res["workload"] = (f"SSSP on a {args.grid}x{args.grid} grid (w in [1,255]), source 0, {args.workers} "
                        f"{'split-unit' if args.split else 'virtual'} workers on 1 B200, OSteal threshold {thr} "
-                       f"active vertices -> m'=1")
+                       f"active vertices; near-far delta {args.delta}; OSteal on includes the m'=1 tail engine "
+                       f"(single launch unit only)")
     return res
 
 
@@ -114,6 +115,7 @@ def main():
     ap.add_argument("--workers", type=int, default=8)
     ap.add_argument("--chunk", type=int, default=2048)
     ap.add_argument("--threshold", type=int, default=4096)
+    ap.add_argument("--delta", type=int, default=0, help="SSSP near-far split (0 = plain frontier)")
     ap.add_argument("--split", action="store_true")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
