@@ -101,6 +101,10 @@ typedef struct {
      * barrier each, until the frontier exceeds 4*tail_vertices or converges; ownership is then given
      * back. 0 = off; gum_config_default sets 8192. */
     uint32_t tail_vertices;
+    /* BFS propagation blocking for dense iterations (single fragment): 17 = bin destination ids by
+     * blocks of 2^17 and set visited bits per block in shared memory; 0 = off (the default: every edge
+     * probes the visited bitmap directly, measured faster on B200). */
+    uint32_t pb_block_log2;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);

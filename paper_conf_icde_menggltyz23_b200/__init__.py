@@ -18,7 +18,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgum.so")
+LIB_PATH = os.environ.get("GUM_LIB") or os.path.join(_HERE, "libgum.so")  # GUM_LIB: build variants (tuning)
 
 GUM_OK, GUM_EINVAL, GUM_ENOMEM, GUM_ESTATE, GUM_ERANGE, GUM_ECUDA, GUM_ENCCL, GUM_EUNSUP = 0, -1, -2, -3, -4, -5, -6, -7
 STATUS_NAMES = {0: "GUM_OK", -1: "GUM_EINVAL", -2: "GUM_ENOMEM", -3: "GUM_ESTATE", -4: "GUM_ERANGE",
@@ -54,7 +54,7 @@ class gum_config(ctypes.Structure):
                 ("osteal_active_threshold", ctypes.c_uint64), ("osteal_edges_per_worker", ctypes.c_uint64),
                 ("chunk_edges", ctypes.c_uint32), ("pr_iterations", ctypes.c_int), ("pr_damping", ctypes.c_double),
                 ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("sssp_delta", ctypes.c_uint32),
-                ("tail_vertices", ctypes.c_uint32),
+                ("tail_vertices", ctypes.c_uint32), ("pb_block_log2", ctypes.c_uint32),
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
@@ -175,7 +175,7 @@ class Context:
 
     def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                  osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, force_mode=None, use_torch_allocator=False, streams=None):
+                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, force_mode=None, use_torch_allocator=False, streams=None):
         lib = load_library()
         cfg = gum_config()
         lib.gum_config_default(ctypes.byref(cfg))
@@ -196,6 +196,7 @@ class Context:
         cfg.max_iterations = int(max_iterations)
         cfg.sssp_delta = int(sssp_delta)
         cfg.tail_vertices = int(tail_vertices)
+        cfg.pb_block_log2 = int(pb_block_log2)
         flags = 0
         if trace:
             flags |= CFG_TRACE

@@ -11,13 +11,18 @@ namespace gum {
 
 constexpr int kMaxW = GUM_MAX_WORKERS;
 constexpr int kThreads = 256;          // CTA size of advance / filter
-constexpr int kTileMax = 2048;         // max edges per claimable chunk (smem sized for it)
-constexpr int kEdgesPerThread = kTileMax / kThreads;
+#ifndef GUM_ADV_THREADS
+#define GUM_ADV_THREADS 256
+#endif
+constexpr int kAdvThreads = GUM_ADV_THREADS;  // CTA size of the advance (its barrier domain)
+constexpr int kEdgesPerThread = 8;
+constexpr int kTileMax = kAdvThreads * kEdgesPerThread;  // max edges per claimable chunk (smem sized for it)
 constexpr int kDenseWordsPerWarp = 32;                            // dense filter: bitmap words per warp
 constexpr int kDenseWordsPerPart = (kThreads / 32) * kDenseWordsPerWarp;  // 256 words = 8192 vertices
 constexpr int kFilterAppPerThread = 8;                            // sparse filter: list entries per thread
 constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;
+constexpr int kPbMaxBins = 1024;       // propagation blocking: max destination blocks per fragment
 
 // Per-fragment control block (fragment memory, peer-visible). Counters that thieves touch
 // (claim) and that the filter publishes (qlen, qedges, ntiles) live here.
@@ -59,6 +64,7 @@ struct alignas(128) RunCtl {
     unsigned int tsplit_cnt[2];       // tail engine: high-degree vertices deferred to the split phase
     unsigned int tail_iters;  // iterations run by the tail engine (stats)
     unsigned int bodies;      // iteration bodies executed (control launches that did work)
+    unsigned int pb;          // the current advance bins its discoveries (apply runs next body)
     unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
     unsigned int nf_sweeps;   // number of threshold bumps so far (far_min slot parity)
     unsigned long long nf_T;  // SSSP near-far: current split distance (near iff dist < nf_T)
@@ -95,6 +101,11 @@ struct FragPtrs {
     double* x;                          // PR [V_f]
     double* acc;                        // PR [V_f]
     double* cx;                         // PR [V_f] x[u]/outdeg(u): the value pushed along out-edges
+    // BFS propagation blocking (dense iterations): destination ids binned per block of 2^pb_shift ids
+    const unsigned long long* pb_off;   // [nb+1] static bin capacity prefix (in-degree per block)
+    unsigned int* pb_fill;              // [nb] entries written this iteration
+    unsigned int* pb_done;              // [nb] apply CTAs finished with the bin
+    unsigned int* pb_buf;               // [E_in] binned destination ids (local)
     const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
     unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
     unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
@@ -133,6 +144,8 @@ struct DevCtx {
     unsigned int nf_delta;      // SSSP near-far split increment (0 = plain BSP frontier, the paper's)
     unsigned int tail_enter;    // tail engine: enter when the frontier has <= tail_enter vertices (0 = off)
     unsigned int tail_exit;     // tail engine: hand back when the next frontier exceeds tail_exit vertices
+    unsigned int pb_shift;      // BFS propagation blocking: log2(block size); 0 = off
+    unsigned int pb_nb;         // bins of fragment 0 (single-fragment only)
 };
 
 }  // namespace gum

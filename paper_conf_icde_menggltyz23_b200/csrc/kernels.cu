@@ -141,6 +141,7 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     rc->tail_iters = 0;
     rc->bodies = 0;
     rc->tsplit_cnt[0] = rc->tsplit_cnt[1] = 0;
+    rc->pb = 0;
     rc->nf_T = c.nf_delta ? (unsigned long long)c.nf_delta : 0xFFFFFFFFull;
 }
 
@@ -568,6 +569,8 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             r->owners = m;
             r->steal_ok = rc->steal_ok;
         }
+        // BFS propagation blocking for dense iterations (single fragment)
+        rc->pb = (ALG == ALG_BFS && c.pb_shift && c.P == 1 && rc->next_dense) ? 1u : 0u;
         // long tail: hand small frontiers to the cooperative tail engine (OSteal m'=1 engine)
         // (OSteal's m'=1 mode: worker 0 owns every fragment while the engine runs)
         rc->tail = 0;
@@ -583,6 +586,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             m = 1;
             rc->m = 1;
             rc->steal_ok = 0;
+            rc->pb = 0;
             if (tr && k < (unsigned)kTraceMax) tr[k].owners = 1;
         }
         rc->iter = k + 1;
@@ -641,12 +645,18 @@ __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned
 }
 
 template <int ALG, bool MULTI>
-__global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
+__global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
     __shared__ long long s_base[kTileMax + 1];
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
     __shared__ unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
-    __shared__ unsigned s_wmax[kThreads / 32];
+    // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
+    constexpr int PBB = (ALG == ALG_BFS && !MULTI) ? kPbMaxBins : 1;
+    constexpr int PBS = (ALG == ALG_BFS && !MULTI) ? kTileMax : 1;
+    __shared__ unsigned s_pbcnt[PBB], s_pboff[PBB], s_pbg[PBB];
+    __shared__ unsigned short s_stbin[PBS];
+    unsigned* const s_stage = s_head;  // s_head is dead once the chunk's col ids are loaded
+    __shared__ unsigned s_wmax[kAdvThreads / 32];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
     __shared__ int s_f;
@@ -661,6 +671,9 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
     const unsigned k = rc->iter - 1;
     const bool steal = rc->steal_ok != 0;
     const bool next_dense = rc->next_dense != 0;
+    const bool pb = (ALG == ALG_BFS && !MULTI) && rc->pb != 0;
+    if (pb)
+        for (unsigned b = threadIdx.x; b < (unsigned)PBB; b += kAdvThreads) s_pbcnt[b] = 0;
     const unsigned long long t0 = globaltimer();
     if (threadIdx.x < (unsigned)c.P) {
         FragCtl* ct = c.f[threadIdx.x].ctl;
@@ -671,7 +684,7 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
     }
     __syncthreads();
     const unsigned CH = c.chunk;
-    for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kThreads) s_head[e] = 0;
+    for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kAdvThreads) s_head[e] = 0;
     unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0;
@@ -750,7 +763,7 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
 
         // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
         seq++;
-        for (unsigned kk = threadIdx.x; kk < nv; kk += kThreads) {
+        for (unsigned kk = threadIdx.x; kk < nv; kk += kAdvThreads) {
             const unsigned i = i0 + kk;
             const unsigned long long off = __ldcs(F.q_off + i);
             // PR's blocked queue stores edges contiguously in queue order: col index == q_off + j
@@ -800,7 +813,7 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
         VT cv[kEdgesPerThread];
 #pragma unroll
         for (int j = 0; j < kEdgesPerThread; j++) {
-            const unsigned e = j * kThreads + threadIdx.x;
+            const unsigned e = j * kAdvThreads + threadIdx.x;
             vv[j] = GUM_INF;
             cv[j] = (VT)0;
             if (e < tlen) {
@@ -834,6 +847,66 @@ __global__ void __launch_bounds__(kThreads, (ALG == ALG_BFS) ? 5 : 4) k_advance(
                     }
                     atomicAdd(c.f[tf].acc + lv, (double)cv[j]);
                 }
+            }
+        } else if (ALG == ALG_BFS && pb) {
+            // Propagation blocking (dense BFS iteration): instead of one random visited-bit probe per
+            // edge, group the chunk's destination ids by 2^pb_shift-id block (shared-memory counting
+            // sort), reserve each block's run with ONE atomic and copy it out coalesced. k_pb_apply then
+            // tests and sets the visited bits of one block in shared memory (P:236 message buffers,
+            // aggregated on chip instead of serialised).
+            const unsigned sh = c.pb_shift, nb = c.pb_nb;
+            unsigned rank[kEdgesPerThread];
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++)
+                if (vv[j] != GUM_INF) rank[j] = atomicAdd(&s_pbcnt[vv[j] >> sh], 1u);
+            __syncthreads();
+            {   // exclusive scan of the block counts (4 bins per thread) + one global reservation per bin
+                const unsigned b0 = threadIdx.x * 4;
+                unsigned cn[4], sum = 0;
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    cn[q] = (b0 + q < nb) ? s_pbcnt[b0 + q] : 0u;
+                    sum += cn[q];
+                }
+                unsigned inc = sum;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned x = __shfl_up_sync(0xffffffffu, inc, o);
+                    if (lane_id() >= (unsigned)o) inc += x;
+                }
+                if (lane_id() == 31) s_wmax[threadIdx.x >> 5] = inc;
+                __syncthreads();
+                unsigned run = inc - sum;
+                for (unsigned i = 0; i < (threadIdx.x >> 5); i++) run += s_wmax[i];
+                unsigned g[4];
+#pragma unroll
+                for (int q = 0; q < 4; q++)  // four independent reservations in flight per thread
+                    g[q] = cn[q] ? atomicAdd(&F.pb_fill[b0 + q], cn[q]) : 0u;
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    if (b0 + q < nb) {
+                        s_pboff[b0 + q] = run;
+                        s_pbg[b0 + q] = g[q];
+                        s_pbcnt[b0 + q] = 0;
+                        run += cn[q];
+                    }
+                }
+            }
+            __syncthreads();
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                if (vv[j] != GUM_INF) {
+                    const unsigned b = vv[j] >> sh;
+                    const unsigned p = s_pboff[b] + rank[j];
+                    s_stage[p] = vv[j];
+                    s_stbin[p] = (unsigned short)b;
+                }
+            }
+            __syncthreads();
+            for (unsigned p = threadIdx.x; p < tlen; p += kAdvThreads) {
+                const unsigned b = s_stbin[p];
+                F.pb_buf[F.pb_off[b] + s_pbg[b] + (p - s_pboff[b])] = s_stage[p];
+                s_stage[p] = 0;  // s_head again: its entries must not look like sequence-tagged heads
             }
         } else if (ALG == ALG_BFS) {
             // BFS: check the visited bit (1 bit/vertex, L1-cacheable) instead of the 4-byte depth.
@@ -1276,6 +1349,70 @@ static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t
     return cudaLaunchKernelEx(&cfg, k_tail<ALG, false>, c, L.w0);
 }
 
+// ------------------------------------------------------------------------------------------ PB apply
+// Second half of a propagation-blocked BFS iteration (runs first in the next body, before the filter):
+// CTA (block b, part) loads block b's visited bits (2^pb_shift bits) into shared memory, sets the bits of
+// its slice of the binned ids there, and publishes the newly set bits as visited + next-frontier bits
+// with word-wide red.or, writing depth k+1 for each new vertex. Parts of one block may both discover a
+// vertex: the bit ORs and the depth store are idempotent.
+constexpr int kPbParts = 8;
+
+__global__ void __launch_bounds__(kThreads) k_pb_apply(const __grid_constant__ DevCtx c, int w0) {
+    RunCtl* rc = c.rctl[w0];
+    if (!vload(&rc->pb) || vload(&rc->done)) return;
+    extern __shared__ unsigned s_pbw[];  // [2 * W]: working bits, original bits
+    const unsigned W = 1u << (c.pb_shift - 5);
+    unsigned* s_vis = s_pbw;
+    unsigned* s_org = s_pbw + W;
+    const FragPtrs& F = c.f[0];
+    const unsigned b = blockIdx.x / kPbParts, part = blockIdx.x % kPbParts;
+    if (b >= c.pb_nb) return;
+    const unsigned level = rc->iter;  // the advance of iteration iter-1 discovered depth iter
+    const unsigned nwords = (F.V + 31) / 32;
+    const unsigned w_lo = b * W;
+    for (unsigned w = threadIdx.x; w < W; w += kThreads) {
+        const unsigned x = (w_lo + w < nwords) ? F.vis[w_lo + w] : 0xFFFFFFFFu;
+        s_vis[w] = x;
+        s_org[w] = x;
+    }
+    __syncthreads();
+    const unsigned long long base = F.pb_off[b];
+    const unsigned n = vload(&F.pb_fill[b]);
+    const unsigned lo = (unsigned)((unsigned long long)n * part / kPbParts);
+    const unsigned hi = (unsigned)((unsigned long long)n * (part + 1) / kPbParts);
+    for (unsigned i = lo + threadIdx.x; i < hi; i += kThreads) {
+        const unsigned v = __ldcs(F.pb_buf + base + i);
+        const unsigned lw = (v >> 5) - w_lo, bit = 1u << (v & 31);
+        if (!(s_vis[lw] & bit)) atomicOr(&s_vis[lw], bit);
+    }
+    __syncthreads();
+    unsigned acts = 0;
+    for (unsigned w = threadIdx.x; w < W; w += kThreads) {
+        const unsigned nw = s_vis[w] & ~s_org[w];
+        if (!nw) continue;
+        atomicOr(F.vis + w_lo + w, nw);
+        atomicOr(F.bm + w_lo + w, nw);
+        unsigned x = nw;
+        while (x) {
+            const unsigned bb = __ffs(x) - 1;
+            x &= x - 1;
+            F.state[(w_lo + w) * 32 + bb] = level;
+            acts++;
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acts += __shfl_xor_sync(0xffffffffu, acts, o);
+    if (lane_id() == 0 && acts) atomicAdd(&F.ctl->activations, (unsigned long long)acts);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&F.pb_done[b], 1u) == kPbParts - 1) {  // last part resets the bin for next time
+            F.pb_fill[b] = 0;
+            F.pb_done[b] = 0;
+        }
+    }
+}
+
 // ------------------------------------------------------------------------------------------ PR finalize
 __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
@@ -1352,12 +1489,16 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
         case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
         case KER_ADVANCE:
             if (c.P > 1)
-                k_advance<ALG, true><<<L.adv_grid, kThreads, 0, s>>>(c, L.w0, L.nw);
+                k_advance<ALG, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             else
-                k_advance<ALG, false><<<L.adv_grid, kThreads, 0, s>>>(c, L.w0, L.nw);
+                k_advance<ALG, false><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             break;
         case KER_FINALIZE: k_pr_finalize<<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
         case KER_TAIL: return launch_tail<ALG>(c, L, s);
+        case KER_APPLY:
+            if (ALG == ALG_BFS && c.pb_shift)
+                k_pb_apply<<<c.pb_nb * kPbParts, kThreads, 2u * (1u << (c.pb_shift - 5)) * 4u, s>>>(c, L.w0);
+            break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
@@ -1376,6 +1517,11 @@ cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L
 int phase_kernels(int alg, int phase, int* kinds) {
     if (alg != ALG_PR) {
         if (phase == 0) {
+            if (alg == ALG_BFS) {
+                kinds[0] = KER_APPLY;  // second half of a propagation-blocked advance
+                kinds[1] = KER_FILTER;
+                return 2;
+            }
             kinds[0] = KER_FILTER;
             return 1;
         }
@@ -1438,7 +1584,7 @@ static void carveout() {
 
 template <int ALG, bool MULTI>
 static cudaError_t occ_of(int* n) {
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(n, k_advance<ALG, MULTI>, kThreads, 0);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(n, k_advance<ALG, MULTI>, kAdvThreads, 0);
 }
 
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm) {

@@ -18,7 +18,7 @@ struct LaunchCfg {
     int tail_grid;    // tail engine CTAs (cooperative; 0 = engine disabled)
 };
 
-enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_COUNT = 6 };
+enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_APPLY = 6, KER_COUNT = 7 };
 cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                           cudaGraphConditionalHandle h, int use_h);
 int phase_kernels(int alg, int phase, int* kinds);
@@ -29,6 +29,10 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
+// BFS propagation blocking: static per-block capacities (in-degree histogram of the blocks) -> pb_off
+cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,
+                             unsigned long long* pb_off, void* tmp, size_t tmp_bytes, cudaStream_t s);
+size_t setup_pb_tmp_bytes(unsigned nb);
 
 // ---- setup (setup.cu): validation, partitioning, relabelling, symmetrisation -------------------
 cudaError_t setup_validate(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,

@@ -57,6 +57,11 @@ struct FragBufs {
     unsigned long long* pr_q_off = nullptr;
     unsigned* pr_tile = nullptr;
     unsigned long long pr_qlen = 0, pr_qedges = 0;
+    // BFS propagation blocking
+    unsigned long long* pb_off = nullptr;
+    unsigned* pb_fill = nullptr;
+    unsigned* pb_done = nullptr;
+    unsigned* pb_buf = nullptr;
 };
 
 }  // namespace
@@ -95,6 +100,8 @@ struct gum_ctx {
     unsigned* p_w = nullptr;
     bool sym_ready = false;
     bool pr_ready = false;
+    bool pb_ready = false;
+    unsigned pb_shift = 0, pb_nb = 0;
     int pr_blocks = 1;
     FragBufs fr[kMaxW];
     unsigned long long n_dangling = 0;
@@ -184,6 +191,8 @@ void drop_partition(gum_ctx* c) {
     c->partitioned = false;
     c->sym_ready = false;
     c->pr_ready = false;
+    c->pb_ready = false;
+    c->pb_shift = c->pb_nb = 0;
     c->has_result = false;
     c->inv = nullptr;
     c->p_row_ptr = nullptr;
@@ -240,6 +249,10 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.x = F.x;
         p.acc = F.acc;
         p.cx = F.cx;
+        p.pb_off = F.pb_off;
+        p.pb_fill = F.pb_fill;
+        p.pb_done = F.pb_done;
+        p.pb_buf = F.pb_buf;
         p.orig = F.orig;
         p.bm = F.bm;
         p.vis = F.vis;
@@ -289,6 +302,8 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.nf_delta = alg == GUM_SSSP ? c->cfg.sssp_delta : 0u;
     d.tail_enter = (c->n_units == 1 && alg != GUM_PR) ? c->cfg.tail_vertices : 0u;
     d.tail_exit = 4u * c->cfg.tail_vertices;
+    d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
+    d.pb_nb = c->pb_nb;
     return d;
 }
 
@@ -443,6 +458,41 @@ gum_status build_pr(gum_ctx* c) {
     return GUM_OK;
 }
 
+// BFS propagation blocking (single fragment): per destination block of 2^17 ids, a region of the binned
+// buffer sized by the block's in-degree (an upper bound for any iteration: each edge is expanded once).
+gum_status build_pb(gum_ctx* c) {
+    if (c->pb_ready || c->P != 1 || c->cfg.pb_block_log2 == 0) return GUM_OK;
+    const unsigned shift = c->cfg.pb_block_log2;
+    if (shift != 17) return fail(c, GUM_EINVAL, "pb_block_log2 must be 0 or 17");
+    const unsigned long long nb = ((unsigned long long)c->V + (1ull << shift) - 1) >> shift;
+    if (nb > (unsigned long long)kPbMaxBins) return GUM_OK;  // too many blocks: keep the plain advance
+    FragBufs& F = c->fr[0];
+    CK(cudaSetDevice(F.dev));
+    cudaStream_t s = c->stream[0];
+    F.pb_off = (unsigned long long*)dalloc(c, F.dev, (nb + 1) * 8, c->part_allocs);
+    F.pb_fill = (unsigned*)dalloc(c, F.dev, nb * 4, c->part_allocs);
+    F.pb_done = (unsigned*)dalloc(c, F.dev, nb * 4, c->part_allocs);
+    F.pb_buf = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.E, 1) * 4, c->part_allocs);
+    std::vector<Alloc> tmp;
+    const size_t tb = setup_pb_tmp_bytes((unsigned)nb);
+    void* t = dalloc(c, F.dev, tb, tmp);
+    if (!F.pb_off || !F.pb_fill || !F.pb_done || !F.pb_buf || !t) {
+        free_list(c, tmp);
+        return fail(c, GUM_ENOMEM, "propagation-blocking buffers alloc failed");
+    }
+    CK(cudaMemsetAsync(F.pb_fill, 0, nb * 4, s));
+    CK(cudaMemsetAsync(F.pb_done, 0, nb * 4, s));
+    cudaError_t e = setup_pb_offsets(F.col, F.E, shift, (unsigned)nb, F.pb_off, t, tb, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    free_list(c, tmp);
+    if (e != cudaSuccess) return fail(c, GUM_ECUDA, "pb offsets: %s", cudaGetErrorString(e));
+    c->pb_shift = shift;
+    c->pb_nb = (unsigned)nb;
+    c->pb_ready = true;
+    drop_graphs(c);
+    return GUM_OK;
+}
+
 gum_status capture_graph(gum_ctx* c, int alg, const DevCtx& d, const LaunchCfg& L) {
     if (c->gexec[alg]) return GUM_OK;
     cudaStream_t s = c->stream[0];
@@ -493,6 +543,7 @@ void gum_config_default(gum_config* cfg) {
     cfg->pr_iterations = 20;
     cfg->pr_damping = 0.85;
     cfg->tail_vertices = 8192;
+    cfg->pb_block_log2 = 0;  // propagation blocking is opt-in (slower than the probe path)
 }
 
 const char* gum_last_error(const gum_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
@@ -503,8 +554,8 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     if (cfg->num_gpus < 1 || cfg->num_gpus > kMaxW) return GUM_EINVAL;
     gum_ctx* c = new gum_ctx();
     c->cfg = *cfg;
-    if (c->cfg.chunk_edges == 0) c->cfg.chunk_edges = kTileMax;
-    if (c->cfg.chunk_edges > (unsigned)kTileMax || c->cfg.chunk_edges % 32 != 0) {
+    if (c->cfg.chunk_edges == 0 || c->cfg.chunk_edges > (unsigned)kTileMax) c->cfg.chunk_edges = kTileMax;
+    if (c->cfg.chunk_edges % 32 != 0) {
         delete c;
         return GUM_EINVAL;
     }
@@ -869,6 +920,7 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
     if (alg == GUM_WCC) return build_sym(c);
     if (alg == GUM_PR) return build_pr(c);
+    if (alg == GUM_BFS) return build_pb(c);
     if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
     return GUM_OK;
 }

@@ -313,6 +313,37 @@ cudaError_t setup_pr_blocked(const unsigned long long* rp, const unsigned* col, 
     return cudaGetLastError();
 }
 
+// ---- BFS propagation blocking: per destination block capacity = in-degree of the block ---------
+__global__ void k_pb_hist(const unsigned* col, unsigned long long E, unsigned shift, unsigned long long* cnt) {
+    extern __shared__ unsigned s_h[];
+    const unsigned nb = blockDim.x * 4;  // caller sizes the block so that 4 * blockDim >= nb
+    for (unsigned b = threadIdx.x; b < nb; b += blockDim.x) s_h[b] = 0;
+    __syncthreads();
+    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < E;
+         e += (unsigned long long)gridDim.x * blockDim.x)
+        atomicAdd(s_h + (col[e] >> shift), 1u);
+    __syncthreads();
+    for (unsigned b = threadIdx.x; b < nb; b += blockDim.x)
+        if (s_h[b]) atomicAdd(cnt + b, (unsigned long long)s_h[b]);
+}
+
+size_t setup_pb_tmp_bytes(unsigned nb) {
+    size_t bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, bytes, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (size_t)nb + 1);
+    return bytes + 256;
+}
+
+cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,
+                             unsigned long long* pb_off, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(pb_off, 0, ((size_t)nb + 1) * 8, s);
+    if (e != cudaSuccess) return e;
+    k_pb_hist<<<1184, 256, 1024 * sizeof(unsigned), s>>>(col, E, shift, pb_off);
+    e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, pb_off, pb_off, (size_t)nb + 1, s);
+    if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+
 __global__ void k_count_dangling(const unsigned long long* rp, unsigned V, unsigned long long* cnt) {
     unsigned long long c = 0;
     for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)

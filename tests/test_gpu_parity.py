@@ -242,3 +242,13 @@ def test_tail_engine_long_chains(alg, tail):
                 assert st.tail_iterations == 0
         if alg == "sssp":
             check(g, alg, s, csr=csr, ref=ref, tail_vertices=tail, sssp_delta=20)
+
+
+@pytest.mark.parametrize("P", [1, 2])
+def test_bfs_propagation_blocking_option(P):
+    """pb_block_log2=17 (opt-in): dense BFS iterations bin destination ids and set visited bits in
+    shared memory; identical depths (the option is ignored for P > 1)."""
+    for g in (inputs.rmat(18, 16, seed=61, weighted=False), inputs.grid(200, unit_weights=True)):
+        s = inputs.pick_source(g, 61)
+        check(g, "bfs", s, num_gpus=P, pb_block_log2=17)
+        check(g, "bfs", s, num_gpus=P, pb_block_log2=17, tail_vertices=0, force_mode="dense")
