@@ -71,7 +71,11 @@ typedef struct {
     int num_gpus;
     const int* device_ids;
     /* FSteal (§III) and its gating thresholds t1, t2 (P:248 Example 5): stealing is enabled in an
-     * iteration only if max_i l_i >= t1 and max_i l_i - min_i l_i >= t2 (l_i = active edges). */
+     * iteration only if max_i l_i >= t1 and max_i l_i - min_i l_i >= t2 (l_i = active edges).
+     * fsteal = 0: off; 1: steal queue (idle workers claim chunks of the most loaded peer queue, the
+     * default); 2: planned (NEXT-2): each iteration solves Eq. (1) on the uniform fabric (closed form,
+     * see gum_fsteal_plan) and carves every queue into consecutive chunk ranges per worker (Alg. 1);
+     * used while all workers own their fragment (no OSteal shrink), else falls back to the queue. */
     int fsteal;
     uint64_t t1_min_max_edges;
     uint64_t t2_min_spread_edges;
@@ -105,6 +109,9 @@ typedef struct {
      * blocks of 2^17 and set visited bits per block in shared memory; 0 = off (the default: every edge
      * probes the visited bitmap directly, measured faster on B200). */
     uint32_t pb_block_log2;
+    /* Planned FSteal: cost of processing a remote edge relative to a local one (c_ij / c_ii of
+     * P:101-108 with uniform B_ij; 0 => 1). */
+    double fsteal_remote_cost;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);
@@ -205,6 +212,12 @@ typedef struct {
     uint32_t filter_launches, control_launches, advance_launches, finalize_launches, init_launches, tail_launches;
 } gum_kernel_times;
 gum_status gum_profile(const gum_ctx* ctx, gum_kernel_times* out);
+
+/* Host helper of the planned FSteal (NEXT-2): the LP relaxation of Eq. (1) for loads l[0..n)
+ * with local cost 1 and remote cost remote_cost (uniform fabric). Writes X[i*n+j] = edges resident on
+ * worker i assigned to worker j (row sums = loads) and *z = the min-max makespan. The device control
+ * kernel runs the same routine each iteration. */
+gum_status gum_fsteal_plan(const uint64_t* loads, int n, double remote_cost, double* X, double* z);
 
 /* Library version (major*10000 + minor*100 + patch). */
 int gum_version(void);

@@ -34,7 +34,7 @@ LOAD_DEVICE = 0x1
 # exported symbols of include/gum.h (tests check the .so exports exactly these)
 ABI_SYMBOLS = ("gum_config_default", "gum_create", "gum_destroy", "gum_last_error", "gum_build_csr",
                "gum_load_csr", "gum_partition", "gum_partition_bounds", "gum_prepare", "gum_run", "gum_result",
-               "gum_result_device", "gum_trace", "gum_profile", "gum_version")
+               "gum_result_device", "gum_trace", "gum_profile", "gum_fsteal_plan", "gum_version")
 
 
 class GumError(RuntimeError):
@@ -55,6 +55,7 @@ class gum_config(ctypes.Structure):
                 ("chunk_edges", ctypes.c_uint32), ("pr_iterations", ctypes.c_int), ("pr_damping", ctypes.c_double),
                 ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("sssp_delta", ctypes.c_uint32),
                 ("tail_vertices", ctypes.c_uint32), ("pb_block_log2", ctypes.c_uint32),
+                ("fsteal_remote_cost", ctypes.c_double),
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
@@ -111,6 +112,7 @@ def load_library():
         "gum_result_device": (i32, [vp, vp, u64]),
         "gum_trace": (i32, [vp, vp, u32, ctypes.POINTER(u32)]),
         "gum_profile": (i32, [vp, ctypes.POINTER(gum_kernel_times)]),
+        "gum_fsteal_plan": (i32, [vp, i32, ctypes.c_double, vp, ctypes.POINTER(ctypes.c_double)]),
         "gum_version": (i32, []),
     }
     for name, (res, args) in sig.items():
@@ -175,7 +177,7 @@ class Context:
 
     def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                  osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, force_mode=None, use_torch_allocator=False, streams=None):
+                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, fsteal_remote_cost=1.0, force_mode=None, use_torch_allocator=False, streams=None):
         lib = load_library()
         cfg = gum_config()
         lib.gum_config_default(ctypes.byref(cfg))
@@ -184,7 +186,8 @@ class Context:
         if device_ids is not None:
             self._dev_ids = (ctypes.c_int * len(device_ids))(*device_ids)
             cfg.device_ids = ctypes.cast(self._dev_ids, ctypes.POINTER(ctypes.c_int))
-        cfg.fsteal = int(bool(fsteal))
+        cfg.fsteal = 2 if fsteal == "planned" else int(bool(fsteal))
+        cfg.fsteal_remote_cost = float(fsteal_remote_cost)
         cfg.osteal = int(bool(osteal))
         cfg.t1_min_max_edges = int(t1)
         cfg.t2_min_spread_edges = int(t2)
@@ -326,6 +329,18 @@ class Context:
                              frontier_vertices=r.frontier_vertices, frontier_edges=r.frontier_edges,
                              owners=r.owners, steal_ok=r.steal_ok))
         return recs
+
+
+def fsteal_plan(loads, remote_cost=1.0):
+    """NEXT-2 planner (host helper of the device routine): returns (z, X) for Eq. (1) on a uniform fabric."""
+    n = len(loads)
+    l = np.ascontiguousarray(loads, dtype=np.uint64)
+    X = np.zeros(n * n, dtype=np.float64)
+    z = ctypes.c_double()
+    st = load_library().gum_fsteal_plan(_ptr(l), n, float(remote_cost), _ptr(X), ctypes.byref(z))
+    if st != GUM_OK:
+        raise GumError(st, "gum_fsteal_plan: bad arguments")
+    return z.value, X.reshape(n, n)
 
 
 def version():

@@ -50,6 +50,7 @@ struct alignas(128) FragCtl {
     unsigned int far_min[2];           // SSSP near-far: min distance of far vertices, by sweep parity
     unsigned int tcnt[3];              // tail engine: list counters (current / next / next-but-one)
     unsigned long long tedges[3];      // tail engine: out-edges of the listed vertices
+    unsigned long long pclaim[kMaxW];  // FSteal planned mode: per-worker claim counters of this queue
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
@@ -65,6 +66,8 @@ struct alignas(128) RunCtl {
     unsigned int tail_iters;  // iterations run by the tail engine (stats)
     unsigned int bodies;      // iteration bodies executed (control launches that did work)
     unsigned int pb;          // the current advance bins its discoveries (apply runs next body)
+    unsigned int plan_lo[kMaxW][kMaxW], plan_hi[kMaxW][kMaxW];  // FSteal plan: chunks [lo,hi) of queue f -> worker w
+    double plan_z;            // planned makespan (edges) of the current iteration
     unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
     unsigned int nf_sweeps;   // number of threshold bumps so far (far_min slot parity)
     unsigned long long nf_T;  // SSSP near-far: current split distance (near iff dist < nf_T)
@@ -134,7 +137,8 @@ struct DevCtx {
     int P;                      // fragments == workers
     unsigned int chunk;         // edges per chunk
     unsigned int num_vertices;  // |V|
-    int fsteal, osteal;
+    int fsteal, osteal;         // fsteal: 0 off, 1 steal queue, 2 planned (Eq. 1 / Alg. 1)
+    double remote_cost;         // planned FSteal: cost of a remote edge relative to a local one
     unsigned long long t1, t2, os_thresh, os_epw;
     unsigned int max_iter;
     int pr_iters;

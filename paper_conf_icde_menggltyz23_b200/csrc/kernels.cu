@@ -19,6 +19,7 @@
 
 #include "gum_internal.h"
 #include "kernels.h"
+#include "planner.h"
 
 namespace gum {
 
@@ -379,6 +380,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
                     ct->qedges = td;
                     ct->ntiles = (td + chunk - 1) / chunk;
                     ct->claim = 0;
+                    for (int q = 0; q < kMaxW; q++) ct->pclaim[q] = 0;
                     ct->app_cnt = 0;
                     ct->dense = dense ? 1u : 0u;
                     ct->frontier_edges += td;
@@ -549,6 +551,37 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             mn = l[i] < mn ? l[i] : mn;
         }
         rc->steal_ok = (c.fsteal && m > 1 && mx >= c.t1 && mx - mn >= c.t2) ? 1u : 0u;
+        if (c.fsteal == 2 && m == (unsigned)c.P) {
+            // NEXT-2 planned FSteal: solve Eq. (1) for this iteration's loads (closed form on a uniform
+            // fabric), then carve each queue into consecutive chunk ranges (Alg. 1 l.9-18: prefix sums of
+            // the planned edge counts searched in the queue's chunk (edge) prefix): the owner's kept
+            // share first, then each thief's share in worker order.
+            double X[kMaxW * kMaxW];
+            unsigned long long lw[kMaxW];
+            for (int f = 0; f < c.P; f++) lw[f] = l[f];
+            if (rc->steal_ok) {
+                rc->plan_z = fsteal_waterfill(lw, c.P, c.remote_cost, X);
+            } else {
+                for (int q = 0; q < c.P * c.P; q++) X[q] = 0.0;
+                for (int f = 0; f < c.P; f++) X[f * c.P + f] = (double)lw[f];
+                rc->plan_z = (double)mx;
+            }
+            for (int f = 0; f < c.P; f++) {
+                const unsigned long long nt = vload(&c.f[f].ctl->ntiles);
+                double cum = 0.0;
+                unsigned prev = 0;
+                for (int q = 0; q < c.P; q++) {
+                    const int wk = q == 0 ? f : (q <= f ? q - 1 : q);  // owner first, then others
+                    cum += X[f * c.P + wk];
+                    unsigned hi = (unsigned)(cum / (double)c.chunk + 0.5);
+                    if (q == c.P - 1 || hi > nt) hi = (unsigned)nt;
+                    if (hi < prev) hi = prev;
+                    rc->plan_lo[f][wk] = prev;
+                    rc->plan_hi[f][wk] = hi;
+                    prev = hi;
+                }
+            }
+        }
         // frontier density switch: expanding more than V/dense_div edges is expected to activate a
         // dense next frontier -> the advance only sets bitmap bits (fire-and-forget) and the next
         // filter scans the bitmap; otherwise activations are deduplicated and appended to a list.
@@ -671,6 +704,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
     const unsigned k = rc->iter - 1;
     const bool steal = rc->steal_ok != 0;
     const bool next_dense = rc->next_dense != 0;
+    const bool planned = c.fsteal == 2 && m == (unsigned)c.P;  // NEXT-2 plan (else the steal queue)
     const bool pb = (ALG == ALG_BFS && !MULTI) && rc->pb != 0;
     if (pb)
         for (unsigned b = threadIdx.x; b < (unsigned)PBB; b += kAdvThreads) s_pbcnt[b] = 0;
@@ -697,7 +731,23 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             int f = -1;
             unsigned long long t = 0;
             int stolen = 0;
-            if (pf_f >= 0 && pf_t < s_ntiles[pf_f]) {
+            if (planned) {
+                // NEXT-2: process the chunk ranges the plan assigned to this worker, queue by queue
+                while (own_cursor < c.P) {
+                    const int g = (w + own_cursor) % c.P;
+                    const unsigned lo = rc->plan_lo[g][w], hi = rc->plan_hi[g][w];
+                    if (hi > lo) {
+                        const unsigned long long tt = lo + atomicAdd(&c.f[g].ctl->pclaim[w], 1ull);
+                        if (tt < hi) {
+                            f = g;
+                            t = tt;
+                            stolen = g != w;
+                            break;
+                        }
+                    }
+                    own_cursor++;
+                }
+            } else if (pf_f >= 0 && pf_t < s_ntiles[pf_f]) {
                 f = pf_f;
                 t = pf_t;
             } else {
@@ -716,7 +766,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
                 }
             }
             pf_f = -1;
-            if (f < 0 && steal) {
+            if (f < 0 && steal && !planned) {
                 // FSteal: claim a chunk of the active owner queue with the most remaining chunks
                 for (;;) {
                     int best = -1;
@@ -743,7 +793,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             s_f = f;
             s_t = t;
             s_stolen = stolen;
-            if (f >= 0 && !stolen) {
+            if (f >= 0 && !stolen && !planned) {
                 pf_f = f;
                 pf_t = atomicAdd(&c.f[f].ctl->claim, 1ull);
             }

@@ -15,6 +15,7 @@
 #include "gum.h"
 #include "gum_internal.h"
 #include "kernels.h"
+#include "planner.h"
 
 using namespace gum;
 
@@ -289,6 +290,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.chunk = c->cfg.chunk_edges;
     d.num_vertices = c->V;
     d.fsteal = c->cfg.fsteal;
+    d.remote_cost = c->cfg.fsteal_remote_cost > 0.0 ? c->cfg.fsteal_remote_cost : 1.0;
     d.osteal = c->cfg.osteal;
     d.t1 = c->cfg.t1_min_max_edges;
     d.t2 = c->cfg.t2_min_spread_edges;
@@ -1102,6 +1104,15 @@ gum_status gum_result_device(gum_ctx* c, void* out, uint64_t out_bytes) {
     const size_t es = c->last_alg == GUM_PR ? 8 : 4;
     if (out_bytes < (uint64_t)c->V * es) return fail(c, GUM_EINVAL, "output buffer too small");
     return gather_result(c, out);
+}
+
+gum_status gum_fsteal_plan(const uint64_t* loads, int n, double remote_cost, double* X, double* z) {
+    if (!loads || !X || n < 1 || n > kMaxW) return GUM_EINVAL;
+    unsigned long long l[kMaxW];
+    for (int i = 0; i < n; i++) l[i] = loads[i];
+    const double zz = fsteal_waterfill(l, n, remote_cost > 0.0 ? remote_cost : 1.0, X);
+    if (z) *z = zz;
+    return GUM_OK;
 }
 
 gum_status gum_profile(const gum_ctx* c, gum_kernel_times* out) {

@@ -252,3 +252,25 @@ def test_bfs_propagation_blocking_option(P):
         s = inputs.pick_source(g, 61)
         check(g, "bfs", s, num_gpus=P, pb_block_log2=17)
         check(g, "bfs", s, num_gpus=P, pb_block_log2=17, tail_vertices=0, force_mode="dense")
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc", "pr"])
+def test_planned_fsteal(alg):
+    """fsteal='planned' (NEXT-2): per-iteration Eq. (1) plan + chunk carving instead of the steal queue;
+    outputs identical, every chunk processed once, and the executed per-worker loads follow the plan."""
+    g = inputs.rmat(16, 16, seed=71, scramble=False)
+    s = inputs.pick_source(g, 71)
+    ref = oracle.run(alg, g, s)
+    csr = csr_of(g)
+    for kw in (dict(num_gpus=4), dict(num_gpus=3, fsteal_remote_cost=2.0), dict(num_gpus=2, split_units=True),
+               dict(num_gpus=4, tail_vertices=0, chunk_edges=256)):
+        _, st, tr = check(g, alg, s, csr=csr, ref=ref, fsteal="planned", trace=True, **kw)
+        for r in tr:
+            assert sum(r["edges_own"]) + sum(r["edges_stolen"]) == r["frontier_edges"]
+    # balance: on the heaviest iteration the executed loads are within a few chunks of each other
+    _, st, tr = check(g, "bfs", s, csr=csr, ref=oracle.run("bfs", g, s), fsteal="planned", trace=True,
+                      num_gpus=4, tail_vertices=0, chunk_edges=256)
+    big = max(tr, key=lambda r: r["frontier_edges"])
+    done = [a + b for a, b in zip(big["edges_own"], big["edges_stolen"])]
+    assert max(done) - min(done) <= 4 * 256 + 2 * big["frontier_edges"] // 100
+    assert st.chunks_stolen > 0
