@@ -677,15 +677,16 @@ __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned
     return done;
 }
 
-template <int ALG, bool MULTI>
+template <int ALG, bool MULTI, bool PB = false>
 __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
     __shared__ long long s_base[kTileMax + 1];
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
     __shared__ unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
     // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
-    constexpr int PBB = (ALG == ALG_BFS && !MULTI) ? kPbMaxBins : 1;
-    constexpr int PBS = (ALG == ALG_BFS && !MULTI) ? kTileMax : 1;
+    constexpr int PBB = (ALG == ALG_BFS && !MULTI && PB) ? kPbMaxBins : 1;  // (own instantiation:
+    // the shared arrays would otherwise shrink L1, which the random probes of the plain path live on)
+    constexpr int PBS = (ALG == ALG_BFS && !MULTI && PB) ? kTileMax : 1;
     __shared__ unsigned s_pbcnt[PBB], s_pboff[PBB], s_pbg[PBB];
     __shared__ unsigned short s_stbin[PBS];
     unsigned* const s_stage = s_head;  // s_head is dead once the chunk's col ids are loaded
@@ -705,7 +706,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
     const bool steal = rc->steal_ok != 0;
     const bool next_dense = rc->next_dense != 0;
     const bool planned = c.fsteal == 2 && m == (unsigned)c.P;  // NEXT-2 plan (else the steal queue)
-    const bool pb = (ALG == ALG_BFS && !MULTI) && rc->pb != 0;
+    const bool pb = (ALG == ALG_BFS && !MULTI && PB) && rc->pb != 0;
     if (pb)
         for (unsigned b = threadIdx.x; b < (unsigned)PBB; b += kAdvThreads) s_pbcnt[b] = 0;
     const unsigned long long t0 = globaltimer();
@@ -1332,8 +1333,10 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
             total_next += vload(&c.f[f].ctl->tcnt[ns]);
             next_edges += vload(&c.f[f].ctl->tedges[ns]);
         }
-        if (total_next == 0 || total_next > c.tail_exit || next_edges > 4ull * c.tail_exit ||
-            k + 1 >= c.max_iter || vload(&c.f[0].ctl->err))
+        // every CTA must take the same decision: only values that are final after the barrier (next-list
+        // counters) enter it -- not the error flag, which next-iteration work of a fast CTA may already
+        // set (overflowing candidates are simply not relaxed; control reports GUM_ERANGE afterwards)
+        if (total_next == 0 || total_next > c.tail_exit || next_edges > 4ull * c.tail_exit || k + 1 >= c.max_iter)
             break;
     }
     for (int f = 0; f < nfrag; f++) {
@@ -1473,7 +1476,10 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
     const FragPtrs& F = c.f[f];
     // PR's frontier queue is static: re-arm its steal-queue head for the next advance (every
     // advance of this iteration has finished: kernel boundary / cross-device barrier)
-    if (blockIdx.x == 0 && threadIdx.x == 0) F.ctl->claim = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        F.ctl->claim = 0;
+        for (int q = 0; q < kMaxW; q++) F.ctl->pclaim[q] = 0;
+    }
     const double N = (double)c.num_vertices, d = c.pr_d, D = rc->pr_D;
     double dang = 0.0, res = 0.0;
     for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
@@ -1541,7 +1547,10 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
             if (c.P > 1)
                 k_advance<ALG, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             else
-                k_advance<ALG, false><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
+                if (ALG == ALG_BFS && c.pb_shift)
+                    k_advance<ALG, false, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
+                else
+                    k_advance<ALG, false><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             break;
         case KER_FINALIZE: k_pr_finalize<<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
         case KER_TAIL: return launch_tail<ALG>(c, L, s);

@@ -8,6 +8,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <ctime>
 #include <cstdlib>
 #include <string>
 #include <vector>
@@ -979,6 +980,20 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     if (profile) CK(cudaEventRecord(init_b, c->stream[0]));
     if (graph_mode) {
         CK(cudaGraphLaunch(c->gexec[alg], c->stream[0]));
+        if (getenv("GUM_DEBUG")) {  // watchdog: sample the run control block from a side stream
+            cudaStream_t side;
+            cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking);
+            for (int i = 0; i < 50 && cudaStreamQuery(c->stream[0]) == cudaErrorNotReady; i++) {
+                RunCtl r;
+                cudaMemcpyAsync(&r, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost, side);
+                cudaStreamSynchronize(side);
+                fprintf(stderr, "[gum] graph running: iter=%u done=%u tail=%u err=%u bodies=%u tail_iters=%u tbar=%u/%u\n",
+                        r.iter, r.done, r.tail, r.err, r.bodies, r.tail_iters, r.tbar_cnt, r.tbar_gen);
+                struct timespec ts = {0, 100000000};
+                nanosleep(&ts, nullptr);
+            }
+            cudaStreamDestroy(side);
+        }
     } else {
         // host-driven loop: launch batches of iterations, then poll the device-side done flag
         const int B = profile ? 1 : 8;
@@ -998,6 +1013,10 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             CK(cudaSetDevice(c->dev[0]));
             CK(cudaMemcpyAsync(c->h_rctl, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost, c->stream[0]));
             CK(cudaStreamSynchronize(c->stream[0]));
+            if (getenv("GUM_DEBUG"))
+                fprintf(stderr, "[gum] host loop: iter=%u done=%u tail=%u err=%u bodies=%u tail_iters=%u\n",
+                        c->h_rctl->iter, c->h_rctl->done, c->h_rctl->tail, c->h_rctl->err, c->h_rctl->bodies,
+                        c->h_rctl->tail_iters);
             if (c->h_rctl->done) break;
         }
         st = unit_barrier(c);
