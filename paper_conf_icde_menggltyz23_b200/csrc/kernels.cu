@@ -680,7 +680,7 @@ __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned
 template <int ALG, bool MULTI, bool PB = false>
 __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
-    __shared__ long long s_base[kTileMax + 1];
+    __shared__ unsigned s_base[kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
     __shared__ unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
     // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
@@ -818,7 +818,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             const unsigned i = i0 + kk;
             const unsigned long long off = __ldcs(F.q_off + i);
             // PR's blocked queue stores edges contiguously in queue order: col index == q_off + j
-            s_base[kk] = (ALG == ALG_PR) ? 0ll : __ldcs(F.q_base + i);
+            s_base[kk] = (unsigned)((long long)tb + ((ALG == ALG_PR) ? 0ll : __ldcs(F.q_base + i)));
             if (ALG == ALG_PR) {
                 const unsigned u = __ldcs(F.q_v + i);
                 s_val[kk] = (VT)__ldcg(F.cx + u);
@@ -869,7 +869,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             cv[j] = (VT)0;
             if (e < tlen) {
                 const unsigned kk = s_head[e];
-                const unsigned long long ci = (unsigned long long)((long long)(tb + e) + s_base[kk]);
+                const unsigned long long ci = (unsigned)(s_base[kk] + e);  // mod 2^32: the base may wrap
                 vv[j] = __ldcs(F.col + ci);
                 if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
                 if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];

@@ -368,6 +368,7 @@ gum_status build_sym(gum_ctx* c) {
     for (int f = 0; f < c->P; f++) {
         FragBufs& F = c->fr[f];
         F.sE = hb[f + 1] - hb[f];
+        if (F.sE >= (1ull << 32)) return fail(c, GUM_EUNSUP, "symmetric fragment %d has >= 2^32 entries", f);
         if (c->P == 1 && c->single_device) {
             F.s_row_ptr = srp;
             F.s_col = scol;
@@ -821,6 +822,7 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.base = c->bounds[f];
         F.V = c->bounds[f + 1] - c->bounds[f];
         F.E = eb[f + 1] - eb[f];
+        if (F.E >= (1ull << 32)) return fail(c, GUM_EUNSUP, "fragment %d has >= 2^32 edges: use more workers", f);
         const size_t Vn = std::max<size_t>(F.V, 1);
         if (c->P == 1 && c->single_device) {
             F.row_ptr = c->p_row_ptr;
