@@ -205,6 +205,7 @@ def main():
     ap.add_argument("--sssp-delta", type=int, default=None,
                     help="near-far split for SSSP (default: 4096 on the C3 grid, 0 = plain BSP frontier otherwise)")
     ap.add_argument("--tail", type=int, default=8192, help="tail engine threshold (vertices; 0 = off)")
+    ap.add_argument("--bfs-pull", type=int, default=0, help="NEXT-4 direction-optimising BFS (bottom-up iterations)")
     args = ap.parse_args()
     alg = args.alg or DEFAULT_ALG[args.config]
     rank = env_int("RANK", 0)
@@ -226,6 +227,7 @@ def main():
     sssp_delta = args.sssp_delta if args.sssp_delta is not None else (4096 if args.config == "C3" else 0)
     cfg_desc = {"workload": f"{args.config}: {WORKLOADS[args.config]}", "alg": alg, "partition": args.part,
                 "fsteal": args.fsteal, "osteal": args.osteal, "tail_engine_vertices": args.tail,
+                "bfs_direction_opt": bool(args.bfs_pull) if alg == "bfs" else None,
                 "sssp_near_far_delta": sssp_delta if alg == "sssp" else None,
                 "l2": "inputs larger than L2 (col array > 126 MB); no flush"}
 
@@ -275,7 +277,7 @@ def main():
     E = g.num_edges
     dev_ids = list(range(N)) if N > 1 else None
     ctx_kw = dict(num_gpus=N, device_ids=dev_ids, fsteal=bool(args.fsteal), osteal=bool(args.osteal),
-                  sssp_delta=sssp_delta, tail_vertices=args.tail)
+                  sssp_delta=sssp_delta, tail_vertices=args.tail, bfs_direction_opt=bool(args.bfs_pull))
 
     # ---------------------------------------------------------------- device-resident timed region
     ctx = gum.Context(streams=[stream] * N if N == 1 else None, **ctx_kw)

@@ -112,6 +112,10 @@ typedef struct {
     /* Planned FSteal: cost of processing a remote edge relative to a local one (c_ij / c_ii of
      * P:101-108 with uniform B_ij; 0 => 1). */
     double fsteal_remote_cost;
+    /* NEXT-4 direction-optimising BFS (Beamer et al.): 1 = build the in-CSR at gum_prepare(BFS) and run
+     * large-frontier iterations bottom-up (every unvisited vertex looks for a parent at the current
+     * depth among its in-edges). Same depths; 0 = push only (the paper's GUM, the default). */
+    int bfs_direction_opt;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);

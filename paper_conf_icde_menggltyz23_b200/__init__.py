@@ -55,7 +55,7 @@ class gum_config(ctypes.Structure):
                 ("chunk_edges", ctypes.c_uint32), ("pr_iterations", ctypes.c_int), ("pr_damping", ctypes.c_double),
                 ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("sssp_delta", ctypes.c_uint32),
                 ("tail_vertices", ctypes.c_uint32), ("pb_block_log2", ctypes.c_uint32),
-                ("fsteal_remote_cost", ctypes.c_double),
+                ("fsteal_remote_cost", ctypes.c_double), ("bfs_direction_opt", ctypes.c_int),
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
@@ -177,7 +177,7 @@ class Context:
 
     def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                  osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, fsteal_remote_cost=1.0, force_mode=None, use_torch_allocator=False, streams=None):
+                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None, use_torch_allocator=False, streams=None):
         lib = load_library()
         cfg = gum_config()
         lib.gum_config_default(ctypes.byref(cfg))
@@ -188,6 +188,7 @@ class Context:
             cfg.device_ids = ctypes.cast(self._dev_ids, ctypes.POINTER(ctypes.c_int))
         cfg.fsteal = 2 if fsteal == "planned" else int(bool(fsteal))
         cfg.fsteal_remote_cost = float(fsteal_remote_cost)
+        cfg.bfs_direction_opt = int(bool(bfs_direction_opt))
         cfg.osteal = int(bool(osteal))
         cfg.t1_min_max_edges = int(t1)
         cfg.t2_min_spread_edges = int(t2)

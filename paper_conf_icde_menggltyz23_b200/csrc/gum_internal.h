@@ -51,6 +51,7 @@ struct alignas(128) FragCtl {
     unsigned int tcnt[3];              // tail engine: list counters (current / next / next-but-one)
     unsigned long long tedges[3];      // tail engine: out-edges of the listed vertices
     unsigned long long pclaim[kMaxW];  // FSteal planned mode: per-worker claim counters of this queue
+    unsigned long long pull_checked;   // bottom-up BFS: in-edges inspected
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
@@ -63,9 +64,11 @@ struct alignas(128) RunCtl {
     unsigned int tail;        // tail engine active for the current iteration (k_tail runs it)
     unsigned int tbar_cnt, tbar_gen;  // tail engine grid barrier
     unsigned int tsplit_cnt[2];       // tail engine: high-degree vertices deferred to the split phase
+    unsigned int fbar_cnt, fbar_gen;  // filter grid barrier
     unsigned int tail_iters;  // iterations run by the tail engine (stats)
     unsigned int bodies;      // iteration bodies executed (control launches that did work)
     unsigned int pb;          // the current advance bins its discoveries (apply runs next body)
+    unsigned int pull;        // the current BFS iteration runs bottom-up (k_bfs_pull instead of advance)
     unsigned int plan_lo[kMaxW][kMaxW], plan_hi[kMaxW][kMaxW];  // FSteal plan: chunks [lo,hi) of queue f -> worker w
     double plan_z;            // planned makespan (edges) of the current iteration
     unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
@@ -109,6 +112,9 @@ struct FragPtrs {
     unsigned int* pb_fill;              // [nb] entries written this iteration
     unsigned int* pb_done;              // [nb] apply CTAs finished with the bin
     unsigned int* pb_buf;               // [E_in] binned destination ids (local)
+    // bottom-up BFS (NEXT-4 direction optimisation): in-edges of the fragment's vertices
+    const unsigned long long* in_row_ptr;  // [V_f + 1]
+    const unsigned int* in_col;            // [E_in] global source ids
     const unsigned int* orig;           // [V_f] original ids (RANDOM relabel) or null (identity)
     unsigned int* bm;                   // [ceil(V_f/32)] activation bitmap (dedupe + dense frontier)
     unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
@@ -150,6 +156,8 @@ struct DevCtx {
     unsigned int tail_exit;     // tail engine: hand back when the next frontier exceeds tail_exit vertices
     unsigned int pb_shift;      // BFS propagation blocking: log2(block size); 0 = off
     unsigned int pb_nb;         // bins of fragment 0 (single-fragment only)
+    unsigned int bfs_pull;      // direction-optimising BFS enabled (in-CSR built)
+    unsigned long long total_edges;  // sum of the fragments' out-edges
 };
 
 }  // namespace gum

@@ -105,6 +105,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->frontier_vertices = 0;
         ct->far_cnt = 0;
         ct->far_min[0] = ct->far_min[1] = GUM_INF;
+        ct->pull_checked = 0;
     }
 }
 
@@ -142,7 +143,9 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     rc->tail_iters = 0;
     rc->bodies = 0;
     rc->tsplit_cnt[0] = rc->tsplit_cnt[1] = 0;
+    rc->fbar_cnt = 0;
     rc->pb = 0;
+    rc->pull = 0;
     rc->nf_T = c.nf_delta ? (unsigned long long)c.nf_delta : 0xFFFFFFFFull;
 }
 
@@ -604,6 +607,20 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         }
         // BFS propagation blocking for dense iterations (single fragment)
         rc->pb = (ALG == ALG_BFS && c.pb_shift && c.P == 1 && rc->next_dense) ? 1u : 0u;
+        // NEXT-4 direction-optimising BFS (Beamer's rule): go bottom-up when the frontier's out-edges m_f
+        // exceed 1/14 of the edges not yet reached m_u; stay while the frontier holds >= V/24 vertices.
+        if (ALG == ALG_BFS && c.bfs_pull) {
+            unsigned long long seen = 0;
+            for (int f = 0; f < c.P; f++) seen += vload(&c.f[f].ctl->frontier_edges);
+            const unsigned long long mu = c.total_edges > seen ? c.total_edges - seen : 0;
+            const bool pull = rc->pull ? active * 24ull >= (unsigned long long)c.num_vertices
+                                       : total_edges * 14ull > mu && active * 64ull >= (unsigned long long)c.num_vertices;
+            rc->pull = pull ? 1u : 0u;
+            if (pull) {
+                rc->pb = 0;
+                rc->next_dense = 1;  // the bottom-up step writes the next frontier as bits
+            }
+        }
         // long tail: hand small frontiers to the cooperative tail engine (OSteal m'=1 engine)
         // (OSteal's m'=1 mode: worker 0 owns every fragment while the engine runs)
         rc->tail = 0;
@@ -620,6 +637,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             rc->m = 1;
             rc->steal_ok = 0;
             rc->pb = 0;
+            rc->pull = 0;
             if (tr && k < (unsigned)kTraceMax) tr[k].owners = 1;
         }
         rc->iter = k + 1;
@@ -699,6 +717,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
 
     RunCtl* rc = c.rctl[w0];
     if (vload(&rc->done) || vload(&rc->tail)) return;  // tail engine runs this iteration
+    if (ALG == ALG_BFS && vload(&rc->pull)) return;   // bottom-up step runs this iteration
     const int w = w0 + (int)(blockIdx.x % (unsigned)nw);
     const unsigned m = rc->m;
     if ((unsigned)w >= m) return;  // evicted by OSteal: this worker's GPU only serves as memory
@@ -1377,6 +1396,10 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
     }
 }
 
+cudaError_t filter_occupancy(int* blocks_per_sm) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_filter, kThreads, 0);
+}
+
 cudaError_t tail_occupancy(int* blocks_per_sm) {
     int a = 0, b = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_tail<ALG_SSSP, true>, kTailThreads, 0);
@@ -1400,6 +1423,63 @@ static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t
     cfg.numAttrs = 1;
     if (c.P > 1) return cudaLaunchKernelEx(&cfg, k_tail<ALG, true>, c, L.w0);
     return cudaLaunchKernelEx(&cfg, k_tail<ALG, false>, c, L.w0);
+}
+
+// ------------------------------------------------------------------------------------------ bottom-up
+// NEXT-4 direction-optimising BFS: in a bottom-up iteration every unvisited vertex of an owned fragment
+// looks for a parent at depth k among its in-edges and stops at the first one (a warp per 32-vertex
+// visited word, a lane per vertex). New vertices get depth k+1 and their visited and next-frontier bits
+// (one word store per warp: each word has a single writer). The frontier's out-edges are counted as
+// expanded (the result is the same BFS tree depth); pull_checked records the in-edges inspected.
+template <bool MULTI>
+__global__ void __launch_bounds__(kThreads) k_bfs_pull(const __grid_constant__ DevCtx c, int w0, int nw) {
+    RunCtl* rc = c.rctl[w0];
+    if (!vload(&rc->pull) || vload(&rc->done) || vload(&rc->tail)) return;
+    const int f = blockIdx.y;
+    const unsigned o = rc->owner[f];
+    if ((int)o < w0 || (int)o >= w0 + nw) return;
+    const FragPtrs& F = c.f[f];
+    const unsigned k = rc->iter - 1;
+    const unsigned lane = lane_id();
+    const unsigned nwords = (F.V + 31) / 32;
+    const unsigned warps = gridDim.x * (kThreads / 32);
+    unsigned long long checked = 0;
+    for (unsigned w = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5); w < nwords; w += warps) {
+        const unsigned vw = F.vis[w];
+        const unsigned rem = F.V - w * 32;
+        const unsigned valid = rem >= 32 ? 0xFFFFFFFFu : ((1u << rem) - 1u);
+        const unsigned todo = ~vw & valid;
+        if (!todo) continue;  // warp-uniform
+        bool found = false;
+        if ((todo >> lane) & 1u) {
+            const unsigned v = w * 32 + lane;
+            const unsigned long long e1 = __ldg(F.in_row_ptr + v + 1);
+            for (unsigned long long e = __ldg(F.in_row_ptr + v); e < e1; e++) {
+                const unsigned u = __ldg(F.in_col + e);
+                const int tf = MULTI ? frag_of(c, u) : 0;
+                const unsigned lu = MULTI ? u - c.bounds[tf] : u;
+                checked++;
+                if (__ldcg(c.f[tf].state + lu) == k) {
+                    found = true;
+                    break;
+                }
+            }
+            if (found) F.state[v] = k + 1;
+        }
+        const unsigned nb = __ballot_sync(0xffffffffu, found);
+        if (lane == 0 && nb) {
+            F.vis[w] = vw | nb;
+            atomicOr(F.bm + w, nb);
+        }
+    }
+#pragma unroll
+    for (int q = 16; q > 0; q >>= 1) checked += __shfl_xor_sync(0xffffffffu, checked, q);
+    if (lane == 0 && checked) atomicAdd(&F.ctl->pull_checked, checked);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        // conservation: the frontier's out-edges count as expanded in a bottom-up iteration
+        atomicAdd(&F.ctl->edges_done, vload(&F.ctl->qedges));
+        atomicAdd(&F.ctl->chunks_done, vload(&F.ctl->ntiles));
+    }
 }
 
 // ------------------------------------------------------------------------------------------ PB apply
@@ -1554,6 +1634,12 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
             break;
         case KER_FINALIZE: k_pr_finalize<<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
         case KER_TAIL: return launch_tail<ALG>(c, L, s);
+        case KER_PULL:
+            if (ALG == ALG_BFS && c.bfs_pull) {
+                if (c.P > 1) k_bfs_pull<true><<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+                else k_bfs_pull<false><<<dim3(L.fin_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+            }
+            break;
         case KER_APPLY:
             if (ALG == ALG_BFS && c.pb_shift)
                 k_pb_apply<<<c.pb_nb * kPbParts, kThreads, 2u * (1u << (c.pb_shift - 5)) * 4u, s>>>(c, L.w0);
@@ -1587,6 +1673,10 @@ int phase_kernels(int alg, int phase, int* kinds) {
         kinds[0] = KER_CONTROL;
         kinds[1] = KER_ADVANCE;
         kinds[2] = KER_TAIL;
+        if (alg == ALG_BFS) {
+            kinds[3] = KER_PULL;
+            return 4;
+        }
         return 3;
     }
     if (phase == 0) {
@@ -1600,10 +1690,11 @@ int phase_kernels(int alg, int phase, int* kinds) {
 
 cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                          cudaGraphConditionalHandle h, int use_h) {
-    int kinds[3];
+    int kinds[4];
     const int n = phase_kernels(alg, phase, kinds);
     for (int i = 0; i < n; i++) {
         if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
+        if (kinds[i] == KER_PULL && !c.bfs_pull) continue;
         cudaError_t e = launch_kernel(alg, kinds[i], c, L, s, h, use_h);
         if (e != cudaSuccess) return e;
     }

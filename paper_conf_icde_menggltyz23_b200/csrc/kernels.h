@@ -18,7 +18,7 @@ struct LaunchCfg {
     int tail_grid;    // tail engine CTAs (cooperative; 0 = engine disabled)
 };
 
-enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_APPLY = 6, KER_COUNT = 7 };
+enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_APPLY = 6, KER_PULL = 7, KER_COUNT = 8 };
 cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                           cudaGraphConditionalHandle h, int use_h);
 int phase_kernels(int alg, int phase, int* kinds);
@@ -29,6 +29,7 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
+cudaError_t filter_occupancy(int* blocks_per_sm);
 // BFS propagation blocking: static per-block capacities (in-degree histogram of the blocks) -> pb_off
 cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,
                              unsigned long long* pb_off, void* tmp, size_t tmp_bytes, cudaStream_t s);
@@ -50,6 +51,9 @@ cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* 
                              unsigned long long* s_row_ptr, unsigned* s_col, unsigned long long* cursor, void* tmp,
                              size_t tmp_bytes, cudaStream_t s);
 // fragment extraction: rebased row_ptr slice; orig ids slice (or identity when inv == null)
+cudaError_t setup_transpose(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                            unsigned long long* t_row_ptr, unsigned* t_col, unsigned long long* cursor, void* tmp,
+                            size_t tmp_bytes, cudaStream_t s);
 cudaError_t setup_rebase_rows(const unsigned long long* row_ptr, unsigned b0, unsigned b1, unsigned long long* out,
                               cudaStream_t s);
 // PR destination-blocked static queue: pcol may be null when B == 1 (then the fragment col is used as is)

@@ -60,6 +60,8 @@ struct FragBufs {
     unsigned* pr_tile = nullptr;
     unsigned long long pr_qlen = 0, pr_qedges = 0;
     // BFS propagation blocking
+    unsigned long long* in_row_ptr = nullptr;  // bottom-up BFS in-CSR
+    unsigned* in_col = nullptr;
     unsigned long long* pb_off = nullptr;
     unsigned* pb_fill = nullptr;
     unsigned* pb_done = nullptr;
@@ -79,6 +81,7 @@ struct gum_ctx {
     bool own_stream[kMaxW] = {false};
     int nsm = 148;
     int tail_occ = 1;
+    int filter_occ = 2;
     int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
     std::string err;
     bool poisoned = false;
@@ -103,6 +106,7 @@ struct gum_ctx {
     bool sym_ready = false;
     bool pr_ready = false;
     bool pb_ready = false;
+    bool in_ready = false;
     unsigned pb_shift = 0, pb_nb = 0;
     int pr_blocks = 1;
     FragBufs fr[kMaxW];
@@ -194,6 +198,7 @@ void drop_partition(gum_ctx* c) {
     c->sym_ready = false;
     c->pr_ready = false;
     c->pb_ready = false;
+    c->in_ready = false;
     c->pb_shift = c->pb_nb = 0;
     c->has_result = false;
     c->inv = nullptr;
@@ -255,6 +260,8 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.pb_fill = F.pb_fill;
         p.pb_done = F.pb_done;
         p.pb_buf = F.pb_buf;
+        p.in_row_ptr = F.in_row_ptr;
+        p.in_col = F.in_col;
         p.orig = F.orig;
         p.bm = F.bm;
         p.vis = F.vis;
@@ -307,6 +314,8 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.tail_exit = 4u * c->cfg.tail_vertices;
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
     d.pb_nb = c->pb_nb;
+    d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
+    for (int f = 0; f < c->P; f++) d.total_edges += c->fr[f].E;
     return d;
 }
 
@@ -399,10 +408,11 @@ gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const Laun
         CK(launch_phase(alg, phase, d, L, s, 0, 0));
         return GUM_OK;
     }
-    int kinds[3];
+    int kinds[4];
     const int n = phase_kernels(alg, phase, kinds);
     for (int i = 0; i < n; i++) {
         if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
+        if (kinds[i] == KER_PULL && !d.bfs_pull) continue;
         cudaEvent_t a, b;
         CK(cudaEventCreate(&a));
         CK(cudaEventCreate(&b));
@@ -493,6 +503,53 @@ gum_status build_pb(gum_ctx* c) {
     c->pb_shift = shift;
     c->pb_nb = (unsigned)nb;
     c->pb_ready = true;
+    drop_graphs(c);
+    return GUM_OK;
+}
+
+// In-CSR (transpose) of the partitioned graph, sliced per fragment, for bottom-up BFS iterations.
+gum_status build_in(gum_ctx* c) {
+    if (c->in_ready || !c->cfg.bfs_direction_opt) return GUM_OK;
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    std::vector<Alloc> tmp;
+    unsigned long long* trp = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, c->part_allocs);
+    unsigned* tcol = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(c->E, 1) * 4, c->part_allocs);
+    unsigned long long* cursor = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, tmp);
+    const size_t tb = setup_scan_tmp_bytes(c->V);
+    void* t = dalloc(c, d0, tb, tmp);
+    if (!trp || !tcol || !cursor || !t) {
+        free_list(c, tmp);
+        return fail(c, GUM_ENOMEM, "in-CSR alloc failed");
+    }
+    cudaError_t e = setup_transpose(c->p_row_ptr, c->p_col, c->V, c->E, trp, tcol, cursor, t, tb, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    free_list(c, tmp);
+    if (e != cudaSuccess) return fail(c, GUM_ECUDA, "transpose: %s", cudaGetErrorString(e));
+    std::vector<unsigned long long> hb(c->P + 1);
+    for (int f = 0; f <= c->P; f++) CK(cudaMemcpy(&hb[f], trp + c->bounds[f], 8, cudaMemcpyDeviceToHost));
+    for (int f = 0; f < c->P; f++) {
+        FragBufs& F = c->fr[f];
+        const unsigned long long iE = hb[f + 1] - hb[f];
+        if (c->P == 1 && c->single_device) {
+            F.in_row_ptr = trp;
+            F.in_col = tcol;
+            continue;
+        }
+        F.in_row_ptr = (unsigned long long*)dalloc(c, F.dev, (F.V + 1ull) * 8, c->part_allocs);
+        F.in_col = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(iE, 1) * 4, c->part_allocs);
+        if (!F.in_row_ptr || !F.in_col) return fail(c, GUM_ENOMEM, "in-CSR fragment alloc failed");
+        std::vector<Alloc> t2;
+        unsigned long long* tmp_rp = F.in_row_ptr;
+        if (F.dev != d0) tmp_rp = (unsigned long long*)dalloc(c, d0, (F.V + 1ull) * 8, t2);
+        CK(setup_rebase_rows(trp, c->bounds[f], c->bounds[f + 1], tmp_rp, s));
+        if (F.dev != d0) CK(cudaMemcpyPeerAsync(F.in_row_ptr, F.dev, tmp_rp, d0, (F.V + 1ull) * 8, s));
+        if (iE) CK(cudaMemcpyPeerAsync(F.in_col, F.dev, tcol + hb[f], d0, iE * 4, s));
+        CK(cudaStreamSynchronize(s));
+        free_list(c, t2);
+    }
+    c->in_ready = true;
     drop_graphs(c);
     return GUM_OK;
 }
@@ -640,6 +697,9 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     {
         int occ = 0;
         if (tail_occupancy(&occ) == cudaSuccess && occ > 0) c->tail_occ = std::min(occ, 2);
+        cudaGetLastError();
+        occ = 0;
+        if (filter_occupancy(&occ) == cudaSuccess && occ > 0) c->filter_occ = std::min(occ, 4);
         cudaGetLastError();
     }
     cudaEventCreate(&c->ev0);
@@ -925,7 +985,10 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
     if (alg == GUM_WCC) return build_sym(c);
     if (alg == GUM_PR) return build_pr(c);
-    if (alg == GUM_BFS) return build_pb(c);
+    if (alg == GUM_BFS) {
+        gum_status st = build_pb(c);
+        return st == GUM_OK ? build_in(c) : st;
+    }
     if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
     return GUM_OK;
 }

@@ -185,6 +185,37 @@ cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* 
     return cudaGetLastError();
 }
 
+// in-CSR (transpose) for bottom-up BFS: in-row of v = sources of its in-edges (any order)
+__global__ void k_tr_deg(const unsigned* col, unsigned long long E, unsigned long long* trp) {
+    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < E;
+         e += (unsigned long long)gridDim.x * blockDim.x)
+        atomicAdd(trp + col[e], 1ull);
+}
+
+__global__ void k_tr_fill(const unsigned long long* rp, const unsigned* col, unsigned V, unsigned* tcol,
+                          unsigned long long* cursor) {
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
+    const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
+    for (unsigned long long u = warp; u < V; u += nwarps)
+        for (unsigned long long e = rp[u] + lane; e < rp[u + 1]; e += 32)
+            tcol[atomicAdd(cursor + col[e], 1ull)] = (unsigned)u;
+}
+
+cudaError_t setup_transpose(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
+                            unsigned long long* t_row_ptr, unsigned* t_col, unsigned long long* cursor, void* tmp,
+                            size_t tmp_bytes, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(t_row_ptr, 0, ((size_t)V + 1) * 8, s);
+    if (e != cudaSuccess) return e;
+    k_tr_deg<<<1184, 256, 0, s>>>(col, E, t_row_ptr);
+    e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, t_row_ptr, t_row_ptr, (size_t)V + 1, s);
+    if (e != cudaSuccess) return e;
+    e = cudaMemcpyAsync(cursor, t_row_ptr, ((size_t)V + 1) * 8, cudaMemcpyDeviceToDevice, s);
+    if (e != cudaSuccess) return e;
+    k_tr_fill<<<1184, 256, 0, s>>>(row_ptr, col, V, t_col, cursor);
+    return cudaGetLastError();
+}
+
 __global__ void k_rebase(const unsigned long long* rp, unsigned b0, unsigned b1, unsigned long long* out) {
     const unsigned long long base = rp[b0];
     for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i <= b1 - b0; i += gridDim.x * blockDim.x)

@@ -274,3 +274,17 @@ def test_planned_fsteal(alg):
     done = [a + b for a, b in zip(big["edges_own"], big["edges_stolen"])]
     assert max(done) - min(done) <= 4 * 256 + 2 * big["frontier_edges"] // 100
     assert st.chunks_stolen > 0
+
+
+def test_bfs_direction_optimising():
+    """NEXT-4 bottom-up BFS iterations (bfs_direction_opt): identical depths on RMAT (where the switch
+    fires) and a grid (where it should not), across workers, partitions and launch-unit modes."""
+    g = inputs.rmat(17, 16, seed=81, weighted=False)
+    s = inputs.pick_source(g, 81)
+    ref = oracle.run("bfs", g, s)
+    csr = csr_of(g)
+    for kw in (dict(), dict(num_gpus=3), dict(num_gpus=4, part="random", seed=6), dict(num_gpus=2, split_units=True),
+               dict(tail_vertices=0), dict(num_gpus=2, osteal=False)):
+        _, st, _ = check(g, "bfs", s, csr=csr, ref=ref, bfs_direction_opt=True, **kw)
+    g2 = inputs.grid(64, unit_weights=True)
+    check(g2, "bfs", 0, bfs_direction_opt=True)
