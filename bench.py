@@ -199,6 +199,7 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-variants", action="store_true", help="skip the NEXT-4 variant measurement")
     ap.add_argument("--part", default="seg")
     ap.add_argument("--fsteal", type=int, default=1)
     ap.add_argument("--osteal", type=int, default=1)
@@ -315,7 +316,8 @@ def main():
 
     # ---------------------------------------------------------------- roofline of the advance kernel
     peak, peak_src = load_peak()
-    pctx = gum.Context(profile=True, **ctx_kw) if N == 1 else None
+    # (bottom-up BFS iterations replace the advance, so its per-edge byte model does not apply)
+    pctx = gum.Context(profile=True, **ctx_kw) if N == 1 and not args.bfs_pull else None
     roof = None
     share = None
     if pctx is not None:
@@ -341,6 +343,31 @@ def main():
                 "avg_launch_ms": adv_ms / max(adv_launches, 1),
                 "how": "CUDA events around every k_advance launch on its stream (profile pass, host loop)"}
         share = adv_ms / all_ms if all_ms else None
+
+    # ---------------------------------------------------------------- NEXT-4 variant beside the headline
+    do_bfs = None
+    if alg == "bfs" and not args.bfs_pull and N == 1 and not args.no_variants:
+        dctx = gum.Context(**dict(ctx_kw, bfs_direction_opt=True))
+        dctx.load_csr(row_ptr, col, w)
+        dctx.partition(args.part, 1)
+        dctx.prepare(alg)
+        for s in sources:
+            dctx.run(alg, s)
+        torch.cuda.synchronize()
+        d0, d1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        d0.record()
+        tot = 0
+        for i in range(args.steps):
+            s = sources[i % len(sources)]
+            dctx.run(alg, s)
+            tot += edges_of[s]
+        d1.record()
+        torch.cuda.synchronize()
+        dms = d0.elapsed_time(d1)
+        do_bfs = {"value": round(tot / (dms / 1e3) / 1e9, 3), "unit": "GTEPS", "ms_per_step": round(dms / args.steps, 4),
+                  "what": "direction-optimising BFS (SURVEY NEXT-4, bottom-up iterations under Beamer's rule): "
+                          "same depths, not the paper's push-only method, so not the headline"}
+        dctx.close()
 
     # ---------------------------------------------------------------- end to end through the C ABI
     e2e = None
@@ -416,6 +443,7 @@ def main():
                    "iterations_first_source": st0.iterations if st0 else None,
                    "edges_traversed_first_source": edges_of.get(sources[0]),
                    "advance_share_of_step": share, "parity_full_size": parity,
+                   "bfs_direction_optimising": do_bfs,
                    "setup_s": {"generate": round(t_gen, 2), "build_csr": round(t_csr, 2)}},
     }
     barrier()
