@@ -69,6 +69,7 @@ struct alignas(128) RunCtl {
     unsigned int bodies;      // iteration bodies executed (control launches that did work)
     unsigned int pb;          // the current advance bins its discoveries (apply runs next body)
     unsigned int pull;        // the current BFS iteration runs bottom-up (k_bfs_pull instead of advance)
+    unsigned int skip_filter; // the first iteration's queue is static (WCC blocked): no filter pass
     unsigned int plan_lo[kMaxW][kMaxW], plan_hi[kMaxW][kMaxW];  // FSteal plan: chunks [lo,hi) of queue f -> worker w
     double plan_z;            // planned makespan (edges) of the current iteration
     unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
@@ -130,6 +131,12 @@ struct FragPtrs {
     unsigned int base;                  // global id of local vertex 0
     unsigned long long E;
     unsigned long long pr_qlen, pr_qedges;  // PR's static destination-blocked queue (gum_prepare)
+    // WCC: static destination-blocked queue of the symmetric graph for iteration 0 (all vertices active)
+    const unsigned int* sq_col;
+    const unsigned int* sq_q_v;
+    const unsigned long long* sq_q_off;
+    const unsigned int* sq_tile;
+    unsigned long long sq_len, sq_edges;
 };
 
 struct DevCtx {

@@ -78,7 +78,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         }
         if (i < nwords) {
             unsigned wv = 0;
-            if (ALG == ALG_WCC || ALG == ALG_PR) {
+            if (ALG == ALG_PR || (ALG == ALG_WCC && !F.sq_col)) {
                 unsigned rem = F.V - i * 32;
                 wv = rem >= 32 ? 0xFFFFFFFFu : ((1u << rem) - 1u);
             }
@@ -92,10 +92,12 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         FragCtl* ct = F.ctl;
         ct->claim = 0;
         // PR: the frontier is the static destination-blocked queue built by gum_prepare(PR)
-        ct->ntiles = (ALG == ALG_PR) ? (F.pr_qedges + c.chunk - 1) / c.chunk : 0;
-        ct->qlen = (ALG == ALG_PR) ? F.pr_qlen : 0;
-        ct->qedges = (ALG == ALG_PR) ? F.pr_qedges : 0;
-        ct->app_cnt = (ALG == ALG_WCC) ? F.V : 0;
+        // WCC with a blocked symmetric graph: iteration 0 runs on that static queue (no filter pass)
+        const bool sq = ALG == ALG_WCC && F.sq_col;
+        ct->ntiles = (ALG == ALG_PR) ? (F.pr_qedges + c.chunk - 1) / c.chunk : (sq ? (F.sq_edges + c.chunk - 1) / c.chunk : 0);
+        ct->qlen = (ALG == ALG_PR) ? F.pr_qlen : (sq ? F.sq_len : 0);
+        ct->qedges = (ALG == ALG_PR) ? F.pr_qedges : (sq ? F.sq_edges : 0);
+        ct->app_cnt = (ALG == ALG_WCC && !sq) ? F.V : 0;
         ct->err = 0;
         ct->dense = 0;
         ct->pr_dang[0] = ct->pr_dang[1] = 0.0;
@@ -106,6 +108,10 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->far_cnt = 0;
         ct->far_min[0] = ct->far_min[1] = GUM_INF;
         ct->pull_checked = 0;
+        if (sq) {
+            ct->frontier_edges = F.sq_edges;
+            ct->frontier_vertices = F.sq_len;
+        }
     }
 }
 
@@ -119,9 +125,11 @@ __global__ void k_init_source(const __grid_constant__ DevCtx c, int f, unsigned 
     F.ctl->app_cnt = 1;
 }
 
-__global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, unsigned next_dense0) {
+__global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, unsigned next_dense0,
+                           unsigned skip_filter0) {
     RunCtl* rc = c.rctl[w0];
     rc->next_dense = next_dense0;
+    rc->skip_filter = skip_filter0;
     rc->iter = 0;
     rc->done = 0;
     rc->m = c.P;
@@ -232,7 +240,7 @@ __device__ __forceinline__ bool nf_classify(const FragPtrs& F, FragCtl* ct, unsi
 
 __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
-    if (vload(&rc->done)) return;
+    if (vload(&rc->done) || vload(&rc->skip_filter)) return;
     const int f = blockIdx.y;
     const unsigned o = rc->owner[f];
     if ((int)o < w0 || (int)o >= w0 + nw) return;
@@ -643,6 +651,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         rc->iter = k + 1;
     }
     rc->bodies = rc->bodies + 1;
+    rc->skip_filter = 0;
     for (int f = 0; f < kMaxW; f++) rc->ticket[f] = 0;
     rc->epoch = rc->epoch + 1;
     if (done) {
@@ -827,22 +836,29 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
         const unsigned long long tb = t * CH;
         const unsigned long long qe = s_qedges[f];
         const unsigned tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
-        const unsigned i0 = __ldg(F.tile + t);
-        const unsigned i1 = (t + 1 < s_ntiles[f]) ? __ldg(F.tile + t + 1) : (unsigned)(s_qlen[f] - 1);
+        // WCC iteration 0 runs on the static destination-blocked queue (edges contiguous in queue order)
+        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const unsigned* const tilep = sq ? F.sq_tile : F.tile;
+        const unsigned* const qvp = sq ? F.sq_q_v : F.q_v;
+        const unsigned long long* const qoffp = sq ? F.sq_q_off : F.q_off;
+        const unsigned* const colp = sq ? F.sq_col : F.col;
+        const unsigned i0 = __ldg(tilep + t);
+        const unsigned i1 = (t + 1 < s_ntiles[f]) ? __ldg(tilep + t + 1) : (unsigned)(s_qlen[f] - 1);
         const unsigned nv = i1 - i0 + 1;
 
         // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
         seq++;
         for (unsigned kk = threadIdx.x; kk < nv; kk += kAdvThreads) {
             const unsigned i = i0 + kk;
-            const unsigned long long off = __ldcs(F.q_off + i);
-            // PR's blocked queue stores edges contiguously in queue order: col index == q_off + j
-            s_base[kk] = (unsigned)((long long)tb + ((ALG == ALG_PR) ? 0ll : __ldcs(F.q_base + i)));
+            const unsigned long long off = __ldcs(qoffp + i);
+            // PR's (and WCC iteration 0's) blocked queue stores edges contiguously in queue order:
+            // col index == q_off + j
+            s_base[kk] = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(F.q_base + i)));
             if (ALG == ALG_PR) {
                 const unsigned u = __ldcs(F.q_v + i);
                 s_val[kk] = (VT)__ldcg(F.cx + u);
             } else if (ALG != ALG_BFS) {
-                const unsigned u = __ldcs(F.q_v + i);
+                const unsigned u = __ldcs(qvp + i);
                 s_val[kk] = (VT)__ldcg(F.state + u);
             }
             const long long rel = (long long)off - (long long)tb;
@@ -889,7 +905,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             if (e < tlen) {
                 const unsigned kk = s_head[e];
                 const unsigned long long ci = (unsigned)(s_base[kk] + e);  // mod 2^32: the base may wrap
-                vv[j] = __ldcs(F.col + ci);
+                vv[j] = __ldcs(colp + ci);
                 if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
                 if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];
                 if (ALG == ALG_SSSP) {
@@ -1712,7 +1728,7 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
     }
     // the initial frontier: {source} as a list (BFS/SSSP) or every vertex as a full bitmap (WCC/PR)
     const unsigned nd0 = c.force_mode == 1 ? 0u : ((alg == ALG_WCC || alg == ALG_PR) ? 1u : 0u);
-    k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, nd0);
+    k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, nd0, (alg == ALG_WCC && c.f[0].sq_col) ? 1u : 0u);
     if (src_frag >= f0 && src_frag < f0 + nf) k_init_source<<<1, 1, 0, s>>>(c, src_frag, src_local);
     return cudaGetLastError();
 }

@@ -59,6 +59,12 @@ struct FragBufs {
     unsigned long long* pr_q_off = nullptr;
     unsigned* pr_tile = nullptr;
     unsigned long long pr_qlen = 0, pr_qedges = 0;
+    // WCC iteration-0 static destination-blocked queue over the symmetric graph
+    unsigned* sq_col = nullptr;
+    unsigned* sq_q_v = nullptr;
+    unsigned long long* sq_q_off = nullptr;
+    unsigned* sq_tile = nullptr;
+    unsigned long long sq_len = 0, sq_edges = 0;
     // BFS propagation blocking
     unsigned long long* in_row_ptr = nullptr;  // bottom-up BFS in-CSR
     unsigned* in_col = nullptr;
@@ -262,6 +268,14 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.pb_buf = F.pb_buf;
         p.in_row_ptr = F.in_row_ptr;
         p.in_col = F.in_col;
+        if (alg == GUM_WCC && F.sq_col) {
+            p.sq_col = F.sq_col;
+            p.sq_q_v = F.sq_q_v;
+            p.sq_q_off = F.sq_q_off;
+            p.sq_tile = F.sq_tile;
+            p.sq_len = F.sq_len;
+            p.sq_edges = F.sq_edges;
+        }
         p.orig = F.orig;
         p.bm = F.bm;
         p.vis = F.vis;
@@ -396,6 +410,44 @@ gum_status build_sym(gum_ctx* c) {
         }
         gum_status st = ensure_fragment_state(c, f, std::max(F.E, F.sE));
         if (st != GUM_OK) return st;
+    }
+    // Iteration 0 of WCC has every vertex active: when the label array does not fit L2, regroup the
+    // symmetric graph block-major by destination block (as for PR) so its atomics stay L2-resident.
+    const unsigned long long block_bytes = getenv("GUM_WCC_BLOCK_BYTES") ? strtoull(getenv("GUM_WCC_BLOCK_BYTES"), 0, 10)
+                                                                        : (48ull << 20);
+    if ((unsigned long long)c->V * 4 > block_bytes + (block_bytes >> 1)) {
+        unsigned long long S = std::max<unsigned long long>(256, block_bytes / 4);
+        int B = (int)((c->V + S - 1) / S);
+        if (B > 64) {
+            B = 64;
+            S = (c->V + 63) / 64;
+        }
+        for (int f = 0; f < c->P; f++) {
+            FragBufs& F = c->fr[f];
+            CK(cudaSetDevice(F.dev));
+            cudaStream_t s2 = c->stream[c->split ? f : 0];
+            const unsigned long long cap = std::min<unsigned long long>((unsigned long long)B * F.V, F.sE) + 1;
+            F.sq_col = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(F.sE, 1) * 4, c->part_allocs);
+            F.sq_q_v = (unsigned*)dalloc(c, F.dev, cap * 4, c->part_allocs);
+            F.sq_q_off = (unsigned long long*)dalloc(c, F.dev, (cap + 1) * 8, c->part_allocs);
+            F.sq_tile = (unsigned*)dalloc(c, F.dev, (F.sE / c->cfg.chunk_edges + 2) * 4, c->part_allocs);
+            std::vector<Alloc> tmp2;
+            const size_t tb2 = setup_pr_tmp_bytes(F.V, B);
+            void* t2 = dalloc(c, F.dev, tb2, tmp2);
+            if (!F.sq_col || !F.sq_q_v || !F.sq_q_off || !F.sq_tile || !t2) {
+                free_list(c, tmp2);
+                return fail(c, GUM_ENOMEM, "WCC blocked queue alloc failed (fragment %d)", f);
+            }
+            unsigned long long Q = 0;
+            cudaError_t e2 = setup_pr_blocked(F.s_row_ptr, F.s_col, F.V, F.sE, (unsigned)S, B, c->cfg.chunk_edges,
+                                              F.sq_col, F.sq_q_v, F.sq_q_off, F.sq_tile, &Q, t2, tb2, s2);
+            if (e2 == cudaSuccess) e2 = cudaStreamSynchronize(s2);
+            free_list(c, tmp2);
+            if (e2 != cudaSuccess) return fail(c, GUM_ECUDA, "WCC blocked queue: %s", cudaGetErrorString(e2));
+            F.sq_len = Q;
+            F.sq_edges = F.sE;
+        }
+        CK(cudaSetDevice(c->dev[0]));
     }
     c->sym_ready = true;
     drop_graphs(c);

@@ -288,3 +288,14 @@ def test_bfs_direction_optimising():
         _, st, _ = check(g, "bfs", s, csr=csr, ref=ref, bfs_direction_opt=True, **kw)
     g2 = inputs.grid(64, unit_weights=True)
     check(g2, "bfs", 0, bfs_direction_opt=True)
+
+
+@pytest.mark.parametrize("P", [1, 3])
+def test_wcc_blocked_first_iteration(monkeypatch, P):
+    """WCC iteration 0 on the static destination-blocked symmetric queue (forced with tiny blocks)."""
+    monkeypatch.setenv("GUM_WCC_BLOCK_BYTES", "4096")
+    g = inputs.rmat(14, 8, seed=91, weighted=False)
+    ref = oracle.run("wcc", g)
+    csr = csr_of(g)
+    for kw in (dict(), dict(part="random", seed=2), dict(tail_vertices=0), dict(split_units=P > 1)):
+        check(g, "wcc", 0, csr=csr, ref=ref, num_gpus=P, **kw)
