@@ -9,8 +9,9 @@ vertices / time), whole job. Inputs (1.07 GB col) are larger than L2, so no L2 f
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2]
 
 --impl reference times the CPU oracle (the tier's reference arm) on the same metric/config.
-Under torchrun (N>1) rank 0 drives all N GPUs from one process (single-process multi-device mode
-with P2P peer mappings); the other ranks only join the barriers.
+Under torchrun (N>1) every rank drives its own GPU (one process per GPU, gum_create_mp: fragments
+mapped between processes with CUDA IPC, device-side signal-pad barriers); the step time is the max
+over ranks. `--gpus N` without torchrun uses the single-process multi-device mode instead.
 """
 import argparse
 import json
@@ -144,13 +145,6 @@ def advance_bytes(alg, st):
     return per_edge * st.edges_expanded + per_vertex * st.vertices_frontier + 8 * st.activations
 
 
-def launches_per_run(alg, st):
-    init = {"bfs": 3, "sssp": 3, "wcc": 2, "pr": 3}[alg]
-    if alg == "pr":
-        return init + 3 * st.iterations + 1
-    return init + 3 * (st.iterations + 1)
-
-
 def oracle_bench(g, alg, sources, outdeg, budget_s, reps=None):
     """Times the oracle as it stands (single-threaded by construction). Returns dict."""
     import oracle
@@ -185,6 +179,109 @@ def oracle_bench(g, alg, sources, outdeg, budget_s, reps=None):
         if reps is None and (t_solve >= budget_s or (alg in ("wcc", "pr") and solved >= 1)):
             break
     return dict(value=edges / t_solve / 1e9, solves=solved, solve_s=t_solve, build_s=t_build, outs=outs)
+
+
+def slowest_rank_ms(ms, world):
+    """The job's time is the slowest rank's device time (max over ranks; identity at N=1)."""
+    if world <= 1:
+        return float(ms)
+    from paper_conf_icde_menggltyz23_b200 import dist as gdist
+
+    return gdist.max_over_ranks(ms)
+
+
+def run_multiprocess(args, alg, metric, cfg_desc, ctx_kw, rank, world):
+    """N>1 under torchrun: one process per GPU (gum_create_mp). Every rank builds the same seeded graph,
+    keeps only its own fragment, maps the peers' fragments with CUDA IPC and drives its own GPU; the
+    step time is the max over ranks of each rank's CUDA-event time."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icde_menggltyz23_b200 as gum
+    from paper_conf_icde_menggltyz23_b200 import dist as gdist
+
+    # GUM_BENCH_DEVICE pins every rank to one device (exercises this path on a one-GPU box; not a bench value)
+    local = env_int("GUM_BENCH_DEVICE", env_int("LOCAL_RANK", rank))
+    torch.cuda.set_device(local)
+    g = inputs.make_config(args.config, weighted=(alg == "sssp"))
+    sources, outdeg = pick_sources(g, {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}[args.config], args.sources)
+    if args.config == "C3":
+        sources = [0]
+    if alg in ("wcc", "pr"):
+        sources = sources[:1]
+    row_ptr, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if alg == "sssp" else None)
+    E = g.num_edges
+    kw = dict(ctx_kw)
+    kw.pop("num_gpus", None)
+    kw.pop("device_ids", None)
+    group = gdist.host_group()
+    ctx = gdist.mp_context(device=local, group=group, **kw)
+    ctx.load_csr(row_ptr, col, w)
+    ctx.partition(args.part, 1)
+    ctx.prepare(alg)
+    edges_of = {}
+    for i in range(max(args.warmup, len(sources) if alg in ("bfs", "sssp") else args.warmup)):
+        s = sources[i % len(sources)]
+        ctx.run(alg, s)
+        if s not in edges_of:
+            r = ctx.result()
+            edges_of[s] = traversed_edges(alg, r, outdeg, E) if alg != "pr" else 20 * E
+    stream = torch.cuda.current_stream()
+    dist.barrier(group=group)
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    total_edges, dev_ms, launches = 0, 0.0, 0
+    sampler = ClockSampler(local)
+    with sampler:
+        ev0.record(stream)
+        for i in range(args.steps):
+            s = sources[i % len(sources)]
+            st = ctx.run(alg, s)  # synchronous: returns after this rank's unit converged
+            dev_ms += st.ms
+            launches += st.kernel_launches
+            total_edges += edges_of[s]
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    dist.barrier(group=group)
+    ms = slowest_rank_ms(dev_ms, world)
+    lt = torch.tensor([float(launches)], dtype=torch.float64)
+    dist.all_reduce(lt, group=group)  # whole job: every rank's kernels (incl. its barrier kernels)
+    launches = int(lt.item())
+    # end to end through the ABI (each rank: pinned host CSR in, full result out)
+    e2e = None
+    if not args.no_e2e:
+        K2 = max(3, min(args.steps, 5))
+        out = np.empty(g.num_vertices, dtype=np.float64 if alg == "pr" else np.uint32)
+        dist.barrier(group=group)
+        t0 = time.perf_counter()
+        tot = 0
+        for i in range(K2):
+            s = sources[i % len(sources)]
+            ctx.load_csr(row_ptr, col, w)
+            ctx.partition(args.part, 1)
+            ctx.run(alg, s)
+            ctx.result(out)
+            tot += edges_of[s]
+        e_s = slowest_rank_ms((time.perf_counter() - t0) * 1e3, world) / 1e3
+        h2d = row_ptr.nbytes + col.nbytes + (w.nbytes if w is not None else 0)
+        e2e = {"value": tot / e_s / 1e9, "unit": "GTEPS", "h2d_bytes_per_step": int(h2d) * world,
+               "d2h_bytes_per_step": int(out.nbytes) * world, "steps": K2, "ms_per_step": e_s * 1e3 / K2,
+               "path": "per rank: gum_load_csr(host CSR) + gum_partition (+ IPC exchange) + gum_run + gum_result",
+               "clock": "host wall clock, max over ranks (the call is synchronous)"}
+    ctx.close()
+    if rank == 0:
+        value = total_edges / (ms / 1e3) / 1e9
+        cfg = dict(cfg_desc, processes=world, mode="one process per GPU (gum_create_mp, CUDA IPC peers)")
+        line = {"metric": metric, "value": round(value, 3), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 4), "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "u32" if alg != "pr" else "f64",
+                "data": "synthetic", "config": cfg,
+                "roofline": None, "roofline_note": "per-kernel events need GUM_CFG_PROFILE (single process); see N=1",
+                "cpu_baseline": None, "e2e": e2e,
+                "gpu_launches": launches, "clocks": sampler.summary(),
+                "detail": {"time": "sum of gum_run device times (CUDA events) per rank, max over ranks",
+                           "rank0_event_ms": ev0.elapsed_time(ev1)}}
+        print(json.dumps(line), flush=True)
 
 
 def main():
@@ -232,10 +329,13 @@ def main():
                 "sssp_near_far_delta": sssp_delta if alg == "sssp" else None,
                 "l2": "inputs larger than L2 (col array > 126 MB); no flush"}
 
+    if world > 1 and args.impl == "ours":
+        ctx_kw = dict(fsteal=bool(args.fsteal), osteal=bool(args.osteal), sssp_delta=sssp_delta,
+                      tail_vertices=args.tail, bfs_direction_opt=bool(args.bfs_pull))
+        run_multiprocess(args, alg, metric, cfg_desc, ctx_kw, rank, world)
+        return
     if rank != 0:
-        # rank 0 drives every GPU of the job (single-process multi-device); others only synchronise
-        barrier()
-        barrier()
+        # reference arm under torchrun: rank 0 alone runs the oracle; the others exit without work
         return
 
     t_gen = time.perf_counter()
@@ -248,7 +348,6 @@ def main():
     t_gen = time.perf_counter() - t_gen
 
     if args.impl == "reference":
-        barrier()
         steps_total = args.warmup + args.steps
         ob = oracle_bench(g, alg, sources, outdeg, 0, reps=max(1, args.steps))
         line = {"impl": "reference", "metric": metric, "value": ob["value"], "unit": "GTEPS", "n_gpus": N,
@@ -262,7 +361,6 @@ def main():
                                            f"(adjacency build {ob['build_s']:.1f}s excluded); warm-up skipped "
                                            f"(the oracle has no warm state), requested {steps_total}"},
                 "e2e": {"value": ob["value"], "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-        barrier()
         print(json.dumps(line), flush=True)
         return
 
@@ -305,7 +403,7 @@ def main():
                 s = sources[i % len(sources)]
                 st = ctx.run(alg, s)
                 total_edges += edges_of[s]
-                launches += launches_per_run(alg, st)
+                launches += st.kernel_launches
             ev1.record(stream)
         torch.cuda.synchronize()
     ms = ev0.elapsed_time(ev1)

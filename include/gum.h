@@ -36,7 +36,7 @@ typedef enum {
     GUM_ESTATE = -3, /* wrong call order (run before partition, result before run) or poisoned ctx */
     GUM_ERANGE = -4, /* source >= V, or an SSSP distance reaches 2^32-1 */
     GUM_ECUDA = -5,  /* CUDA runtime error (context is poisoned) */
-    GUM_ENCCL = -6,  /* reserved (collective failure) */
+    GUM_ENCCL = -6,  /* multi-process exchange failed, or a peer never reached a barrier */
     GUM_EUNSUP = -7  /* configuration not supported by this build */
 } gum_status;
 
@@ -144,6 +144,9 @@ typedef struct {
     uint32_t tail_iterations; /* of `iterations`, run inside the tail engine */
     uint32_t bodies;          /* iteration bodies (filter/control/advance/tail launches) executed */
     double pr_last_residual;  /* PR: sum_v |x_K - x_{K-1}| */
+    uint64_t kernel_launches; /* this process's kernel launches in the run: exact in host-loop and
+                                 multi-process mode (incl. barrier kernels); CUDA-graph mode counts every
+                                 body kernel once per executed WHILE iteration (iterations + 1) */
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:
@@ -222,6 +225,46 @@ gum_status gum_profile(const gum_ctx* ctx, gum_kernel_times* out);
  * worker i assigned to worker j (row sums = loads) and *z = the min-max makespan. The device control
  * kernel runs the same routine each iteration. */
 gum_status gum_fsteal_plan(const uint64_t* loads, int n, double remote_cost, double* X, double* z);
+
+/* ---- multi-process mode: one process per GPU (SURVEY.md §8(b) "optional multi-process adapter",
+ * §8(e); the paper runs one worker per GPU) ---------------------------------------------
+ * Each of `world` processes owns fragment `rank` on CUDA device `device`. Peers' fragment arrays are
+ * mapped into every process with CUDA IPC (cudaIpcGetMemHandle / cudaIpcOpenMemHandle), so the
+ * advance's remote updates (a9), frontier steals (a7) and OSteal's "extended memory" reads (a6)
+ * are the same one-sided loads/atomics as in single-process mode. The per-phase barrier (a10) is a
+ * device-side signal-pad barrier (fence.sys + st.release.sys of an epoch into every peer's pad, then
+ * ld.acquire.sys spin on the local pad); no collective is on the data path.
+ *
+ * exchange: host all-gather supplied by the caller (e.g. a torch.distributed gloo group). Every rank
+ * passes `bytes` bytes in `send`; on return `recv` holds world*bytes bytes, rank r's block at
+ * r*bytes. Returns 0 on success, nonzero on failure (reported as GUM_ENCCL). The library calls it
+ * from gum_create_mp, gum_partition, gum_prepare/gum_run (handle exchange, convergence agreement once
+ * per launch batch -- the "global convergence flag" of the north_star) and gum_destroy. */
+typedef int (*gum_exchange_fn)(const void* send, uint64_t bytes, void* recv, void* user);
+typedef struct {
+    int rank;                 /* this process's worker id in [0, world) */
+    int world;                /* number of processes == cfg->num_gpus, 1..GUM_MAX_WORKERS */
+    int device;               /* CUDA device of this process */
+    gum_exchange_fn exchange; /* host all-gather (required) */
+    void* user;               /* passed to exchange */
+} gum_mp_config;
+
+/* Host-only (no GPU needed): all-gathers {magic, library version, ABI struct sizes, rank, world, hash of
+ * every semantic gum_config field} and checks that the ranks form a permutation of [0, world), that
+ * cfg->num_gpus == world on every rank and that every rank runs the same library and configuration.
+ * Returns GUM_OK on every rank or the same error on every rank (GUM_EINVAL on mismatch, GUM_ENCCL if
+ * the exchange fails). gum_create_mp calls it first. */
+gum_status gum_mp_handshake(const gum_config* cfg, const gum_mp_config* mp);
+
+/* Collective: creates this rank's context (fragment `rank` on `mp->device`). cfg->num_gpus must equal
+ * mp->world; cfg->device_ids and cfg->alloc must be NULL (IPC needs whole cudaMalloc allocations).
+ * Afterwards every ABI call is collective and must be made by all ranks with the same arguments:
+ * gum_load_csr (every rank loads the whole graph; validated against the peers at gum_partition),
+ * gum_partition (each rank builds and keeps only its own fragment, then the fragments are
+ * IPC-exchanged), gum_prepare, gum_run (each rank drives its own unit; stats->ms is this rank's device
+ * time -- take the max over ranks), gum_result (every rank gathers the full result through the peer
+ * mappings), gum_destroy. GUM_CFG_PROFILE is not supported (EUNSUP). */
+gum_status gum_create_mp(const gum_config* cfg, const gum_mp_config* mp, gum_ctx** out);
 
 /* Library version (major*10000 + minor*100 + patch). */
 int gum_version(void);

@@ -34,7 +34,8 @@ LOAD_DEVICE = 0x1
 # exported symbols of include/gum.h (tests check the .so exports exactly these)
 ABI_SYMBOLS = ("gum_config_default", "gum_create", "gum_destroy", "gum_last_error", "gum_build_csr",
                "gum_load_csr", "gum_partition", "gum_partition_bounds", "gum_prepare", "gum_run", "gum_result",
-               "gum_result_device", "gum_trace", "gum_profile", "gum_fsteal_plan", "gum_version")
+               "gum_result_device", "gum_trace", "gum_profile", "gum_fsteal_plan", "gum_version",
+               "gum_mp_handshake", "gum_create_mp")
 
 
 class GumError(RuntimeError):
@@ -60,6 +61,14 @@ class gum_config(ctypes.Structure):
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
 
+EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class gum_mp_config(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_int), ("world", ctypes.c_int), ("device", ctypes.c_int),
+                ("exchange", EXCHANGE_FN), ("user", ctypes.c_void_p)]
+
+
 class gum_run_stats(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_uint32), ("ms", ctypes.c_double), ("edges_expanded", ctypes.c_uint64),
                 ("edges_frontier", ctypes.c_uint64), ("edges_stolen", ctypes.c_uint64),
@@ -67,7 +76,7 @@ class gum_run_stats(ctypes.Structure):
                 ("remote_updates", ctypes.c_uint64), ("activations", ctypes.c_uint64),
                 ("vertices_frontier", ctypes.c_uint64), ("final_owners", ctypes.c_uint32), ("osteal_iteration", ctypes.c_uint32),
                 ("tail_iterations", ctypes.c_uint32), ("bodies", ctypes.c_uint32),
-                ("pr_last_residual", ctypes.c_double)]
+                ("pr_last_residual", ctypes.c_double), ("kernel_launches", ctypes.c_uint64)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -114,6 +123,8 @@ def load_library():
         "gum_profile": (i32, [vp, ctypes.POINTER(gum_kernel_times)]),
         "gum_fsteal_plan": (i32, [vp, i32, ctypes.c_double, vp, ctypes.POINTER(ctypes.c_double)]),
         "gum_version": (i32, []),
+        "gum_mp_handshake": (i32, [ctypes.POINTER(gum_config), ctypes.POINTER(gum_mp_config)]),
+        "gum_create_mp": (i32, [ctypes.POINTER(gum_config), ctypes.POINTER(gum_mp_config), ctypes.POINTER(vp)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -170,76 +181,103 @@ class RunStats:
     tail_iterations: int
     bodies: int
     pr_last_residual: float
+    kernel_launches: int
+
+
+def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
+                osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
+                trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192,
+                pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
+                use_torch_allocator=False, streams=None):
+    """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
+    config points to and must live as long as the context."""
+    lib = load_library()
+    keep = []
+    cfg = gum_config()
+    lib.gum_config_default(ctypes.byref(cfg))
+    cfg.num_gpus = int(num_gpus)
+    if device_ids is not None:
+        ids = (ctypes.c_int * len(device_ids))(*device_ids)
+        keep.append(ids)
+        cfg.device_ids = ctypes.cast(ids, ctypes.POINTER(ctypes.c_int))
+    cfg.fsteal = 2 if fsteal == "planned" else int(bool(fsteal))
+    cfg.fsteal_remote_cost = float(fsteal_remote_cost)
+    cfg.bfs_direction_opt = int(bool(bfs_direction_opt))
+    cfg.osteal = int(bool(osteal))
+    cfg.t1_min_max_edges = int(t1)
+    cfg.t2_min_spread_edges = int(t2)
+    cfg.osteal_active_threshold = int(osteal_threshold)
+    cfg.osteal_edges_per_worker = int(osteal_edges_per_worker)
+    cfg.chunk_edges = int(chunk_edges)
+    cfg.pr_iterations = int(pr_iterations)
+    cfg.pr_damping = float(pr_damping)
+    cfg.max_iterations = int(max_iterations)
+    cfg.sssp_delta = int(sssp_delta)
+    cfg.tail_vertices = int(tail_vertices)
+    cfg.pb_block_log2 = int(pb_block_log2)
+    flags = 0
+    if trace:
+        flags |= CFG_TRACE
+    if host_loop:
+        flags |= CFG_HOST_LOOP
+    if profile:
+        flags |= CFG_PROFILE
+    if split_units:
+        flags |= CFG_SPLIT_UNITS
+    if force_mode == "sparse":
+        flags |= CFG_FORCE_SPARSE
+    elif force_mode == "dense":
+        flags |= CFG_FORCE_DENSE
+    cfg.flags = flags
+    if use_torch_allocator:
+        import torch
+
+        def _alloc(nbytes, device, user):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), device=int(device))
+            except Exception:  # noqa: BLE001 - reported to C as a null pointer (GUM_ENOMEM)
+                return None
+
+        def _free(ptr, nbytes, device, user):
+            torch.cuda.caching_allocator_delete(ptr)
+
+        a, f = ALLOC_FN(_alloc), FREE_FN(_free)
+        keep += [a, f]
+        cfg.alloc, cfg.free_fn = a, f
+    if streams is not None:
+        arr = (ctypes.c_void_p * MAX_WORKERS)(*[int(getattr(s, "cuda_stream", s)) for s in streams])
+        keep.append(arr)
+        cfg.streams = ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p))
+    return cfg, keep
 
 
 class Context:
-    """One GUM context: num_gpus workers/fragments (device_ids None => virtual peers on device 0)."""
+    """One GUM context: num_gpus workers/fragments (device_ids None => virtual peers on device 0).
 
-    def __init__(self, num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
-                 osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192, pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None, use_torch_allocator=False, streams=None):
+    Multi-process mode (one process per GPU, include/gum.h gum_create_mp): pass
+    ``mp=(rank, world, device, exchange)`` with num_gpus == world, where ``exchange`` is a host
+    all-gather (see ``paper_conf_icde_menggltyz23_b200.dist.allgather_exchange``). Every later call is
+    then collective over the ranks."""
+
+    def __init__(self, num_gpus=1, mp=None, **kw):
         lib = load_library()
-        cfg = gum_config()
-        lib.gum_config_default(ctypes.byref(cfg))
-        cfg.num_gpus = int(num_gpus)
-        self._dev_ids = None
-        if device_ids is not None:
-            self._dev_ids = (ctypes.c_int * len(device_ids))(*device_ids)
-            cfg.device_ids = ctypes.cast(self._dev_ids, ctypes.POINTER(ctypes.c_int))
-        cfg.fsteal = 2 if fsteal == "planned" else int(bool(fsteal))
-        cfg.fsteal_remote_cost = float(fsteal_remote_cost)
-        cfg.bfs_direction_opt = int(bool(bfs_direction_opt))
-        cfg.osteal = int(bool(osteal))
-        cfg.t1_min_max_edges = int(t1)
-        cfg.t2_min_spread_edges = int(t2)
-        cfg.osteal_active_threshold = int(osteal_threshold)
-        cfg.osteal_edges_per_worker = int(osteal_edges_per_worker)
-        cfg.chunk_edges = int(chunk_edges)
-        cfg.pr_iterations = int(pr_iterations)
-        cfg.pr_damping = float(pr_damping)
-        cfg.max_iterations = int(max_iterations)
-        cfg.sssp_delta = int(sssp_delta)
-        cfg.tail_vertices = int(tail_vertices)
-        cfg.pb_block_log2 = int(pb_block_log2)
-        flags = 0
-        if trace:
-            flags |= CFG_TRACE
-        if host_loop:
-            flags |= CFG_HOST_LOOP
-        if profile:
-            flags |= CFG_PROFILE
-        if split_units:
-            flags |= CFG_SPLIT_UNITS
-        if force_mode == "sparse":
-            flags |= CFG_FORCE_SPARSE
-        elif force_mode == "dense":
-            flags |= CFG_FORCE_DENSE
-        cfg.flags = flags
-        self._keep = []
-        if use_torch_allocator:
-            import torch
-
-            def _alloc(nbytes, device, user):
-                try:
-                    return torch.cuda.caching_allocator_alloc(int(nbytes), device=int(device))
-                except Exception:  # noqa: BLE001 - reported to C as a null pointer (GUM_ENOMEM)
-                    return None
-
-            def _free(ptr, nbytes, device, user):
-                torch.cuda.caching_allocator_delete(ptr)
-
-            a, f = ALLOC_FN(_alloc), FREE_FN(_free)
-            self._keep += [a, f]
-            cfg.alloc, cfg.free_fn = a, f
-        if streams is not None:
-            arr = (ctypes.c_void_p * MAX_WORKERS)(*[int(getattr(s, "cuda_stream", s)) for s in streams])
-            self._keep.append(arr)
-            cfg.streams = ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p))
+        cfg, keep = make_config(num_gpus=num_gpus, **kw)
+        self._keep = keep
         self._cfg = cfg
         self._ctx = ctypes.c_void_p()
-        st = lib.gum_create(ctypes.byref(cfg), ctypes.byref(self._ctx))
-        if st != GUM_OK:
-            raise GumError(st, "gum_create failed (no CUDA device, bad config or unsupported device mix)")
+        if mp is None:
+            st = lib.gum_create(ctypes.byref(cfg), ctypes.byref(self._ctx))
+            if st != GUM_OK:
+                raise GumError(st, "gum_create failed (no CUDA device, bad config or unsupported device mix)")
+        else:
+            rank, world, device, exchange = mp
+            fn = exchange if isinstance(exchange, EXCHANGE_FN) else EXCHANGE_FN(exchange)
+            mpc = gum_mp_config(int(rank), int(world), int(device), fn, None)
+            self._keep += [fn, mpc]
+            st = lib.gum_create_mp(ctypes.byref(cfg), ctypes.byref(mpc), ctypes.byref(self._ctx))
+            if st != GUM_OK:
+                raise GumError(st, "gum_create_mp failed (handshake mismatch, exchange failure or no device)")
+        self.rank = int(mp[0]) if mp is not None else 0
         self.num_gpus = int(num_gpus)
         self.num_vertices = 0
         self._last_alg = None
@@ -330,6 +368,14 @@ class Context:
                              frontier_vertices=r.frontier_vertices, frontier_edges=r.frontier_edges,
                              owners=r.owners, steal_ok=r.steal_ok))
         return recs
+
+
+def mp_handshake(rank, world, exchange, **kw):
+    """Host-only multi-process handshake (gum_mp_handshake): returns the gum_status (0 = all ranks agree)."""
+    cfg, keep = make_config(num_gpus=kw.pop("num_gpus", world), **kw)
+    fn = exchange if isinstance(exchange, EXCHANGE_FN) else EXCHANGE_FN(exchange)
+    mpc = gum_mp_config(int(rank), int(world), 0, fn, None)
+    return int(load_library().gum_mp_handshake(ctypes.byref(cfg), ctypes.byref(mpc)))
 
 
 def fsteal_plan(loads, remote_cost=1.0):

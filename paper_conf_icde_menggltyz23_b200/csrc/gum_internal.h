@@ -139,6 +139,13 @@ struct FragPtrs {
     unsigned long long sq_len, sq_edges;
 };
 
+// Multi-process signal pads (a10): pad[u][s] = last barrier epoch unit s signalled to unit u;
+// pad[u][kMaxW] = timeout flag (a peer never arrived).
+constexpr int kPadWords = 16;
+struct MpPads {
+    unsigned long long* pad[kMaxW];
+};
+
 struct DevCtx {
     FragPtrs f[kMaxW];
     RunCtl* rctl[kMaxW];        // per worker: the replica of the unit that worker belongs to

@@ -1733,6 +1733,35 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------- multi-process barrier (a10)
+// One thread per unit t: fence.sc.sys orders this rank's completed phase (the previous kernels on the
+// stream, incl. their remote atomics into peer memory) before the release-store of `epoch` into
+// peer t's pad slot `me`; then spin with acquire loads until peer t has signalled `epoch` into ours.
+// The next phase starts after this kernel, so it observes everything the peers did before signalling.
+// A peer that never arrives (dead process) trips a 60 s timeout flag instead of hanging the GPU.
+__global__ void k_mp_barrier(const MpPads p, int P, int me, unsigned long long epoch) {
+    const int t = threadIdx.x;
+    if (t >= P) return;
+    asm volatile("fence.sc.sys;" ::: "memory");
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p.pad[t] + me), "l"(epoch) : "memory");
+    const unsigned long long t0 = globaltimer();
+    for (;;) {
+        unsigned long long v;
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p.pad[me] + t) : "memory");
+        if (v >= epoch) break;
+        if (globaltimer() - t0 > 60ull * 1000000000ull) {
+            atomicExch(p.pad[me] + kMaxW, 1ull);
+            break;
+        }
+        __nanosleep(200);
+    }
+}
+
+cudaError_t launch_mp_barrier(const MpPads& p, int P, int me, unsigned long long epoch, cudaStream_t s) {
+    k_mp_barrier<<<1, 32, 0, s>>>(p, P, me, epoch);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid) {
     if (is_pr)
         k_gather<double><<<grid, kThreads, 0, s>>>(c, f, (double*)out, 1);

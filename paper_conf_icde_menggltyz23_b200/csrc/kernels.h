@@ -27,6 +27,8 @@ cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L
 cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream_t s, int f0, int nf, double D0,
                         int src_frag, unsigned src_local);
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
+// multi-process barrier: every rank signals epoch into every peer's pad, then waits for all peers
+cudaError_t launch_mp_barrier(const MpPads& p, int P, int me, unsigned long long epoch, cudaStream_t s);
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
 cudaError_t filter_occupancy(int* blocks_per_sm);

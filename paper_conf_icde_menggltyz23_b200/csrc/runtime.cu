@@ -6,6 +6,8 @@
 
 #include <algorithm>
 #include <cstdarg>
+#include <map>
+#include <utility>
 #include <cstdio>
 #include <cstring>
 #include <ctime>
@@ -133,6 +135,16 @@ struct gum_ctx {
     int last_alg = -1;
     bool has_result = false;
     unsigned last_iters = 0;
+    // multi-process mode (gum_create_mp): this process is worker/unit `rank`; every other fragment's
+    // arrays are CUDA-IPC mappings of the peer process's allocations.
+    bool mp = false;
+    int rank = 0;
+    gum_exchange_fn xch = nullptr;
+    void* xuser = nullptr;
+    unsigned long long* pad[kMaxW] = {nullptr};  // per unit: signal pad (epochs by unit + timeout flag)
+    unsigned long long mp_epoch = 0;
+    unsigned long long launches = 0;  // kernel launches of the current run (gum_run_stats.kernel_launches)
+    std::map<std::pair<int, unsigned long long>, void*> ipc_map;  // (peer, peer pointer) -> mapped pointer
 };
 
 namespace {
@@ -186,6 +198,24 @@ void free_list(gum_ctx* c, std::vector<Alloc>& list) {
     list.clear();
 }
 
+// ---- multi-process mode helpers ------------------------------------------------------------------
+gum_status mp_exchange(gum_ctx* c, const void* send, size_t bytes, void* recv) {
+    if (c->xch(send, bytes, recv, c->xuser) != 0) return fail(c, GUM_ENCCL, "multi-process exchange failed");
+    return GUM_OK;
+}
+
+// host barrier of all ranks (an all-gather of one word)
+gum_status mp_host_barrier(gum_ctx* c) {
+    unsigned long long me = 1, all[kMaxW];
+    return mp_exchange(c, &me, sizeof(me), all);
+}
+
+void mp_close_maps(gum_ctx* c) {
+    for (auto& kv : c->ipc_map) cudaIpcCloseMemHandle(kv.second);
+    c->ipc_map.clear();
+    cudaGetLastError();
+}
+
 void drop_graphs(gum_ctx* c) {
     for (auto& g : c->gexec) {
         if (g) cudaGraphExecDestroy(g);
@@ -199,6 +229,14 @@ void drop_partition(gum_ctx* c) {
         cudaSetDevice(c->dev[d]);
         cudaStreamSynchronize(c->stream[d]);
     }
+    if (c->mp && c->partitioned) {
+        // peers may still read or update this rank's fragment until they are done with it: collective
+        mp_host_barrier(c);
+        mp_close_maps(c);
+        mp_host_barrier(c);
+    }
+    c->mp_epoch = 0;
+    for (auto& p : c->pad) p = nullptr;
     free_list(c, c->part_allocs);
     c->partitioned = false;
     c->sym_ready = false;
@@ -225,6 +263,10 @@ void drop_partition(gum_ctx* c) {
 int unit_w0(const gum_ctx* c, int u) { return c->split ? u : 0; }
 int unit_nw(const gum_ctx* c, int u) { return c->split ? 1 : c->P; }
 int unit_dev(const gum_ctx* c, int u) { return c->dev[unit_w0(c, u)]; }
+// multi-process mode: only this process's unit and fragment are built and launched here
+bool unit_local(const gum_ctx* c, int u) { return !c->mp || u == c->rank; }
+bool frag_local(const gum_ctx* c, int f) { return !c->mp || f == c->rank; }
+int home_unit(const gum_ctx* c) { return c->mp ? c->rank : 0; }
 
 LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     LaunchCfg L;
@@ -335,6 +377,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
 
 gum_status sync_all(gum_ctx* c) {
     for (int u = 0; u < c->n_units; u++) {
+        if (!unit_local(c, u)) continue;
         CK(cudaSetDevice(unit_dev(c, u)));
         CK(cudaStreamSynchronize(c->stream[unit_w0(c, u)]));
     }
@@ -342,8 +385,18 @@ gum_status sync_all(gum_ctx* c) {
 }
 
 // cross-unit barrier (multi-device, single process): every unit's stream waits for every other's.
+// multi-process: a device-side signal-pad barrier on this rank's stream (a10; kernels.cu k_mp_barrier)
 gum_status unit_barrier(gum_ctx* c) {
     if (c->n_units == 1) return GUM_OK;
+    if (c->mp) {
+        MpPads p;
+        memset(&p, 0, sizeof(p));
+        for (int i = 0; i < c->P; i++) p.pad[i] = c->pad[i];
+        CK(cudaSetDevice(c->dev[c->rank]));
+        CK(launch_mp_barrier(p, c->P, c->rank, ++c->mp_epoch, c->stream[c->rank]));
+        c->launches++;
+        return GUM_OK;
+    }
     for (int u = 0; u < c->n_units; u++) {
         CK(cudaSetDevice(unit_dev(c, u)));
         CK(cudaEventRecord(c->bar_ev[u], c->stream[unit_w0(c, u)]));
@@ -352,6 +405,118 @@ gum_status unit_barrier(gum_ctx* c) {
         CK(cudaSetDevice(unit_dev(c, u)));
         for (int v = 0; v < c->n_units; v++)
             if (v != u) CK(cudaStreamWaitEvent(c->stream[unit_w0(c, u)], c->bar_ev[v], 0));
+    }
+    return GUM_OK;
+}
+
+// Multi-process: the device buffers of fragment f that peers map (everything a kernel may touch after
+// OSteal hands the fragment to another worker), plus the unit's run control, trace and signal pad.
+constexpr int kMpFields = 40;
+int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
+    FragBufs& F = c->fr[f];
+    int n = 0;
+#define GUM_FLD(x) out[n++] = (void**)&(x)
+    GUM_FLD(F.row_ptr); GUM_FLD(F.col); GUM_FLD(F.w); GUM_FLD(F.s_row_ptr); GUM_FLD(F.s_col); GUM_FLD(F.orig);
+    GUM_FLD(F.state); GUM_FLD(F.x); GUM_FLD(F.acc); GUM_FLD(F.cx); GUM_FLD(F.bm); GUM_FLD(F.vis); GUM_FLD(F.bm2);
+    GUM_FLD(F.far); GUM_FLD(F.app); GUM_FLD(F.q_v); GUM_FLD(F.q_off); GUM_FLD(F.q_base); GUM_FLD(F.tile);
+    GUM_FLD(F.ctl); GUM_FLD(F.pr_col); GUM_FLD(F.pr_q_v); GUM_FLD(F.pr_q_off); GUM_FLD(F.pr_tile);
+    GUM_FLD(F.sq_col); GUM_FLD(F.sq_q_v); GUM_FLD(F.sq_q_off); GUM_FLD(F.sq_tile); GUM_FLD(F.in_row_ptr);
+    GUM_FLD(F.in_col); GUM_FLD(c->lb[f]); GUM_FLD(c->rctl[f]); GUM_FLD(c->trace[f]); GUM_FLD(c->pad[f]);
+#undef GUM_FLD
+    return n;
+}
+
+struct MpBlob {
+    unsigned magic, status, rank, nfields;
+    unsigned long long V, E, bounds_hash, pr_qlen, sq_len, sE, tile_cap, pad0;
+    unsigned long long ptr[kMpFields];
+    cudaIpcMemHandle_t h[kMpFields];
+};
+constexpr unsigned kMpMagic = 0x47554d31u;  // "GUM1"
+
+unsigned long long hash_words(const void* p, size_t n, unsigned long long h = 1469598103934665603ull) {
+    const unsigned char* b = (const unsigned char*)p;
+    for (size_t i = 0; i < n; i++) h = (h ^ b[i]) * 1099511628211ull;
+    return h;
+}
+
+// Collective: publishes this rank's fragment buffers (IPC handles) and scalars, maps every peer's.
+// local_st = this rank's status of the step just done; if any rank failed, every rank returns an error.
+gum_status mp_publish(gum_ctx* c, gum_status local_st) {
+    if (!c->mp) return local_st;
+    cudaSetDevice(c->dev[c->rank]);
+    if (cudaDeviceSynchronize() != cudaSuccess && local_st == GUM_OK)  // pads/ctl zeroed before peers map them
+        local_st = fail(c, GUM_ECUDA, "device synchronize before the fragment exchange failed");
+    std::vector<MpBlob> all(c->P);
+    MpBlob me;
+    memset(&me, 0, sizeof(me));
+    me.magic = kMpMagic;
+    me.rank = (unsigned)c->rank;
+    void** fl[kMpFields];
+    const int nf = mp_fields(c, c->rank, fl);
+    me.nfields = (unsigned)nf;
+    if (local_st == GUM_OK) {
+        cudaSetDevice(c->dev[c->rank]);
+        for (int i = 0; i < nf; i++) {
+            void* p = *fl[i];
+            me.ptr[i] = (unsigned long long)(uintptr_t)p;
+            if (p && cudaIpcGetMemHandle(&me.h[i], p) != cudaSuccess) {
+                cudaGetLastError();
+                local_st = fail(c, GUM_ECUDA, "cudaIpcGetMemHandle failed (field %d)", i);
+                break;
+            }
+        }
+        const FragBufs& F = c->fr[c->rank];
+        me.V = c->V;
+        me.E = c->E;
+        me.bounds_hash = hash_words(c->bounds, sizeof(unsigned) * (c->P + 1));
+        me.pr_qlen = F.pr_qlen;
+        me.sq_len = F.sq_len;
+        me.sE = F.sE;
+        me.tile_cap = F.tile_cap;
+    }
+    me.status = (unsigned)(-(int)local_st);
+    gum_status st = mp_exchange(c, &me, sizeof(me), all.data());
+    if (st != GUM_OK) return st;
+    if (local_st != GUM_OK) return local_st;
+    for (int r = 0; r < c->P; r++) {
+        const MpBlob& b = all[r];
+        if (b.magic != kMpMagic || b.rank != (unsigned)r || b.nfields != (unsigned)nf)
+            return fail(c, GUM_EINVAL, "multi-process exchange: rank %d sent a malformed blob", r);
+        if (b.status) return fail(c, GUM_ESTATE, "peer rank %d failed (status -%u)", r, b.status);
+        if (b.V != me.V || b.E != me.E || b.bounds_hash != me.bounds_hash)
+            return fail(c, GUM_EINVAL, "rank %d has a different graph or partition (V=%llu E=%llu)", r, b.V, b.E);
+    }
+    for (int r = 0; r < c->P; r++) {
+        if (r == c->rank) continue;
+        const MpBlob& b = all[r];
+        void** pf[kMpFields];
+        mp_fields(c, r, pf);
+        for (int i = 0; i < nf; i++) {
+            if (!b.ptr[i]) {
+                *pf[i] = nullptr;
+                continue;
+            }
+            auto key = std::make_pair(r, b.ptr[i]);
+            auto it = c->ipc_map.find(key);
+            if (it == c->ipc_map.end()) {
+                void* q = nullptr;
+                cudaError_t e = cudaIpcOpenMemHandle(&q, b.h[i], cudaIpcMemLazyEnablePeerAccess);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    return fail(c, GUM_ECUDA, "cudaIpcOpenMemHandle(rank %d, field %d): %s", r, i, cudaGetErrorString(e));
+                }
+                it = c->ipc_map.emplace(key, q).first;
+            }
+            *pf[i] = it->second;
+        }
+        FragBufs& F = c->fr[r];
+        F.pr_qlen = b.pr_qlen;
+        F.pr_qedges = F.E;
+        F.sq_len = b.sq_len;
+        F.sq_edges = b.sE;
+        F.sE = b.sE;
+        F.tile_cap = b.tile_cap;
     }
     return GUM_OK;
 }
@@ -392,6 +557,7 @@ gum_status build_sym(gum_ctx* c) {
         FragBufs& F = c->fr[f];
         F.sE = hb[f + 1] - hb[f];
         if (F.sE >= (1ull << 32)) return fail(c, GUM_EUNSUP, "symmetric fragment %d has >= 2^32 entries", f);
+        if (!frag_local(c, f)) continue;
         if (c->P == 1 && c->single_device) {
             F.s_row_ptr = srp;
             F.s_col = scol;
@@ -423,6 +589,7 @@ gum_status build_sym(gum_ctx* c) {
             S = (c->V + 63) / 64;
         }
         for (int f = 0; f < c->P; f++) {
+            if (!frag_local(c, f)) continue;
             FragBufs& F = c->fr[f];
             CK(cudaSetDevice(F.dev));
             cudaStream_t s2 = c->stream[c->split ? f : 0];
@@ -454,8 +621,23 @@ gum_status build_sym(gum_ctx* c) {
     return GUM_OK;
 }
 
+// kernels launch_phase issues for (alg, phase) under d/L (the skips of kernels.cu launch_phase)
+int count_phase(int alg, int phase, const DevCtx& d, const LaunchCfg& L) {
+    int kinds[4];
+    const int n = phase_kernels(alg, phase, kinds);
+    int k = 0;
+    for (int i = 0; i < n; i++) {
+        if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
+        if (kinds[i] == KER_PULL && !d.bfs_pull) continue;
+        if (kinds[i] == KER_APPLY && !d.pb_shift) continue;
+        k++;
+    }
+    return k;
+}
+
 // Launch one phase; in profile mode bracket every kernel with a pair of CUDA events.
 gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const LaunchCfg& L, cudaStream_t s) {
+    c->launches += count_phase(alg, phase, d, L);
     if (!(c->cfg.flags & GUM_CFG_PROFILE)) {
         CK(launch_phase(alg, phase, d, L, s, 0, 0));
         return GUM_OK;
@@ -495,6 +677,8 @@ gum_status build_pr(gum_ctx* c) {
     c->pr_blocks = B;
     for (int f = 0; f < c->P; f++) {
         FragBufs& F = c->fr[f];
+        F.pr_qedges = F.E;
+        if (!frag_local(c, f)) continue;
         CK(cudaSetDevice(F.dev));
         cudaStream_t s = c->stream[c->split ? f : 0];
         const unsigned long long cap = std::min<unsigned long long>((unsigned long long)B * F.V, F.E) + 1;
@@ -584,6 +768,7 @@ gum_status build_in(gum_ctx* c) {
     for (int f = 0; f < c->P; f++) {
         FragBufs& F = c->fr[f];
         const unsigned long long iE = hb[f + 1] - hb[f];
+        if (!frag_local(c, f)) continue;
         if (c->P == 1 && c->single_device) {
             F.in_row_ptr = trp;
             F.in_col = tcol;
@@ -765,6 +950,90 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     return GUM_OK;
 }
 
+static unsigned long long config_hash(const gum_config* cfg) {
+    unsigned long long h = 1469598103934665603ull;
+#define GUM_HC(x) h = hash_words(&cfg->x, sizeof(cfg->x), h)
+    GUM_HC(num_gpus); GUM_HC(fsteal); GUM_HC(t1_min_max_edges); GUM_HC(t2_min_spread_edges); GUM_HC(osteal);
+    GUM_HC(osteal_active_threshold); GUM_HC(osteal_edges_per_worker); GUM_HC(chunk_edges); GUM_HC(pr_iterations);
+    GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
+    GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt);
+#undef GUM_HC
+    return h;
+}
+
+gum_status gum_mp_handshake(const gum_config* cfg, const gum_mp_config* mp) {
+    if (!cfg || !mp || !mp->exchange) return GUM_EINVAL;
+    if (mp->world < 1 || mp->world > kMaxW) return GUM_EINVAL;
+    struct Hello {
+        unsigned magic, version, sz_cfg, sz_stats;
+        int rank, world, num_gpus, pad;
+        unsigned long long cfg_hash;
+    } me, all[kMaxW];
+    memset(&me, 0, sizeof(me));
+    memset(all, 0, sizeof(all));
+    me.magic = kMpMagic;
+    me.version = (unsigned)gum_version();
+    me.sz_cfg = sizeof(gum_config);
+    me.sz_stats = sizeof(gum_run_stats);
+    me.rank = mp->rank;
+    me.world = mp->world;
+    me.num_gpus = cfg->num_gpus;
+    me.cfg_hash = config_hash(cfg);
+    if (mp->exchange(&me, sizeof(me), all, mp->user) != 0) return GUM_ENCCL;
+    // every rank evaluates the same gathered table, so every rank returns the same status
+    for (int r = 0; r < mp->world; r++) {
+        const Hello& h = all[r];
+        if (h.magic != kMpMagic || h.version != me.version || h.sz_cfg != me.sz_cfg || h.sz_stats != me.sz_stats)
+            return GUM_EINVAL;
+        if (h.rank != r || h.world != all[0].world || h.num_gpus != h.world || h.cfg_hash != all[0].cfg_hash)
+            return GUM_EINVAL;
+    }
+    return GUM_OK;
+}
+
+gum_status gum_create_mp(const gum_config* cfg, const gum_mp_config* mp, gum_ctx** out) {
+    if (!cfg || !mp || !out || !mp->exchange) return GUM_EINVAL;
+    *out = nullptr;
+    if (mp->rank < 0 || mp->rank >= mp->world) return GUM_EINVAL;
+    gum_status st = gum_mp_handshake(cfg, mp);
+    if (st != GUM_OK) return st;
+    gum_status local = GUM_OK;
+    if (cfg->device_ids || cfg->alloc) local = GUM_EUNSUP;  // IPC maps whole cudaMalloc allocations
+    gum_ctx* c = nullptr;
+    if (local == GUM_OK) {
+        gum_config c1 = *cfg;
+        int devs[kMaxW];
+        for (int i = 0; i < kMaxW; i++) devs[i] = mp->device;
+        c1.device_ids = devs;
+        c1.flags &= ~GUM_CFG_SPLIT_UNITS;
+        if (cfg->flags & GUM_CFG_PROFILE) local = GUM_EUNSUP;
+        else local = gum_create(&c1, &c);
+    }
+    // agree: every rank creates its context or none keeps one
+    long long mine = local, all[kMaxW];
+    if (mp->exchange(&mine, sizeof(mine), all, mp->user) != 0) {
+        gum_destroy(c);
+        return GUM_ENCCL;
+    }
+    for (int r = 0; r < mp->world; r++)
+        if (all[r] != GUM_OK) {
+            gum_destroy(c);
+            return local != GUM_OK ? local : GUM_ESTATE;
+        }
+    if (mp->world > 1) {
+        c->mp = true;
+        c->rank = mp->rank;
+        c->xch = mp->exchange;
+        c->xuser = mp->user;
+        c->single_device = false;
+        c->split = true;
+        c->n_units = c->P;
+        for (int i = 1; i < c->P; i++) c->stream[i] = c->stream[0];  // own_stream[0] stays the only owner
+    }
+    *out = c;
+    return GUM_OK;
+}
+
 void gum_destroy(gum_ctx* c) {
     if (!c) return;
     drop_partition(c);
@@ -880,12 +1149,23 @@ gum_status gum_load_csr(gum_ctx* c, uint32_t V, uint64_t E, const uint64_t* row_
     return GUM_OK;
 }
 
+static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed);
+
 gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
     if (!c) return GUM_EINVAL;
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->loaded) return fail(c, GUM_ESTATE, "gum_partition before gum_load_csr");
     if (kind != GUM_PART_SEG && kind != GUM_PART_RANDOM) return fail(c, GUM_EINVAL, "bad partition kind");
     drop_partition(c);
+    gum_status st = partition_body(c, kind, seed);
+    if (c->mp) {
+        st = mp_publish(c, st);
+        c->partitioned = st == GUM_OK;
+    }
+    return st;
+}
+
+static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
     const int d0 = c->dev[0];
     CK(cudaSetDevice(d0));
     cudaStream_t s = c->stream[0];
@@ -935,6 +1215,7 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.V = c->bounds[f + 1] - c->bounds[f];
         F.E = eb[f + 1] - eb[f];
         if (F.E >= (1ull << 32)) return fail(c, GUM_EUNSUP, "fragment %d has >= 2^32 edges: use more workers", f);
+        if (!frag_local(c, f)) continue;  // multi-process: the peer's buffers are mapped by mp_publish
         const size_t Vn = std::max<size_t>(F.V, 1);
         if (c->P == 1 && c->single_device) {
             F.row_ptr = c->p_row_ptr;
@@ -991,13 +1272,21 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
     }
     c->lb_parts = parts;
     for (int f = 0; f < c->P; f++) {
+        if (!frag_local(c, f)) continue;
         c->lb[f] = (LBSlot*)dalloc(c, c->fr[f].dev, (size_t)parts * sizeof(LBSlot), c->part_allocs);
         if (!c->lb[f]) return fail(c, GUM_ENOMEM, "look-back alloc failed");
         CK(cudaSetDevice(c->fr[f].dev));
         CK(cudaMemset(c->lb[f], 0, (size_t)parts * sizeof(LBSlot)));
     }
     for (int u = 0; u < c->n_units; u++) {
+        if (!unit_local(c, u)) continue;
         int w0 = unit_w0(c, u), d = unit_dev(c, u);
+        if (c->mp) {
+            c->pad[w0] = (unsigned long long*)dalloc(c, d, kPadWords * 8, c->part_allocs);
+            if (!c->pad[w0]) return fail(c, GUM_ENOMEM, "signal pad alloc failed");
+            CK(cudaSetDevice(d));
+            CK(cudaMemset(c->pad[w0], 0, kPadWords * 8));
+        }
         c->rctl[w0] = (RunCtl*)dalloc(c, d, sizeof(RunCtl), c->part_allocs);
         c->tsplit[w0] = (TailSplit*)dalloc(c, d, 8192 * sizeof(TailSplit), c->part_allocs);
         if (!c->rctl[w0] || !c->tsplit[w0]) return fail(c, GUM_ENOMEM, "run control alloc failed");
@@ -1035,14 +1324,22 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
     if (!c) return GUM_EINVAL;
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
-    if (alg == GUM_WCC) return build_sym(c);
-    if (alg == GUM_PR) return build_pr(c);
-    if (alg == GUM_BFS) {
-        gum_status st = build_pb(c);
-        return st == GUM_OK ? build_in(c) : st;
-    }
     if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
-    return GUM_OK;
+    gum_status st = GUM_OK;
+    bool built = false;  // multi-process: new buffers must be published (all ranks agree: same state)
+    if (alg == GUM_WCC) {
+        built = !c->sym_ready;
+        st = build_sym(c);
+    } else if (alg == GUM_PR) {
+        built = !c->pr_ready;
+        st = build_pr(c);
+    } else if (alg == GUM_BFS) {
+        built = (!c->pb_ready && c->P == 1 && c->cfg.pb_block_log2) || (!c->in_ready && c->cfg.bfs_direction_opt);
+        st = build_pb(c);
+        if (st == GUM_OK) st = build_in(c);
+    }
+    if (c->mp && built) st = mp_publish(c, st);
+    return st;
 }
 
 gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stats) {
@@ -1080,6 +1377,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     }
     CK(cudaSetDevice(c->dev[0]));
     CK(cudaEventRecord(c->ev0, c->stream[0]));
+    c->launches = 0;
     if (c->n_units > 1) {
         st = unit_barrier(c);
         if (st != GUM_OK) return st;
@@ -1090,9 +1388,11 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         CK(cudaEventRecord(init_a, c->stream[0]));
     }
     for (int u = 0; u < c->n_units; u++) {
+        if (!unit_local(c, u)) continue;
         const LaunchCfg L = make_launch(c, u, alg);
         CK(cudaSetDevice(unit_dev(c, u)));
         CK(launch_init(alg, d, L, c->stream[L.w0], L.w0, L.nw, D0, src_frag, src_local));
+        c->launches += 2 + ((src_frag >= L.w0 && src_frag < L.w0 + L.nw) ? 1 : 0);
     }
     if (profile) CK(cudaEventRecord(init_b, c->stream[0]));
     if (graph_mode) {
@@ -1120,6 +1420,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
                     st = unit_barrier(c);
                     if (st != GUM_OK) return st;
                     for (int u = 0; u < c->n_units; u++) {
+                        if (!unit_local(c, u)) continue;
                         const LaunchCfg L = make_launch(c, u, alg);
                         CK(cudaSetDevice(unit_dev(c, u)));
                         st = run_phase(c, alg, phase, d, L, c->stream[L.w0]);
@@ -1127,14 +1428,32 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
                     }
                 }
             }
-            CK(cudaSetDevice(c->dev[0]));
-            CK(cudaMemcpyAsync(c->h_rctl, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost, c->stream[0]));
-            CK(cudaStreamSynchronize(c->stream[0]));
+            const int hu = home_unit(c);
+            CK(cudaSetDevice(c->dev[hu]));
+            CK(cudaMemcpyAsync(c->h_rctl, c->rctl[hu], sizeof(RunCtl), cudaMemcpyDeviceToHost, c->stream[hu]));
+            CK(cudaStreamSynchronize(c->stream[hu]));
             if (getenv("GUM_DEBUG"))
                 fprintf(stderr, "[gum] host loop: iter=%u done=%u tail=%u err=%u bodies=%u tail_iters=%u\n",
                         c->h_rctl->iter, c->h_rctl->done, c->h_rctl->tail, c->h_rctl->err, c->h_rctl->bodies,
                         c->h_rctl->tail_iters);
-            if (c->h_rctl->done) break;
+            if (c->mp) {
+                // the global convergence flag: every unit decided it redundantly from the same counts;
+                // the ranks leave the loop together (matching barrier sequences) once all agree
+                unsigned long long mine = c->h_rctl->done ? 1ull : 0ull, flags[kMaxW];
+                unsigned long long pad_err = 0;
+                CK(cudaMemcpy(&pad_err, c->pad[c->rank] + kMaxW, 8, cudaMemcpyDeviceToHost));
+                if (pad_err) mine = 2;
+                st = mp_exchange(c, &mine, sizeof(mine), flags);
+                if (st != GUM_OK) return st;
+                bool all = true;
+                for (int r = 0; r < c->P; r++) {
+                    if (flags[r] == 2) return fail(c, GUM_ENCCL, "barrier timeout: rank %d never arrived", r);
+                    all = all && flags[r] == 1;
+                }
+                if (all) break;
+            } else if (c->h_rctl->done) {
+                break;
+            }
         }
         st = unit_barrier(c);
         if (st != GUM_OK) return st;
@@ -1143,7 +1462,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     CK(cudaEventRecord(c->ev1, c->stream[0]));
     st = sync_all(c);
     if (st != GUM_OK) return st;
-    CK(cudaMemcpy(c->h_rctl, c->rctl[0], sizeof(RunCtl), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(c->h_rctl, c->rctl[home_unit(c)], sizeof(RunCtl), cudaMemcpyDeviceToHost));
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
     const RunCtl R = *c->h_rctl;
@@ -1177,6 +1496,11 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         stats->pr_last_residual = R.pr_resid;
         stats->tail_iterations = R.tail_iters;
         stats->bodies = R.bodies;
+        stats->kernel_launches = c->launches;
+        if (graph_mode) {
+            const LaunchCfg L0 = make_launch(c, 0, alg);
+            stats->kernel_launches += (unsigned long long)(R.iter + 1) * (count_phase(alg, 0, d, L0) + count_phase(alg, 1, d, L0));
+        }
         unsigned long long qedges_total = 0;
         for (int f = 0; f < c->P; f++) {
             FragCtl fc;

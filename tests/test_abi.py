@@ -58,7 +58,7 @@ def test_build_csr_edge_cases():
 
 def test_struct_layouts_match_header():
     # sizes fixed by include/gum.h (LP64)
-    assert ctypes.sizeof(gum.gum_run_stats) == 4 + 4 + 9 * 8 + 4 * 4 + 8
+    assert ctypes.sizeof(gum.gum_run_stats) == 4 + 4 + 9 * 8 + 4 * 4 + 8 + 8
     assert ctypes.sizeof(gum.gum_iter_trace) == 4 * 8 * 8 + 16 + 8
 
 
