@@ -15,10 +15,14 @@ constexpr int kThreads = 256;          // CTA size of advance / filter
 #define GUM_ADV_THREADS 256
 #endif
 constexpr int kAdvThreads = GUM_ADV_THREADS;  // CTA size of the advance (its barrier domain)
-constexpr int kEdgesPerThread = 8;
+#ifndef GUM_EPT
+#define GUM_EPT 8
+#endif
+constexpr int kEdgesPerThread = GUM_EPT;
 constexpr int kTileMax = kAdvThreads * kEdgesPerThread;  // max edges per claimable chunk (smem sized for it)
-constexpr int kDenseWordsPerWarp = 32;                            // dense filter: bitmap words per warp
-constexpr int kDenseWordsPerPart = (kThreads / 32) * kDenseWordsPerWarp;  // 256 words = 8192 vertices
+constexpr int kDenseVertsPerThread = 8;                           // dense filter: consecutive vertices per thread
+constexpr int kDenseWordsPerWarp = 32 * kDenseVertsPerThread / 32;   // 8 bitmap words per warp
+constexpr int kDenseWordsPerPart = (kThreads / 32) * kDenseWordsPerWarp;  // 64 words = 2048 vertices
 constexpr int kFilterAppPerThread = 8;                            // sparse filter: list entries per thread
 constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;

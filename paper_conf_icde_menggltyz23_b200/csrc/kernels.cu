@@ -219,26 +219,130 @@ __device__ __forceinline__ unsigned long long warp_excl_scan_u64(unsigned long l
     return inc - x;
 }
 
-// SSSP near-far classification of an activated vertex with out-degree > 0 (phase 1 of the filter):
-// near (dist < T) -> returns true and leaves the far set; far -> parked (bit set), counted, and its
-// distance folded into this sweep epoch's far minimum.
-__device__ __forceinline__ bool nf_classify(const FragPtrs& F, FragCtl* ct, unsigned v, unsigned T, unsigned slot) {
-    const unsigned dist = F.state[v];
-    const unsigned bit = 1u << (v & 31);
-    if (dist >= T) {
+
+#ifndef GUM_FILTER_MINB
+#define GUM_FILTER_MINB 4
+#endif
+
+// One filter tile (2048 items: 64 bitmap words in dense mode, 2048 activation-list entries in sparse
+// mode). Thread t owns 8 consecutive items; returns its (count, degree) of accepted vertices (out-degree
+// > 0 and, with the SSSP near-far split, dist < T) in vertex order.
+//   FT_CLASSIFY (pass 1): near-far parking happens here, once (far bit, far count, far minimum);
+//   FT_COUNT    (pass 2a): pure re-count with the same acceptance (dist < T);
+//   FT_EMIT     (pass 2b): writes the queue entries from pos/off on, clears the consumed bitmap words and
+//                          the far bits of accepted vertices.
+enum { FT_CLASSIFY = 0, FT_COUNT = 1, FT_EMIT = 2 };
+template <int MODE>
+__device__ __forceinline__ bool filter_accept(const FragPtrs& F, FragCtl* ct, unsigned v, bool nf, unsigned nfT,
+                                              unsigned fslot) {
+    if (!nf) return true;
+    if (MODE == FT_CLASSIFY) {
+        const unsigned dist = F.state[v];
+        if (dist < nfT) return true;
+        const unsigned bit = 1u << (v & 31);
         const unsigned ob = atomicOr(F.far + (v >> 5), bit);
         if (!(ob & bit)) atomicAdd(&ct->far_cnt, 1ull);
-        atomicMin(&ct->far_min[slot], dist);
+        atomicMin(&ct->far_min[fslot], dist);
         return false;
     }
-    if (F.far[v >> 5] & bit) {
-        const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
-        if (ob & bit) atomicAdd(&ct->far_cnt, ~0ull);  // -1
+    if (F.state[v] >= nfT) return false;  // parked in pass 1
+    if (MODE == FT_EMIT) {
+        const unsigned bit = 1u << (v & 31);
+        if (F.far[v >> 5] & bit) {
+            const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
+            if (ob & bit) atomicAdd(&ct->far_cnt, ~0ull);  // -1
+        }
     }
     return true;
 }
 
-__global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+template <int MODE>
+__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, FragCtl* ct, unsigned tile, bool dense, bool sweep,
+                                            bool nf, unsigned nfT, unsigned fslot, unsigned nwords, unsigned app_cnt,
+                                            unsigned chunk, unsigned long long pos, unsigned long long off) {
+    const unsigned lane = lane_id();
+    Pair mine{0, 0};
+    if (dense) {
+        const unsigned wbase = tile * kDenseWordsPerPart + (threadIdx.x >> 5) * kDenseWordsPerWarp;
+        const unsigned vb = wbase * 32u + lane * kDenseVertsPerThread;
+        const unsigned wi = wbase + (lane >> 2);
+        unsigned word = 0;
+        if (wi < nwords) {
+            word = F.bm[wi];
+            if (sweep) word |= F.far[wi];
+        }
+        if (MODE == FT_EMIT) {
+            __syncwarp();
+            if ((lane & 3u) == 0 && wi < nwords && F.bm[wi]) F.bm[wi] = 0u;
+        }
+        const unsigned bits = (word >> ((lane & 3u) * 8u)) & 0xFFu;
+        if (bits) {
+            unsigned long long rpv[kDenseVertsPerThread + 1];
+            const unsigned long long* rp = F.row_ptr + vb;  // 64-byte aligned (vb % 8 == 0)
+            if (vb + kDenseVertsPerThread <= F.V) {
+#pragma unroll
+                for (int q = 0; q < kDenseVertsPerThread / 2; q++) {
+                    const ulonglong2 t2 = __ldg(reinterpret_cast<const ulonglong2*>(rp) + q);
+                    rpv[2 * q] = t2.x;
+                    rpv[2 * q + 1] = t2.y;
+                }
+                rpv[kDenseVertsPerThread] = __ldg(rp + kDenseVertsPerThread);
+            } else {
+#pragma unroll
+                for (int q = 0; q <= kDenseVertsPerThread; q++) rpv[q] = (vb + q <= F.V) ? __ldg(rp + q) : 0ull;
+            }
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread; q++) {
+                if ((bits >> q) & 1u) {
+                    const unsigned long long d = rpv[q + 1] - rpv[q];
+                    if (d && filter_accept<MODE>(F, ct, vb + q, nf, nfT, fslot)) {
+                        if (MODE == FT_EMIT) emit_vertex(F, chunk, vb + q, rpv[q], d, pos + mine.cnt, off + mine.deg);
+                        mine.cnt += 1;
+                        mine.deg += d;
+                    }
+                }
+            }
+        }
+    } else {
+        const unsigned long long ibase = (unsigned long long)tile * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
+        unsigned items[kFilterAppPerThread];
+        unsigned long long rp0[kFilterAppPerThread], d[kFilterAppPerThread];
+#pragma unroll
+        for (int j = 0; j < kFilterAppPerThread; j++) {
+            items[j] = 0xFFFFFFFFu;
+            if (ibase + j < app_cnt) items[j] = F.app[ibase + j];
+        }
+#pragma unroll
+        for (int j = 0; j < kFilterAppPerThread; j++) {
+            d[j] = 0;
+            rp0[j] = 0;
+            if (items[j] != 0xFFFFFFFFu) {
+                const unsigned v = items[j];
+                // every set bit belongs to a listed vertex: clearing whole words is exact
+                if (MODE == FT_EMIT) F.bm[v >> 5] = 0u;
+                rp0[j] = __ldg(F.row_ptr + v);
+                d[j] = __ldg(F.row_ptr + v + 1) - rp0[j];
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kFilterAppPerThread; j++) {
+            if (d[j] && filter_accept<MODE>(F, ct, items[j], nf, nfT, fslot)) {
+                if (MODE == FT_EMIT) emit_vertex(F, chunk, items[j], rp0[j], d[j], pos + mine.cnt, off + mine.deg);
+                mine.cnt += 1;
+                mine.deg += d[j];
+            }
+        }
+    }
+    return mine;
+}
+
+// a4 filter / frontier generation (Example 4 Step 1; Alg. 1's degree prefix sum): the
+// fragment's activations (bitmap words when dense, the activation list when sparse) -> queue of
+// vertices with out-degree > 0 (q_v), exclusive out-degree prefix (q_off), col base (q_base) and the
+// edge-balanced chunk table. Reduce-then-scan over a static split of the tiles: CTA b (ticket order)
+// counts its contiguous tile range, publishes the aggregate, sums its predecessors' aggregates (one
+// parallel read, no serial look-back chain) and re-walks its range emitting entries in vertex order.
+__global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
     if (vload(&rc->done) || vload(&rc->skip_filter)) return;
     const int f = blockIdx.y;
@@ -257,207 +361,70 @@ __global__ void __launch_bounds__(kThreads, 4) k_filter(const __grid_constant__ 
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
     const unsigned per = dense ? kDenseWordsPerPart : kFilterAppPerPart;
-    unsigned long long n_parts = (n_items + per - 1) / per;
-    if (n_parts == 0) n_parts = 1;
+    const unsigned n_tiles = (unsigned)((n_items + per - 1) / per);
     const unsigned long long epoch = rc->epoch;
     const unsigned chunk = c.chunk;
     LBSlot* slots = c.lb[f];
-    const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
+    // small lists: only as many CTAs as tiles take part (the others leave before the prefix exchange)
+    const unsigned G = n_tiles < gridDim.x ? (n_tiles ? n_tiles : 1u) : gridDim.x;
 
-    __shared__ unsigned s_part;
+    __shared__ unsigned s_b;
     __shared__ Pair s_warp[kThreads / 32];
-    __shared__ Pair s_excl;
+    if (threadIdx.x == 0) s_b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
+    __syncthreads();
+    const unsigned b = s_b;
+    if (b >= G) return;
+    const unsigned t_lo = (unsigned)(((unsigned long long)n_tiles * b) / G);
+    const unsigned t_hi = (unsigned)(((unsigned long long)n_tiles * (b + 1)) / G);
 
-    for (;;) {
-        if (threadIdx.x == 0) s_part = atomicAdd(&rc->ticket[f], 1u);
-        __syncthreads();
-        const unsigned p = s_part;
-        __syncthreads();
-        if (p >= n_parts) break;
-
-        // ---- phase 1: count vertices with out-degree > 0 and their degrees
-        Pair mine{0, 0};
-        unsigned myword = 0;
-        unsigned items[kFilterAppPerThread];
-        const unsigned wbase = p * kDenseWordsPerPart + wid * kDenseWordsPerWarp;
-        const unsigned long long ibase =
-            (unsigned long long)p * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
-        if (dense) {
-            if (wbase + lane < nwords) {
-                myword = F.bm[wbase + lane];
-                if (myword) F.bm[wbase + lane] = 0u;
-                if (sweep) myword |= F.far[wbase + lane];
-            }
-            unsigned long long wc = 0, wd = 0;
-#pragma unroll
-            for (int i0 = 0; i0 < kDenseWordsPerWarp; i0 += 8) {
-                unsigned long long d[8];
-#pragma unroll
-                for (int k = 0; k < 8; k++) {
-                    const unsigned wv = __shfl_sync(0xffffffffu, myword, i0 + k);
-                    const unsigned v = (wbase + i0 + k) * 32 + lane;
-                    d[k] = 0;
-                    if ((wv >> lane) & 1u) d[k] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
-                    if (nf && d[k] && !nf_classify(F, ct, v, nfT, fslot)) d[k] = 0;
-                }
-#pragma unroll
-                for (int k = 0; k < 8; k++) {
-                    wc += d[k] ? 1 : 0;
-                    wd += d[k];
-                }
-            }
-            wc = warp_sum_u64(wc);
-            wd = warp_sum_u64(wd);
-            if (lane == 0) mine = Pair{wc, wd};  // block scan over warps (lane 0 carries the warp)
-        } else {
-            unsigned long long d[kFilterAppPerThread];
-#pragma unroll
-            for (int j = 0; j < kFilterAppPerThread; j++) {
-                d[j] = 0;
-                items[j] = 0xFFFFFFFFu;
-                if (ibase + j < app_cnt) {
-                    const unsigned v = F.app[ibase + j];
-                    items[j] = v;
-                    F.bm[v >> 5] = 0u;  // every set bit belongs to a listed vertex: clearing whole words is exact
-                    d[j] = __ldg(F.row_ptr + v + 1) - __ldg(F.row_ptr + v);
-                    if (nf && d[j] && !nf_classify(F, ct, v, nfT, fslot)) d[j] = 0;
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < kFilterAppPerThread; j++) {
-                mine.cnt += d[j] ? 1 : 0;
-                mine.deg += d[j];
-            }
-        }
-        Pair agg;
-        Pair texcl = block_excl_scan(mine, s_warp, agg);
-
-        // ---- decoupled look-back over partitions of this fragment (warp 0, 32 predecessors per step)
-        if (wid == 0) {
-            LBSlot* S = slots + p;
-            const unsigned long long AGG = epoch * 4 + 1, INC = epoch * 4 + 2;
-            Pair excl{0, 0};
-            if (lane == 0) {
-                if (p == 0) {
-                    S->inc_cnt = agg.cnt;
-                    S->inc_deg = agg.deg;
-                    st_release_u64(&S->flag, INC);
-                } else {
-                    S->agg_cnt = agg.cnt;
-                    S->agg_deg = agg.deg;
-                    st_release_u64(&S->flag, AGG);
-                }
-            }
-            __syncwarp();
-            if (p > 0) {
-                long long j = (long long)p - 1 - lane;  // lane 0 = nearest predecessor
-                for (;;) {
-                    unsigned long long fl = INC;
-                    if (j >= 0) {
-                        do {
-                            fl = ld_acquire_u64(&slots[j].flag);
-                        } while (fl < AGG);
-                    }
-                    const bool is_inc = fl >= INC;
-                    const unsigned incmask = __ballot_sync(0xffffffffu, is_inc);
-                    const int first = incmask ? __ffs(incmask) - 1 : 32;  // nearest inclusive in window
-                    unsigned long long vc = 0, vd = 0;
-                    if ((int)lane <= first && j >= 0) {
-                        if ((int)lane == first) {
-                            vc = __ldcg(&slots[j].inc_cnt);
-                            vd = __ldcg(&slots[j].inc_deg);
-                        } else {
-                            vc = __ldcg(&slots[j].agg_cnt);
-                            vd = __ldcg(&slots[j].agg_deg);
-                        }
-                    }
-                    excl.cnt += warp_sum_u64(vc);
-                    excl.deg += warp_sum_u64(vd);
-                    if (incmask) break;
-                    j -= 32;
-                }
-                if (lane == 0) {
-                    S->inc_cnt = excl.cnt + agg.cnt;
-                    S->inc_deg = excl.deg + agg.deg;
-                    st_release_u64(&S->flag, INC);
-                }
-            }
-            if (lane == 0) {
-                s_excl = excl;
-                if (p == n_parts - 1) {
-                    const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
-                    F.q_off[tc] = td;
-                    ct->qlen = tc;
-                    ct->qedges = td;
-                    ct->ntiles = (td + chunk - 1) / chunk;
-                    ct->claim = 0;
-                    for (int q = 0; q < kMaxW; q++) ct->pclaim[q] = 0;
-                    ct->app_cnt = 0;
-                    ct->dense = dense ? 1u : 0u;
-                    ct->frontier_edges += td;
-                    ct->frontier_vertices += tc;
-                }
-            }
-        }
-        __syncthreads();
-
-        // ---- phase 2: write queue entries, degree prefix and chunk table
-        if (dense) {
-            unsigned long long pos = s_excl.cnt + __shfl_sync(0xffffffffu, texcl.cnt, 0);
-            unsigned long long off = s_excl.deg + __shfl_sync(0xffffffffu, texcl.deg, 0);
-#pragma unroll
-            for (int i0 = 0; i0 < kDenseWordsPerWarp; i0 += 8) {
-                unsigned long long rp[8], d[8];
-#pragma unroll
-                for (int k = 0; k < 8; k++) {
-                    const unsigned wv = __shfl_sync(0xffffffffu, myword, i0 + k);
-                    const unsigned v = (wbase + i0 + k) * 32 + lane;
-                    d[k] = 0;
-                    rp[k] = 0;
-                    if ((wv >> lane) & 1u) {
-                        rp[k] = __ldg(F.row_ptr + v);
-                        d[k] = __ldg(F.row_ptr + v + 1) - rp[k];
-                        if (nf && d[k] && F.state[v] >= nfT) d[k] = 0;  // parked in phase 1
-                    }
-                }
-#pragma unroll
-                for (int k = 0; k < 8; k++) {
-                    const unsigned bal = __ballot_sync(0xffffffffu, d[k] != 0);
-                    if (bal == 0) continue;  // warp-uniform
-                    unsigned long long dtot;
-                    const unsigned long long dex = warp_excl_scan_u64(d[k], dtot);
-                    if (d[k]) {
-                        const unsigned v = (wbase + i0 + k) * 32 + lane;
-                        emit_vertex(F, chunk, v, rp[k], d[k], pos + __popc(bal & lanemask_lt()), off + dex);
-                    }
-                    pos += __popc(bal);
-                    off += dtot;
-                }
-            }
-        } else {
-            unsigned long long pos = s_excl.cnt + texcl.cnt;
-            unsigned long long off = s_excl.deg + texcl.deg;
-            unsigned long long rp[kFilterAppPerThread], d[kFilterAppPerThread];
-#pragma unroll
-            for (int j = 0; j < kFilterAppPerThread; j++) {
-                rp[j] = 0;
-                d[j] = 0;
-                if (items[j] != 0xFFFFFFFFu) {
-                    rp[j] = __ldg(F.row_ptr + items[j]);
-                    d[j] = __ldg(F.row_ptr + items[j] + 1) - rp[j];
-                    if (nf && d[j] && F.state[items[j]] >= nfT) d[j] = 0;  // parked in phase 1
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < kFilterAppPerThread; j++) {
-                if (d[j]) {
-                    emit_vertex(F, chunk, items[j], rp[j], d[j], pos, off);
-                    pos++;
-                    off += d[j];
-                }
-            }
-        }
-        __syncthreads();
+    // ---- pass 1: aggregate of this CTA's tile range
+    Pair mine{0, 0};
+    for (unsigned t = t_lo; t < t_hi; t++) {
+        const Pair q = filter_tile<FT_CLASSIFY>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, 0, 0);
+        mine.cnt += q.cnt;
+        mine.deg += q.deg;
+    }
+    Pair agg;
+    block_excl_scan(mine, s_warp, agg);
+    if (threadIdx.x == 0) {
+        slots[b].agg_cnt = agg.cnt;
+        slots[b].agg_deg = agg.deg;
+        st_release_u64(&slots[b].flag, epoch * 4 + 1);
+    }
+    // ---- exclusive prefix: the aggregates of CTAs 0..b-1 (relaxed spin, then one acquire fence)
+    Pair pre{0, 0};
+    for (unsigned j = threadIdx.x; j < b; j += kThreads)
+        while (vload(&slots[j].flag) < epoch * 4 + 1) __nanosleep(32);
+    __threadfence();
+    for (unsigned j = threadIdx.x; j < b; j += kThreads) {
+        pre.cnt += __ldcg(&slots[j].agg_cnt);
+        pre.deg += __ldcg(&slots[j].agg_deg);
+    }
+    Pair excl;
+    block_excl_scan(pre, s_warp, excl);  // excl = sum over all predecessors
+    if (b == G - 1 && threadIdx.x == 0) {
+        const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
+        F.q_off[tc] = td;
+        ct->qlen = tc;
+        ct->qedges = td;
+        ct->ntiles = (td + chunk - 1) / chunk;
+        ct->claim = 0;
+        for (int q = 0; q < kMaxW; q++) ct->pclaim[q] = 0;
+        ct->app_cnt = 0;
+        ct->dense = dense ? 1u : 0u;
+        ct->frontier_edges += td;
+        ct->frontier_vertices += tc;
+    }
+    // ---- pass 2: per tile, re-count (L1/L2-resident re-read) for the per-thread offsets, then emit
+    unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
+    for (unsigned t = t_lo; t < t_hi; t++) {
+        const Pair q = filter_tile<FT_COUNT>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, 0, 0);
+        Pair tot;
+        const Pair tex = block_excl_scan(q, s_warp, tot);
+        filter_tile<FT_EMIT>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, run_cnt + tex.cnt,
+                             run_deg + tex.deg);
+        run_cnt += tot.cnt;
+        run_deg += tot.deg;
     }
 }
 

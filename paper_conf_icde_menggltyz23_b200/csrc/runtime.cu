@@ -276,7 +276,9 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     grid = (grid / L.nw) * L.nw;
     if (grid < L.nw) grid = L.nw;
     L.adv_grid = grid;
-    L.filter_grid = std::max(1, (c->nsm * 4) / (c->single_device ? std::min(c->P, 4) : 1));
+    static const int filter_per_sm = getenv("GUM_FILTER_CTAS_PER_SM") ? std::max(1, atoi(getenv("GUM_FILTER_CTAS_PER_SM"))) : 0;
+    L.filter_grid = std::max(1, (c->nsm * (filter_per_sm ? filter_per_sm : c->filter_occ)) /
+                                    (c->single_device ? std::min(c->P, 4) : 1));
     if (c->split && c->single_device) L.adv_grid = std::max(1, L.adv_grid / c->P);
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
@@ -1270,6 +1272,7 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
         unsigned b = (c->fr[f].V + kFilterAppPerPart - 1) / kFilterAppPerPart;
         parts = std::max(parts, std::max(a, b) + 1);
     }
+    parts = std::max<unsigned>(parts, (unsigned)c->nsm * 8);  // one aggregate slot per filter CTA
     c->lb_parts = parts;
     for (int f = 0; f < c->P; f++) {
         if (!frag_local(c, f)) continue;
