@@ -676,7 +676,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
     typedef typename ValT<ALG>::T VT;
     __shared__ unsigned s_base[kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
-    __shared__ unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
+    __shared__ __align__(16) unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
     // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
     constexpr int PBB = (ALG == ALG_BFS && !MULTI && PB) ? kPbMaxBins : 1;  // (own instantiation:
     // the shared arrays would otherwise shrink L1, which the random probes of the plain path live on)
@@ -834,12 +834,23 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
         __syncthreads();
         // blocked inclusive max-scan of s_head: s_head[e] = index of the vertex owning edge e
         {
+            // each thread's 8 consecutive entries move as two 16-byte vectors (a warp touches 1 KB of
+            // contiguous shared memory: conflict-free, instead of 8-way bank conflicts per scalar access)
+            static_assert(kEdgesPerThread % 4 == 0, "vectorised scan needs kEdgesPerThread % 4 == 0");
             const unsigned b = threadIdx.x * kEdgesPerThread;
             unsigned hv[kEdgesPerThread];
+#pragma unroll
+            for (int q = 0; q < kEdgesPerThread / 4; q++) {
+                const uint4 r4 = *reinterpret_cast<const uint4*>(s_head + b + 4 * q);
+                hv[4 * q] = r4.x;
+                hv[4 * q + 1] = r4.y;
+                hv[4 * q + 2] = r4.z;
+                hv[4 * q + 3] = r4.w;
+            }
             unsigned run = 0;
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
-                const unsigned raw = (b + j < tlen) ? s_head[b + j] : 0u;
+                const unsigned raw = (b + j < tlen) ? hv[j] : 0u;
                 hv[j] = (raw >> 12) == seq ? (raw & 0xFFFu) : 0u;
                 run = hv[j] > run ? hv[j] : run;
                 hv[j] = run;
@@ -855,9 +866,16 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             if (lane_id() == 31) s_wmax[threadIdx.x >> 5] = inc;
             __syncthreads();
             for (unsigned i = 0; i < (threadIdx.x >> 5); i++) excl = s_wmax[i] > excl ? s_wmax[i] : excl;
+            // (entries >= tlen are written too: untagged values never match a later sequence tag)
 #pragma unroll
-            for (int j = 0; j < kEdgesPerThread; j++)
-                if (b + j < tlen) s_head[b + j] = hv[j] > excl ? hv[j] : excl;
+            for (int q = 0; q < kEdgesPerThread / 4; q++) {
+                uint4 w4;
+                w4.x = hv[4 * q] > excl ? hv[4 * q] : excl;
+                w4.y = hv[4 * q + 1] > excl ? hv[4 * q + 1] : excl;
+                w4.z = hv[4 * q + 2] > excl ? hv[4 * q + 2] : excl;
+                w4.w = hv[4 * q + 3] > excl ? hv[4 * q + 3] : excl;
+                *reinterpret_cast<uint4*>(s_head + b + 4 * q) = w4;
+            }
         }
         __syncthreads();
 
