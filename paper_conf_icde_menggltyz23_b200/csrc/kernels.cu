@@ -672,7 +672,10 @@ __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned
 }
 
 template <int ALG, bool MULTI, bool PB = false>
-__global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
+#ifndef GUM_ADV_MINB_BFS
+#define GUM_ADV_MINB_BFS 4
+#endif
+__global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_BFS * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
     __shared__ unsigned s_base[kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
@@ -687,9 +690,6 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
     __shared__ unsigned s_wmax[kAdvThreads / 32];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
-    __shared__ int s_f;
-    __shared__ unsigned long long s_t;
-    __shared__ int s_stolen;
 
     RunCtl* rc = c.rctl[w0];
     if (vload(&rc->done) || vload(&rc->tail)) return;  // tail engine runs this iteration
@@ -719,119 +719,187 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0;
 
-    // next own chunk claimed one tile ahead (its atomic overlaps the current chunk's expansion)
+    // Chunk claims run one chunk ahead of the expansion (thread 0): while chunk n is expanded, chunk n+1
+    // is already claimed and its staging data (chunk table entries, degree prefix, col base, source
+    // value) is in flight into registers, so a chunk's staging costs no exposed memory round trip. The
+    // own-queue claim atomic itself is issued one more chunk ahead (pf_f / pf_t).
     int pf_f = -1;
     unsigned long long pf_t = 0;
-    for (;;) {
-        if (threadIdx.x == 0) {
-            int f = -1;
-            unsigned long long t = 0;
-            int stolen = 0;
-            if (planned) {
-                // NEXT-2: process the chunk ranges the plan assigned to this worker, queue by queue
-                while (own_cursor < c.P) {
-                    const int g = (w + own_cursor) % c.P;
-                    const unsigned lo = rc->plan_lo[g][w], hi = rc->plan_hi[g][w];
-                    if (hi > lo) {
-                        const unsigned long long tt = lo + atomicAdd(&c.f[g].ctl->pclaim[w], 1ull);
-                        if (tt < hi) {
-                            f = g;
-                            t = tt;
-                            stolen = g != w;
-                            break;
-                        }
-                    }
-                    own_cursor++;
-                }
-            } else if (pf_f >= 0 && pf_t < s_ntiles[pf_f]) {
-                f = pf_f;
-                t = pf_t;
-            } else {
-                if (pf_f >= 0) own_cursor++;  // prefetched claim overflowed: that queue is drained
-                while (own_cursor < c.P) {
-                    int g = (w + own_cursor) % c.P;
-                    if (s_owner[g] == (unsigned)w) {
-                        unsigned long long tt = atomicAdd(&c.f[g].ctl->claim, 1ull);
-                        if (tt < s_ntiles[g]) {
-                            f = g;
-                            t = tt;
-                            break;
-                        }
-                    }
-                    own_cursor++;
-                }
-            }
-            pf_f = -1;
-            if (f < 0 && steal && !planned) {
-                // FSteal: claim a chunk of the active owner queue with the most remaining chunks
-                for (;;) {
-                    int best = -1;
-                    unsigned long long best_rem = 0;
-                    for (int g = 0; g < c.P; g++) {
-                        if (s_owner[g] == (unsigned)w) continue;
-                        unsigned long long cl = vload(&c.f[g].ctl->claim);
-                        unsigned long long rem = s_ntiles[g] > cl ? s_ntiles[g] - cl : 0;
-                        if (rem > best_rem) {
-                            best_rem = rem;
-                            best = g;
-                        }
-                    }
-                    if (best < 0) break;
-                    unsigned long long tt = atomicAdd(&c.f[best].ctl->claim, 1ull);
-                    if (tt < s_ntiles[best]) {
-                        f = best;
+    auto claim_next = [&](int& f_out, unsigned long long& t_out, int& stolen_out) {
+        int f = -1;
+        unsigned long long t = 0;
+        int stolen = 0;
+        if (planned) {
+            // NEXT-2: process the chunk ranges the plan assigned to this worker, queue by queue
+            while (own_cursor < c.P) {
+                const int g = (w + own_cursor) % c.P;
+                const unsigned lo = rc->plan_lo[g][w], hi = rc->plan_hi[g][w];
+                if (hi > lo) {
+                    const unsigned long long tt = lo + atomicAdd(&c.f[g].ctl->pclaim[w], 1ull);
+                    if (tt < hi) {
+                        f = g;
                         t = tt;
-                        stolen = 1;
+                        stolen = g != w;
                         break;
                     }
                 }
+                own_cursor++;
             }
-            s_f = f;
-            s_t = t;
-            s_stolen = stolen;
-            if (f >= 0 && !stolen && !planned) {
-                pf_f = f;
-                pf_t = atomicAdd(&c.f[f].ctl->claim, 1ull);
+        } else if (pf_f >= 0 && pf_t < s_ntiles[pf_f]) {
+            f = pf_f;
+            t = pf_t;
+        } else {
+            if (pf_f >= 0) own_cursor++;  // prefetched claim overflowed: that queue is drained
+            while (own_cursor < c.P) {
+                int g = (w + own_cursor) % c.P;
+                if (s_owner[g] == (unsigned)w) {
+                    unsigned long long tt = atomicAdd(&c.f[g].ctl->claim, 1ull);
+                    if (tt < s_ntiles[g]) {
+                        f = g;
+                        t = tt;
+                        break;
+                    }
+                }
+                own_cursor++;
             }
         }
-        __syncthreads();
-        const int f = s_f;
-        if (f < 0) break;
-        const unsigned long long t = s_t;
-        const bool stolen = s_stolen != 0;
+        pf_f = -1;
+        if (f < 0 && steal && !planned) {
+            // FSteal: claim a chunk of the active owner queue with the most remaining chunks
+            for (;;) {
+                int best = -1;
+                unsigned long long best_rem = 0;
+                for (int g = 0; g < c.P; g++) {
+                    if (s_owner[g] == (unsigned)w) continue;
+                    unsigned long long cl = vload(&c.f[g].ctl->claim);
+                    unsigned long long rem = s_ntiles[g] > cl ? s_ntiles[g] - cl : 0;
+                    if (rem > best_rem) {
+                        best_rem = rem;
+                        best = g;
+                    }
+                }
+                if (best < 0) break;
+                unsigned long long tt = atomicAdd(&c.f[best].ctl->claim, 1ull);
+                if (tt < s_ntiles[best]) {
+                    f = best;
+                    t = tt;
+                    stolen = 1;
+                    break;
+                }
+            }
+        }
+        f_out = f;
+        t_out = t;
+        stolen_out = stolen;
+        if (f >= 0 && !stolen && !planned) {
+            pf_f = f;
+            pf_t = atomicAdd(&c.f[f].ctl->claim, 1ull);
+        }
+    };
+    // staging descriptor of a claimed chunk (WCC iteration 0 runs on the static destination-blocked
+    // queue: edges contiguous in queue order)
+    struct ChunkRef {
+        int f;
+        unsigned long long t;
+        int stolen;
+        unsigned i0, nv, tlen;
+    };
+    auto chunk_ref = [&](int f, unsigned long long t, int stolen) {
+        ChunkRef r{f, t, stolen, 0u, 0u, 0u};
+        if (f < 0) return r;
         const FragPtrs& F = c.f[f];
-        const unsigned long long tb = t * CH;
-        const unsigned long long qe = s_qedges[f];
-        const unsigned tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
-        // WCC iteration 0 runs on the static destination-blocked queue (edges contiguous in queue order)
         const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
         const unsigned* const tilep = sq ? F.sq_tile : F.tile;
-        const unsigned* const qvp = sq ? F.sq_q_v : F.q_v;
-        const unsigned long long* const qoffp = sq ? F.sq_q_off : F.q_off;
-        const unsigned* const colp = sq ? F.sq_col : F.col;
-        const unsigned i0 = __ldg(tilep + t);
+        const unsigned long long tb = t * CH, qe = s_qedges[f];
+        r.tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
+        r.i0 = __ldg(tilep + t);
         const unsigned i1 = (t + 1 < s_ntiles[f]) ? __ldg(tilep + t + 1) : (unsigned)(s_qlen[f] - 1);
-        const unsigned nv = i1 - i0 + 1;
+        r.nv = i1 - r.i0 + 1;
+        return r;
+    };
+    // per-vertex staging values of queue entry i of chunk r (vertex slot kk): edge prefix, col base, value
+    auto stage_load = [&](const ChunkRef& r, unsigned kk, unsigned long long& off, unsigned& base, unsigned& u) {
+        const FragPtrs& F = c.f[r.f];
+        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const unsigned i = r.i0 + kk;
+        const unsigned long long tb = r.t * CH;
+        off = __ldcs((sq ? F.sq_q_off : F.q_off) + i);
+        // PR's (and WCC iteration 0's) blocked queue stores edges contiguously in queue order:
+        // col index == q_off + j
+        base = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(F.q_base + i)));
+        u = (ALG != ALG_BFS) ? __ldcs((sq ? F.sq_q_v : F.q_v) + i) : 0u;
+    };
+    auto value_of = [&](const ChunkRef& r, unsigned u) -> VT {
+        if (ALG == ALG_PR) return (VT)__ldcg(c.f[r.f].cx + u);
+        if (ALG != ALG_BFS) return (VT)__ldcg(c.f[r.f].state + u);
+        return (VT)0;
+    };
+
+    __shared__ int s_nf;
+    __shared__ unsigned long long s_nt;
+    __shared__ int s_nstolen;
+    if (threadIdx.x == 0) {
+        int f0;
+        unsigned long long t0c;
+        int st0;
+        claim_next(f0, t0c, st0);
+        s_nf = f0;
+        s_nt = t0c;
+        s_nstolen = st0;
+    }
+    __syncthreads();
+    ChunkRef cur = chunk_ref(s_nf, s_nt, s_nstolen);
+    unsigned long long p_off = 0;  // prefetched staging values of vertex slot threadIdx.x
+    unsigned p_base = 0, p_u = 0;
+    VT p_val = (VT)0;
+    if (cur.f >= 0 && threadIdx.x < cur.nv) {
+        stage_load(cur, threadIdx.x, p_off, p_base, p_u);
+        p_val = value_of(cur, p_u);
+    }
+    __syncthreads();  // everyone read s_nf before it is reused
+    for (;;) {
+        const int f = cur.f;
+        if (f < 0) break;
+        const unsigned long long t = cur.t;
+        const bool stolen = cur.stolen != 0;
+        const FragPtrs& F = c.f[f];
+        const unsigned long long tb = t * CH;
+        const unsigned tlen = cur.tlen;
+        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const unsigned* const colp = sq ? F.sq_col : F.col;
+        const unsigned nv = cur.nv;
+        if (threadIdx.x == 0) {
+            int nf_;
+            unsigned long long nt_;
+            int ns_;
+            claim_next(nf_, nt_, ns_);
+            s_nf = nf_;
+            s_nt = nt_;
+            s_nstolen = ns_;
+        }
 
         // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
         seq++;
         for (unsigned kk = threadIdx.x; kk < nv; kk += kAdvThreads) {
-            const unsigned i = i0 + kk;
-            const unsigned long long off = __ldcs(qoffp + i);
-            // PR's (and WCC iteration 0's) blocked queue stores edges contiguously in queue order:
-            // col index == q_off + j
-            s_base[kk] = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(F.q_base + i)));
-            if (ALG == ALG_PR) {
-                const unsigned u = __ldcs(F.q_v + i);
-                s_val[kk] = (VT)__ldcg(F.cx + u);
-            } else if (ALG != ALG_BFS) {
-                const unsigned u = __ldcs(qvp + i);
-                s_val[kk] = (VT)__ldcg(F.state + u);
+            unsigned long long off;
+            unsigned base, u;
+            VT val;
+            if (kk < (unsigned)kAdvThreads) {
+                off = p_off;
+                base = p_base;
+                val = p_val;
+            } else {
+                stage_load(cur, kk, off, base, u);
+                val = value_of(cur, u);
             }
+            s_base[kk] = base;
+            if (ALG != ALG_BFS) s_val[kk] = val;
             const long long rel = (long long)off - (long long)tb;
             if (rel > 0 && rel < (long long)tlen) s_head[rel] = (seq << 12) | kk;
         }
         __syncthreads();
+        // the next chunk's chunk-table entries load while this chunk is scanned
+        const ChunkRef nxt = chunk_ref(s_nf, s_nt, s_nstolen);
         // blocked inclusive max-scan of s_head: s_head[e] = index of the vertex owning edge e
         {
             // each thread's 8 consecutive entries move as two 16-byte vectors (a warp touches 1 KB of
@@ -879,6 +947,11 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
         }
         __syncthreads();
 
+        // the next chunk's per-vertex staging values load while this chunk is expanded
+        if (nxt.f >= 0 && threadIdx.x < nxt.nv) {
+            stage_load(nxt, threadIdx.x, p_off, p_base, p_u);
+            p_val = value_of(nxt, p_u);
+        }
         // ---- expand: striped edges, coalesced streaming col/w loads
         unsigned vv[kEdgesPerThread];
         VT cv[kEdgesPerThread];
@@ -1095,6 +1168,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? 5 * 256 / kAdv
             }
         }
         __syncthreads();
+        cur = nxt;
     }
     // run counters (warp-reduced) and the per-worker busy window of this iteration
 #pragma unroll
