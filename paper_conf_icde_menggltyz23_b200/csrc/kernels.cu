@@ -232,17 +232,22 @@ __device__ __forceinline__ unsigned long long warp_excl_scan_u64(unsigned long l
 //   FT_EMIT     (pass 2b): writes the queue entries from pos/off on, clears the consumed bitmap words and
 //                          the far bits of accepted vertices.
 enum { FT_CLASSIFY = 0, FT_COUNT = 1, FT_EMIT = 2 };
+// per-thread near-far bookkeeping, reduced per warp before touching the fragment's counters (they are
+// single addresses: per-vertex atomics there serialise in the L2 atomic unit)
+struct NfAcc {
+    unsigned long long parked = 0, unparked = 0;
+    unsigned min_dist = 0xFFFFFFFFu;
+};
 template <int MODE>
-__device__ __forceinline__ bool filter_accept(const FragPtrs& F, FragCtl* ct, unsigned v, bool nf, unsigned nfT,
-                                              unsigned fslot) {
+__device__ __forceinline__ bool filter_accept(const FragPtrs& F, unsigned v, bool nf, unsigned nfT, NfAcc& acc) {
     if (!nf) return true;
     if (MODE == FT_CLASSIFY) {
         const unsigned dist = F.state[v];
         if (dist < nfT) return true;
         const unsigned bit = 1u << (v & 31);
         const unsigned ob = atomicOr(F.far + (v >> 5), bit);
-        if (!(ob & bit)) atomicAdd(&ct->far_cnt, 1ull);
-        atomicMin(&ct->far_min[fslot], dist);
+        if (!(ob & bit)) acc.parked++;
+        acc.min_dist = dist < acc.min_dist ? dist : acc.min_dist;
         return false;
     }
     if (F.state[v] >= nfT) return false;  // parked in pass 1
@@ -250,15 +255,25 @@ __device__ __forceinline__ bool filter_accept(const FragPtrs& F, FragCtl* ct, un
         const unsigned bit = 1u << (v & 31);
         if (F.far[v >> 5] & bit) {
             const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
-            if (ob & bit) atomicAdd(&ct->far_cnt, ~0ull);  // -1
+            if (ob & bit) acc.unparked++;
         }
     }
     return true;
 }
 
+// warp-reduce the near-far counters and apply them to the fragment (lane 0 of each warp)
+__device__ __forceinline__ void nf_flush(FragCtl* ct, unsigned fslot, const NfAcc& a) {
+    const unsigned long long p = warp_sum_u64(a.parked), u = warp_sum_u64(a.unparked);
+    const unsigned m = __reduce_min_sync(0xffffffffu, a.min_dist);
+    if (lane_id() == 0) {
+        if (p != u) atomicAdd(&ct->far_cnt, p - u);  // two's complement: a net decrement wraps correctly
+        if (m != 0xFFFFFFFFu) atomicMin(&ct->far_min[fslot], m);
+    }
+}
+
 template <int MODE>
-__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, FragCtl* ct, unsigned tile, bool dense, bool sweep,
-                                            bool nf, unsigned nfT, unsigned fslot, unsigned nwords, unsigned app_cnt,
+__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsigned tile, bool dense, bool sweep,
+                                            bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt,
                                             unsigned chunk, unsigned long long pos, unsigned long long off) {
     const unsigned lane = lane_id();
     Pair mine{0, 0};
@@ -295,7 +310,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, FragCtl* ct, unsi
             for (int q = 0; q < kDenseVertsPerThread; q++) {
                 if ((bits >> q) & 1u) {
                     const unsigned long long d = rpv[q + 1] - rpv[q];
-                    if (d && filter_accept<MODE>(F, ct, vb + q, nf, nfT, fslot)) {
+                    if (d && filter_accept<MODE>(F, vb + q, nf, nfT, acc)) {
                         if (MODE == FT_EMIT) emit_vertex(F, chunk, vb + q, rpv[q], d, pos + mine.cnt, off + mine.deg);
                         mine.cnt += 1;
                         mine.deg += d;
@@ -326,7 +341,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, FragCtl* ct, unsi
         }
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
-            if (d[j] && filter_accept<MODE>(F, ct, items[j], nf, nfT, fslot)) {
+            if (d[j] && filter_accept<MODE>(F, items[j], nf, nfT, acc)) {
                 if (MODE == FT_EMIT) emit_vertex(F, chunk, items[j], rp0[j], d[j], pos + mine.cnt, off + mine.deg);
                 mine.cnt += 1;
                 mine.deg += d[j];
@@ -343,44 +358,64 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, FragCtl* ct, unsi
 // counts its contiguous tile range, publishes the aggregate, sums its predecessors' aggregates (one
 // parallel read, no serial look-back chain) and re-walks its range emitting entries in vertex order.
 __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+    // Prologue by thread 0 only, broadcast through shared memory: the run-control fields are a handful of
+    // L2 lines that every CTA of every kernel reads, and per-warp loads of one address serialise in its
+    // L2 slice (with ~600 CTAs x 8 warps that alone cost tens of microseconds per launch).
+    struct Pro {
+        unsigned go, sweep, dense, nfT, fslot, app_cnt, b, pad;
+        unsigned long long epoch;
+    };
+    __shared__ Pro s_pro;
+    __shared__ Pair s_warp[kThreads / 32];
     RunCtl* rc = c.rctl[w0];
-    if (vload(&rc->done) || vload(&rc->skip_filter)) return;
     const int f = blockIdx.y;
-    const unsigned o = rc->owner[f];
-    if ((int)o < w0 || (int)o >= w0 + nw) return;
     const FragPtrs& F = c.f[f];
     FragCtl* ct = F.ctl;
-    // the advance that produced these activations either appended them (sparse) or only set bits
-    // SSSP near-far: only vertices with dist < T enter the queue; the rest are parked in F.far
     const bool nf = c.nf_delta != 0;
-    const bool sweep = nf && vload(&rc->nf_sweep) != 0;
-    const unsigned nfT = nf ? (unsigned)(rc->nf_T < 0xFFFFFFFFull ? rc->nf_T : 0xFFFFFFFFull) : GUM_INF;
-    const unsigned fslot = rc->nf_sweeps & 1u;
-    const bool dense = sweep || vload(&rc->next_dense) != 0;
-    const unsigned app_cnt = dense ? 0u : vload(&ct->app_cnt);
+    if (threadIdx.x == 0) {
+        Pro p{};
+        const unsigned o = vload(&rc->owner[f]);
+        p.go = !vload(&rc->done) && !vload(&rc->skip_filter) && (int)o >= w0 && (int)o < w0 + nw;
+        if (p.go) {
+            // SSSP near-far: only vertices with dist < T enter the queue; the rest are parked in F.far
+            p.sweep = nf && vload(&rc->nf_sweep) != 0;
+            const unsigned long long T = vload(&rc->nf_T);
+            p.nfT = nf ? (unsigned)(T < 0xFFFFFFFFull ? T : 0xFFFFFFFFull) : GUM_INF;
+            p.fslot = vload(&rc->nf_sweeps) & 1u;
+            // the advance that produced these activations either appended them (sparse) or only set bits
+            p.dense = p.sweep || vload(&rc->next_dense) != 0;
+            p.app_cnt = p.dense ? 0u : vload(&ct->app_cnt);
+            p.epoch = vload(&rc->epoch);
+            p.b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
+        }
+        s_pro = p;
+    }
+    __syncthreads();
+    if (!s_pro.go) return;
+    const bool sweep = s_pro.sweep != 0;
+    const unsigned nfT = s_pro.nfT;
+    const unsigned fslot = s_pro.fslot;
+    const bool dense = s_pro.dense != 0;
+    const unsigned app_cnt = s_pro.app_cnt;
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
     const unsigned per = dense ? kDenseWordsPerPart : kFilterAppPerPart;
     const unsigned n_tiles = (unsigned)((n_items + per - 1) / per);
-    const unsigned long long epoch = rc->epoch;
+    const unsigned long long epoch = s_pro.epoch;
     const unsigned chunk = c.chunk;
     LBSlot* slots = c.lb[f];
     // small lists: only as many CTAs as tiles take part (the others leave before the prefix exchange)
     const unsigned G = n_tiles < gridDim.x ? (n_tiles ? n_tiles : 1u) : gridDim.x;
-
-    __shared__ unsigned s_b;
-    __shared__ Pair s_warp[kThreads / 32];
-    if (threadIdx.x == 0) s_b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
-    __syncthreads();
-    const unsigned b = s_b;
+    const unsigned b = s_pro.b;
     if (b >= G) return;
     const unsigned t_lo = (unsigned)(((unsigned long long)n_tiles * b) / G);
     const unsigned t_hi = (unsigned)(((unsigned long long)n_tiles * (b + 1)) / G);
 
     // ---- pass 1: aggregate of this CTA's tile range
     Pair mine{0, 0};
+    NfAcc nfa;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_CLASSIFY>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, 0, 0);
         mine.cnt += q.cnt;
         mine.deg += q.deg;
     }
@@ -418,14 +453,15 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     // ---- pass 2: per tile, re-count (L1/L2-resident re-read) for the per-thread offsets, then emit
     unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_COUNT>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_COUNT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, 0, 0);
         Pair tot;
         const Pair tex = block_excl_scan(q, s_warp, tot);
-        filter_tile<FT_EMIT>(F, ct, t, dense, sweep, nf, nfT, fslot, nwords, app_cnt, chunk, run_cnt + tex.cnt,
+        filter_tile<FT_EMIT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, run_cnt + tex.cnt,
                              run_deg + tex.deg);
         run_cnt += tot.cnt;
         run_deg += tot.deg;
     }
+    if (nf) nf_flush(ct, fslot, nfa);
 }
 
 // ------------------------------------------------------------------------------------------ control
@@ -690,29 +726,44 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     __shared__ unsigned s_wmax[kAdvThreads / 32];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
+    __shared__ unsigned long long s_cnt[kMaxW][4];  // per fragment: edges, chunks, stolen edges, stolen chunks
 
+    // Prologue: thread 0 reads the run-control header once per CTA (per-warp loads of these few shared
+    // addresses serialise in their L2 slice), threads < P the fragments' queue sizes.
+    __shared__ unsigned s_hdr[6];  // go, m, k, steal_ok, next_dense, pb
     RunCtl* rc = c.rctl[w0];
-    if (vload(&rc->done) || vload(&rc->tail)) return;  // tail engine runs this iteration
-    if (ALG == ALG_BFS && vload(&rc->pull)) return;   // bottom-up step runs this iteration
     const int w = w0 + (int)(blockIdx.x % (unsigned)nw);
-    const unsigned m = rc->m;
-    if ((unsigned)w >= m) return;  // evicted by OSteal: this worker's GPU only serves as memory
-    const unsigned k = rc->iter - 1;
-    const bool steal = rc->steal_ok != 0;
-    const bool next_dense = rc->next_dense != 0;
-    const bool planned = c.fsteal == 2 && m == (unsigned)c.P;  // NEXT-2 plan (else the steal queue)
-    const bool pb = (ALG == ALG_BFS && !MULTI && PB) && rc->pb != 0;
-    if (pb)
-        for (unsigned b = threadIdx.x; b < (unsigned)PBB; b += kAdvThreads) s_pbcnt[b] = 0;
-    const unsigned long long t0 = globaltimer();
+    if (threadIdx.x == 0) {
+        const unsigned m_ = vload(&rc->m);
+        // tail engine or bottom-up step runs this iteration / evicted by OSteal (the GPU only serves as memory)
+        s_hdr[0] = !vload(&rc->done) && !vload(&rc->tail) && !(ALG == ALG_BFS && vload(&rc->pull)) && (unsigned)w < m_;
+        s_hdr[1] = m_;
+        s_hdr[2] = vload(&rc->iter) - 1;
+        s_hdr[3] = vload(&rc->steal_ok);
+        s_hdr[4] = vload(&rc->next_dense);
+        s_hdr[5] = (ALG == ALG_BFS && !MULTI && PB) ? vload(&rc->pb) : 0u;
+    }
     if (threadIdx.x < (unsigned)c.P) {
         FragCtl* ct = c.f[threadIdx.x].ctl;
         s_ntiles[threadIdx.x] = vload(&ct->ntiles);
         s_qlen[threadIdx.x] = vload(&ct->qlen);
         s_qedges[threadIdx.x] = vload(&ct->qedges);
-        s_owner[threadIdx.x] = rc->owner[threadIdx.x];
+        s_owner[threadIdx.x] = vload(&rc->owner[threadIdx.x]);
+        s_cnt[threadIdx.x][0] = s_cnt[threadIdx.x][1] = s_cnt[threadIdx.x][2] = s_cnt[threadIdx.x][3] = 0;
     }
     __syncthreads();
+    if (!s_hdr[0]) return;
+    const unsigned m = s_hdr[1];
+    const unsigned k = s_hdr[2];
+    const bool steal = s_hdr[3] != 0;
+    const bool next_dense = s_hdr[4] != 0;
+    const bool planned = c.fsteal == 2 && m == (unsigned)c.P;  // NEXT-2 plan (else the steal queue)
+    const bool pb = (ALG == ALG_BFS && !MULTI && PB) && s_hdr[5] != 0;
+    if (pb) {
+        for (unsigned b = threadIdx.x; b < (unsigned)PBB; b += kAdvThreads) s_pbcnt[b] = 0;
+        __syncthreads();
+    }
+    const unsigned long long t0 = globaltimer();
     const unsigned CH = c.chunk;
     for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kAdvThreads) s_head[e] = 0;
     unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
@@ -1157,11 +1208,13 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
             }
         }
         if (threadIdx.x == 0) {
-            atomicAdd(&F.ctl->edges_done, (unsigned long long)tlen);
-            atomicAdd(&F.ctl->chunks_done, 1ull);
+            // conservation counters of the chunk's fragment, accumulated per CTA (flushed at exit: the
+            // fragment counters are single addresses)
+            s_cnt[f][0] += tlen;
+            s_cnt[f][1] += 1;
             if (stolen) {
-                atomicAdd(&F.ctl->edges_stolen, (unsigned long long)tlen);
-                atomicAdd(&F.ctl->chunks_stolen, 1ull);
+                s_cnt[f][2] += tlen;
+                s_cnt[f][3] += 1;
                 e_stolen += tlen;
             } else {
                 e_own += tlen;
@@ -1171,6 +1224,15 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         cur = nxt;
     }
     // run counters (warp-reduced) and the per-worker busy window of this iteration
+    if (threadIdx.x < (unsigned)c.P && s_cnt[threadIdx.x][1]) {
+        FragCtl* ct = c.f[threadIdx.x].ctl;
+        atomicAdd(&ct->edges_done, s_cnt[threadIdx.x][0]);
+        atomicAdd(&ct->chunks_done, s_cnt[threadIdx.x][1]);
+        if (s_cnt[threadIdx.x][3]) {
+            atomicAdd(&ct->edges_stolen, s_cnt[threadIdx.x][2]);
+            atomicAdd(&ct->chunks_stolen, s_cnt[threadIdx.x][3]);
+        }
+    }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         remote += __shfl_xor_sync(0xffffffffu, remote, o);
@@ -1278,8 +1340,13 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
             base = __shfl_sync(grp, base, leader);
             unsigned* nxt = (it & 1) ? T.q_v : T.app;
             nxt[base + __popc(grp & lanemask_lt())] = lu;
-            atomicAdd(&T.ctl->tedges[ns], __ldg(T.row_ptr + lu + 1) - __ldg(T.row_ptr + lu));
             acts++;
+        }
+        // out-edges of the appended vertices: one atomic per group (the counter is a single address)
+        const unsigned long long deg = need ? __ldg(c.f[tf].row_ptr + lu + 1) - __ldg(c.f[tf].row_ptr + lu) : 0ull;
+        if (need) {
+            const unsigned hi = __reduce_add_sync(grp, (unsigned)(deg >> 16)), lo = __reduce_add_sync(grp, (unsigned)(deg & 0xFFFFu));
+            if (lane == __ffs(grp) - 1) atomicAdd(&c.f[tf].ctl->tedges[ns], ((unsigned long long)hi << 16) + lo);
         }
     }
     return acts;
@@ -1287,16 +1354,28 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
 
 template <int ALG, bool MULTI>
 __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
+    __shared__ unsigned s_n[kMaxW], s_nsplit, s_go;
+    __shared__ unsigned long long s_tn[kMaxW], s_te[kMaxW];
     RunCtl* rc = c.rctl[w0];
-    if (!vload(&rc->tail) || vload(&rc->done)) return;
+    __shared__ unsigned s_hdr[4];  // gen, k0, nfT, fslot
+    if (threadIdx.x == 0) {
+        s_go = vload(&rc->tail) && !vload(&rc->done);
+        s_hdr[0] = vload(&rc->tbar_gen);
+        s_hdr[1] = vload(&rc->iter) - 1;  // control already counted the first tail iteration
+        const unsigned long long T = vload(&rc->nf_T);
+        s_hdr[2] = (unsigned)(T < 0xFFFFFFFFull ? T : 0xFFFFFFFFull);
+        s_hdr[3] = vload(&rc->nf_sweeps) & 1u;
+    }
+    __syncthreads();
+    if (!s_go) return;
     const unsigned lane = lane_id();
     const unsigned nwarps = gridDim.x * (kTailThreads / 32);
     const unsigned gw = blockIdx.x * (kTailThreads / 32) + (threadIdx.x >> 5);
-    unsigned gen = vload(&rc->tbar_gen);
-    const unsigned k0 = rc->iter - 1;  // control already counted the first tail iteration
+    unsigned gen = s_hdr[0];
+    const unsigned k0 = s_hdr[1];
     const bool nf = (ALG == ALG_SSSP) && c.nf_delta != 0;
-    const unsigned nfT = nf ? (unsigned)(rc->nf_T < 0xFFFFFFFFull ? rc->nf_T : 0xFFFFFFFFull) : GUM_INF;
-    const unsigned fslot = rc->nf_sweeps & 1u;
+    const unsigned nfT = nf ? s_hdr[2] : GUM_INF;
+    const unsigned fslot = s_hdr[3];
     const int nfrag = MULTI ? c.P : 1;
     gum_iter_trace* tr = c.trace[w0];
     TailSplit* split = c.tsplit[w0];
@@ -1310,11 +1389,15 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         const unsigned k = k0 + it;
         unsigned long long it_edges = 0;
         unsigned long long n_all = 0;
+        // list sizes: one load per CTA (per-warp loads of these single addresses serialise in L2)
+        if (threadIdx.x < (unsigned)nfrag)
+            s_n[threadIdx.x] = it == 0 ? (unsigned)vload(&c.f[threadIdx.x].ctl->qlen) : vload(&c.f[threadIdx.x].ctl->tcnt[cs]);
+        __syncthreads();
         // ---- phase 1: one warp per listed vertex; high-degree vertices go to the split list
         for (int f = 0; f < nfrag; f++) {
             const FragPtrs& F = c.f[f];
             const unsigned* cur = (it & 1) ? F.app : F.q_v;
-            const unsigned n = it == 0 ? (unsigned)vload(&F.ctl->qlen) : vload(&F.ctl->tcnt[cs]);
+            const unsigned n = s_n[f];
             n_all += n;
             if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
             for (unsigned i = gw; i < n; i += nwarps) {
@@ -1378,7 +1461,9 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         }
         tail_barrier(rc, gridDim.x, gen);
         // ---- phase 2: split vertices, 256-edge segments dealt round-robin over every warp
-        const unsigned nsplit = min(vload(&rc->tsplit_cnt[it & 1]), kTailSplitCap);
+        if (threadIdx.x == 0) s_nsplit = min(vload(&rc->tsplit_cnt[it & 1]), kTailSplitCap);
+        __syncthreads();
+        const unsigned nsplit = s_nsplit;
         if (nsplit) {
             for (unsigned sid = gw;; sid += nwarps) {
                 // locate segment sid: prefix of segment counts over the split list (warp-parallel)
@@ -1422,10 +1507,15 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         }
         // appends of phase 2 (and the trace row) must be complete before the counts are read
         if (nsplit || tr) tail_barrier(rc, gridDim.x, gen);
+        if (threadIdx.x < (unsigned)nfrag) {
+            s_tn[threadIdx.x] = vload(&c.f[threadIdx.x].ctl->tcnt[ns]);
+            s_te[threadIdx.x] = vload(&c.f[threadIdx.x].ctl->tedges[ns]);
+        }
+        __syncthreads();
         unsigned long long total_next = 0, next_edges = 0;
         for (int f = 0; f < nfrag; f++) {
-            total_next += vload(&c.f[f].ctl->tcnt[ns]);
-            next_edges += vload(&c.f[f].ctl->tedges[ns]);
+            total_next += s_tn[f];
+            next_edges += s_te[f];
         }
         // every CTA must take the same decision: only values that are final after the barrier (next-list
         // counters) enter it -- not the error flag, which next-iteration work of a fast CTA may already
@@ -1509,12 +1599,17 @@ static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t
 template <bool MULTI>
 __global__ void __launch_bounds__(kThreads) k_bfs_pull(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
-    if (!vload(&rc->pull) || vload(&rc->done) || vload(&rc->tail)) return;
     const int f = blockIdx.y;
-    const unsigned o = rc->owner[f];
-    if ((int)o < w0 || (int)o >= w0 + nw) return;
+    __shared__ unsigned s_go, s_k;  // prologue by one thread per CTA (hot run-control addresses)
+    if (threadIdx.x == 0) {
+        const unsigned o = vload(&rc->owner[f]);
+        s_go = vload(&rc->pull) && !vload(&rc->done) && !vload(&rc->tail) && (int)o >= w0 && (int)o < w0 + nw;
+        s_k = vload(&rc->iter) - 1;
+    }
+    __syncthreads();
+    if (!s_go) return;
     const FragPtrs& F = c.f[f];
-    const unsigned k = rc->iter - 1;
+    const unsigned k = s_k;
     const unsigned lane = lane_id();
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned warps = gridDim.x * (kThreads / 32);
@@ -1624,10 +1719,16 @@ __global__ void __launch_bounds__(kThreads) k_pb_apply(const __grid_constant__ D
 // ------------------------------------------------------------------------------------------ PR finalize
 __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
-    if (vload(&rc->done)) return;
     const int f = blockIdx.y;
-    const unsigned o = rc->owner[f];
-    if ((int)o < w0 || (int)o >= w0 + nw) return;
+    __shared__ unsigned s_go;  // prologue by one thread per CTA (hot run-control addresses)
+    __shared__ double s_D;
+    if (threadIdx.x == 0) {
+        const unsigned o = vload(&rc->owner[f]);
+        s_go = !vload(&rc->done) && (int)o >= w0 && (int)o < w0 + nw;
+        s_D = vload(&rc->pr_D);
+    }
+    __syncthreads();
+    if (!s_go) return;
     const FragPtrs& F = c.f[f];
     // PR's frontier queue is static: re-arm its steal-queue head for the next advance (every
     // advance of this iteration has finished: kernel boundary / cross-device barrier)
@@ -1635,7 +1736,7 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
         F.ctl->claim = 0;
         for (int q = 0; q < kMaxW; q++) F.ctl->pclaim[q] = 0;
     }
-    const double N = (double)c.num_vertices, d = c.pr_d, D = rc->pr_D;
+    const double N = (double)c.num_vertices, d = c.pr_d, D = s_D;
     double dang = 0.0, res = 0.0;
     for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
         const double xo = F.x[i];

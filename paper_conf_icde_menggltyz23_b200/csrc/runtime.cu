@@ -1436,9 +1436,9 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             CK(cudaMemcpyAsync(c->h_rctl, c->rctl[hu], sizeof(RunCtl), cudaMemcpyDeviceToHost, c->stream[hu]));
             CK(cudaStreamSynchronize(c->stream[hu]));
             if (getenv("GUM_DEBUG"))
-                fprintf(stderr, "[gum] host loop: iter=%u done=%u tail=%u err=%u bodies=%u tail_iters=%u\n",
+                fprintf(stderr, "[gum] host loop: iter=%u done=%u tail=%u err=%u bodies=%u tail_iters=%u nf_sweeps=%u\n",
                         c->h_rctl->iter, c->h_rctl->done, c->h_rctl->tail, c->h_rctl->err, c->h_rctl->bodies,
-                        c->h_rctl->tail_iters);
+                        c->h_rctl->tail_iters, c->h_rctl->nf_sweeps);
             if (c->mp) {
                 // the global convergence flag: every unit decided it redundantly from the same counts;
                 // the ranks leave the loop together (matching barrier sequences) once all agree
