@@ -14,6 +14,7 @@
 //                  activation = atomicOr on the owner's bitmap + warp-aggregated append.
 //   k_pr_finalize a11  x' = (1-d)/V + d(acc + D/V), dangling mass and residual (PR, fp64).
 #include <cuda_runtime.h>
+#include <cstdio>
 #include <stdint.h>
 #include <stdlib.h>
 
@@ -238,27 +239,48 @@ struct NfAcc {
     unsigned long long parked = 0, unparked = 0;
     unsigned min_dist = 0xFFFFFFFFu;
 };
+// Acceptance of a thread's 8 candidates (bit q of cand: vertex vs[q] has out-degree > 0) under the
+// near-far split, batched so that the 8 state loads and then the 8 far-bit atomics are each in flight
+// together (one dependent round trip per step instead of one per vertex). Returns the accepted mask.
 template <int MODE>
-__device__ __forceinline__ bool filter_accept(const FragPtrs& F, unsigned v, bool nf, unsigned nfT, NfAcc& acc) {
-    if (!nf) return true;
-    if (MODE == FT_CLASSIFY) {
-        const unsigned dist = F.state[v];
-        if (dist < nfT) return true;
-        const unsigned bit = 1u << (v & 31);
-        const unsigned ob = atomicOr(F.far + (v >> 5), bit);
-        if (!(ob & bit)) acc.parked++;
-        acc.min_dist = dist < acc.min_dist ? dist : acc.min_dist;
-        return false;
+__device__ __forceinline__ unsigned filter_accept8(const FragPtrs& F, const unsigned* vs, unsigned cand, bool nf,
+                                                   unsigned nfT, NfAcc& acc) {
+    if (!nf || !cand) return cand;
+    unsigned st[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) st[q] = ((cand >> q) & 1u) ? F.state[vs[q]] : 0u;
+    unsigned ok = 0, park = 0;
+#pragma unroll
+    for (int q = 0; q < 8; q++) {
+        if (!((cand >> q) & 1u)) continue;
+        if (st[q] < nfT) ok |= 1u << q;
+        else park |= 1u << q;
     }
-    if (F.state[v] >= nfT) return false;  // parked in pass 1
-    if (MODE == FT_EMIT) {
-        const unsigned bit = 1u << (v & 31);
-        if (F.far[v >> 5] & bit) {
-            const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
-            if (ob & bit) acc.unparked++;
+    if (MODE == FT_CLASSIFY && park) {
+        unsigned ob[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+            ob[q] = ((park >> q) & 1u) ? atomicOr(F.far + (vs[q] >> 5), 1u << (vs[q] & 31)) : 0xFFFFFFFFu;
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            if (!((park >> q) & 1u)) continue;
+            if (!(ob[q] & (1u << (vs[q] & 31)))) acc.parked++;
+            acc.min_dist = st[q] < acc.min_dist ? st[q] : acc.min_dist;
         }
     }
-    return true;
+    if (MODE == FT_EMIT && ok) {
+        // accepted vertices leave the far set (their bit may be left from an earlier parking)
+        unsigned fw[8], ob[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++) fw[q] = ((ok >> q) & 1u) ? F.far[vs[q] >> 5] : 0u;
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+            ob[q] = (((ok >> q) & 1u) && (fw[q] & (1u << (vs[q] & 31)))) ? atomicAnd(F.far + (vs[q] >> 5), ~(1u << (vs[q] & 31))) : 0u;
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+            if (ob[q] & (1u << (vs[q] & 31))) acc.unparked++;
+    }
+    return ok;
 }
 
 // warp-reduce the near-far counters and apply them to the fragment (lane 0 of each warp)
@@ -273,7 +295,7 @@ __device__ __forceinline__ void nf_flush(FragCtl* ct, unsigned fslot, const NfAc
 
 template <int MODE>
 __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsigned tile, bool dense, bool sweep,
-                                            bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt,
+                                            bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt, unsigned ipt,
                                             unsigned chunk, unsigned long long pos, unsigned long long off) {
     const unsigned lane = lane_id();
     Pair mine{0, 0};
@@ -306,26 +328,33 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsig
 #pragma unroll
                 for (int q = 0; q <= kDenseVertsPerThread; q++) rpv[q] = (vb + q <= F.V) ? __ldg(rp + q) : 0ull;
             }
+            static_assert(kDenseVertsPerThread == 8, "filter_accept8 takes 8 candidates");
+            unsigned vs[8], cand = 0;
 #pragma unroll
             for (int q = 0; q < kDenseVertsPerThread; q++) {
-                if ((bits >> q) & 1u) {
+                vs[q] = vb + q;
+                if (((bits >> q) & 1u) && rpv[q + 1] != rpv[q]) cand |= 1u << q;
+            }
+            const unsigned ok = filter_accept8<MODE>(F, vs, cand, nf, nfT, acc);
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread; q++) {
+                if ((ok >> q) & 1u) {
                     const unsigned long long d = rpv[q + 1] - rpv[q];
-                    if (d && filter_accept<MODE>(F, vb + q, nf, nfT, acc)) {
-                        if (MODE == FT_EMIT) emit_vertex(F, chunk, vb + q, rpv[q], d, pos + mine.cnt, off + mine.deg);
-                        mine.cnt += 1;
-                        mine.deg += d;
-                    }
+                    if (MODE == FT_EMIT) emit_vertex(F, chunk, vb + q, rpv[q], d, pos + mine.cnt, off + mine.deg);
+                    mine.cnt += 1;
+                    mine.deg += d;
                 }
             }
         }
     } else {
-        const unsigned long long ibase = (unsigned long long)tile * kFilterAppPerPart + threadIdx.x * kFilterAppPerThread;
+        // ipt (1..8) items per thread: short lists use small tiles so they spread over every SM
+        const unsigned long long ibase = (unsigned long long)tile * (kThreads * ipt) + threadIdx.x * ipt;
         unsigned items[kFilterAppPerThread];
         unsigned long long rp0[kFilterAppPerThread], d[kFilterAppPerThread];
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
             items[j] = 0xFFFFFFFFu;
-            if (ibase + j < app_cnt) items[j] = F.app[ibase + j];
+            if ((unsigned)j < ipt && ibase + j < app_cnt) items[j] = F.app[ibase + j];
         }
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
@@ -339,9 +368,15 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsig
                 d[j] = __ldg(F.row_ptr + v + 1) - rp0[j];
             }
         }
+        static_assert(kFilterAppPerThread == 8, "filter_accept8 takes 8 candidates");
+        unsigned cand = 0;
+#pragma unroll
+        for (int j = 0; j < kFilterAppPerThread; j++)
+            if (d[j]) cand |= 1u << j;
+        const unsigned ok = filter_accept8<MODE>(F, items, cand, nf, nfT, acc);
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
-            if (d[j] && filter_accept<MODE>(F, items[j], nf, nfT, acc)) {
+            if ((ok >> j) & 1u) {
                 if (MODE == FT_EMIT) emit_vertex(F, chunk, items[j], rp0[j], d[j], pos + mine.cnt, off + mine.deg);
                 mine.cnt += 1;
                 mine.deg += d[j];
@@ -357,7 +392,15 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsig
 // edge-balanced chunk table. Reduce-then-scan over a static split of the tiles: CTA b (ticket order)
 // counts its contiguous tile range, publishes the aggregate, sums its predecessors' aggregates (one
 // parallel read, no serial look-back chain) and re-walks its range emitting entries in vertex order.
+#ifdef GUM_FILTER_TIMING
+__device__ unsigned long long g_ftime[1024][8];
+__device__ unsigned g_fcall;
+#define FT_MARK(i) do { if (threadIdx.x == 0 && g_fcall == GUM_FILTER_TIMING) g_ftime[blockIdx.x][i] = globaltimer(); } while (0)
+#else
+#define FT_MARK(i) do {} while (0)
+#endif
 __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+    FT_MARK(0);
     // Prologue by thread 0 only, broadcast through shared memory: the run-control fields are a handful of
     // L2 lines that every CTA of every kernel reads, and per-warp loads of one address serialise in its
     // L2 slice (with ~600 CTAs x 8 warps that alone cost tens of microseconds per launch).
@@ -391,6 +434,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
         s_pro = p;
     }
     __syncthreads();
+    FT_MARK(1);
     if (!s_pro.go) return;
     const bool sweep = s_pro.sweep != 0;
     const unsigned nfT = s_pro.nfT;
@@ -399,7 +443,13 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     const unsigned app_cnt = s_pro.app_cnt;
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
-    const unsigned per = dense ? kDenseWordsPerPart : kFilterAppPerPart;
+    // sparse lists: items per thread so that the tiles cover the grid (1..8)
+    unsigned ipt = kFilterAppPerThread;
+    if (!dense) {
+        const unsigned long long per_cta = (n_items + gridDim.x - 1) / gridDim.x;
+        ipt = per_cta <= kThreads ? 1u : per_cta <= 2u * kThreads ? 2u : per_cta <= 4u * kThreads ? 4u : 8u;
+    }
+    const unsigned per = dense ? kDenseWordsPerPart : kThreads * ipt;
     const unsigned n_tiles = (unsigned)((n_items + per - 1) / per);
     const unsigned long long epoch = s_pro.epoch;
     const unsigned chunk = c.chunk;
@@ -415,12 +465,13 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     Pair mine{0, 0};
     NfAcc nfa;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
         mine.cnt += q.cnt;
         mine.deg += q.deg;
     }
+    FT_MARK(2);
     Pair agg;
-    block_excl_scan(mine, s_warp, agg);
+    const Pair tex1 = block_excl_scan(mine, s_warp, agg);  // per-thread offsets when the CTA has one tile
     if (threadIdx.x == 0) {
         slots[b].agg_cnt = agg.cnt;
         slots[b].agg_deg = agg.deg;
@@ -435,6 +486,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
         pre.cnt += __ldcg(&slots[j].agg_cnt);
         pre.deg += __ldcg(&slots[j].agg_deg);
     }
+    FT_MARK(3);
     Pair excl;
     block_excl_scan(pre, s_warp, excl);  // excl = sum over all predecessors
     if (b == G - 1 && threadIdx.x == 0) {
@@ -452,16 +504,26 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     }
     // ---- pass 2: per tile, re-count (L1/L2-resident re-read) for the per-thread offsets, then emit
     unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
-    for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_COUNT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, 0, 0);
-        Pair tot;
-        const Pair tex = block_excl_scan(q, s_warp, tot);
-        filter_tile<FT_EMIT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, chunk, run_cnt + tex.cnt,
-                             run_deg + tex.deg);
-        run_cnt += tot.cnt;
-        run_deg += tot.deg;
+    if (t_hi - t_lo == 1) {
+        // one tile: pass 1's per-thread counts are this tile's (same acceptance), no re-count
+        filter_tile<FT_EMIT>(F, nfa, t_lo, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
+                             run_deg + tex1.deg);
+    } else {
+        for (unsigned t = t_lo; t < t_hi; t++) {
+            const Pair q = filter_tile<FT_COUNT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+            Pair tot;
+            const Pair tex = block_excl_scan(q, s_warp, tot);
+            filter_tile<FT_EMIT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
+                                 run_deg + tex.deg);
+            run_cnt += tot.cnt;
+            run_deg += tot.deg;
+        }
     }
     if (nf) nf_flush(ct, fslot, nfa);
+    FT_MARK(4);
+#ifdef GUM_FILTER_TIMING
+    if (threadIdx.x == 0 && g_fcall == GUM_FILTER_TIMING) { g_ftime[blockIdx.x][5] = b; g_ftime[blockIdx.x][6] = G; g_ftime[blockIdx.x][7] = app_cnt; }
+#endif
 }
 
 // ------------------------------------------------------------------------------------------ control
@@ -469,6 +531,9 @@ template <int ALG>
 __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cudaGraphConditionalHandle h, int use_h) {
     if (threadIdx.x != 0) return;
     RunCtl* rc = c.rctl[w0];
+#ifdef GUM_FILTER_TIMING
+    g_fcall++;
+#endif
     if (rc->done) {
         if (use_h) cudaGraphSetConditional(h, 0);
         return;
@@ -1560,6 +1625,22 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         }
     }
 }
+
+#ifdef GUM_FILTER_TIMING
+void dump_filter_timing() {
+    static unsigned long long h[1024][8];
+    cudaDeviceSynchronize();
+    cudaMemcpyFromSymbol(h, g_ftime, sizeof(h));
+    unsigned long long t0 = ~0ull;
+    for (int i = 0; i < 1024; i++) if (h[i][0] && h[i][0] < t0) t0 = h[i][0];
+    for (int i = 0; i < 1024; i++) {
+        if (!h[i][0]) continue;
+        fprintf(stderr, "cta %4d b=%4llu G=%llu app=%llu start=%7.2f pro=%7.2f p1=%7.2f pre=%7.2f end=%7.2f\n", i, h[i][5], h[i][6], h[i][7],
+                (h[i][0] - t0) / 1e3, (h[i][1] - t0) / 1e3, h[i][2] ? (h[i][2] - t0) / 1e3 : -1.0, h[i][3] ? (h[i][3] - t0) / 1e3 : -1.0,
+                h[i][4] ? (h[i][4] - t0) / 1e3 : -1.0);
+    }
+}
+#endif
 
 cudaError_t filter_occupancy(int* blocks_per_sm) {
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_filter, kThreads, 0);

@@ -21,6 +21,9 @@
 #include "planner.h"
 
 using namespace gum;
+#ifdef GUM_FILTER_TIMING
+namespace gum { void dump_filter_timing(); }
+#endif
 
 namespace {
 
@@ -1487,6 +1490,9 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             }
         }
     }
+#ifdef GUM_FILTER_TIMING
+    dump_filter_timing();
+#endif
     c->last_alg = alg;
     c->last_iters = R.iter;
     if (R.err) return fail(c, GUM_ERANGE, "SSSP distance reached 2^32-1");
