@@ -83,7 +83,13 @@ typedef struct {
      * vertices is below osteal_active_threshold the active owners are the survivors {0..m'-1}
      * (uniform NVSwitch reduction tree, reading #13), m' = clamp(ceil(active_edges /
      * osteal_edges_per_worker), 1, num_gpus) (0 => m' = 1); above it ownership is given back.
-     * Fragment f is owned by worker f if f < m', else by f mod m'. */
+     * Fragment f is owned by worker f if f < m', else by f mod m'.
+     * osteal = 0: off; 1: this active-vertex threshold trigger (the north_star's rule, the default);
+     * 2: the paper's cost model (NEXT-3, Alg. 2 P:201-211 with Eq. (4)): every iteration,
+     * for m = 1..num_gpus, E(m) = z(m) + p*m with z(m) the Eq. (1) makespan when only workers {0..m-1}
+     * process (evicted fragments' edges at the remote cost, see gum_osteal_plan) and p =
+     * osteal_sync_edges; the first m with the lowest E(m) becomes the active owner set (shrinking or
+     * giving ownership back). */
     int osteal;
     uint64_t osteal_active_threshold;
     uint64_t osteal_edges_per_worker;
@@ -116,6 +122,10 @@ typedef struct {
      * large-frontier iterations bottom-up (every unvisited vertex looks for a parent at the current
      * depth among its in-edges). Same depths; 0 = push only (the paper's GUM, the default). */
     int bfs_direction_opt;
+    /* OSteal cost model (osteal = 2): p of Eq. (4), the per-worker synchronisation cost of one
+     * iteration expressed in edge-processing time units (edges); 0 => 500000 (B200: ~3.5 us of
+     * per-unit launch + barrier cost at ~7 ps per expanded edge). */
+    double osteal_sync_edges;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);
@@ -265,6 +275,11 @@ gum_status gum_mp_handshake(const gum_config* cfg, const gum_mp_config* mp);
  * time -- take the max over ranks), gum_result (every rank gathers the full result through the peer
  * mappings), gum_destroy. GUM_CFG_PROFILE is not supported (EUNSUP). */
 gum_status gum_create_mp(const gum_config* cfg, const gum_mp_config* mp, gum_ctx** out);
+
+/* Host helper of the OSteal cost model (NEXT-3): Alg. 2 over m = 1..n for per-fragment loads l[0..n)
+ * (active edges), remote cost b (local 1) and sync cost p (edges). cost[m-1] = E(m) = z(m) + p*m
+ * (nullable); *m_out = the chosen cluster size. The device control kernel runs the same routine. */
+gum_status gum_osteal_plan(const uint64_t* loads, int n, double remote_cost, double p, double* cost, int* m_out);
 
 /* Library version (major*10000 + minor*100 + patch). */
 int gum_version(void);

@@ -35,7 +35,7 @@ LOAD_DEVICE = 0x1
 ABI_SYMBOLS = ("gum_config_default", "gum_create", "gum_destroy", "gum_last_error", "gum_build_csr",
                "gum_load_csr", "gum_partition", "gum_partition_bounds", "gum_prepare", "gum_run", "gum_result",
                "gum_result_device", "gum_trace", "gum_profile", "gum_fsteal_plan", "gum_version",
-               "gum_mp_handshake", "gum_create_mp")
+               "gum_mp_handshake", "gum_create_mp", "gum_osteal_plan")
 
 
 class GumError(RuntimeError):
@@ -57,6 +57,7 @@ class gum_config(ctypes.Structure):
                 ("max_iterations", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("sssp_delta", ctypes.c_uint32),
                 ("tail_vertices", ctypes.c_uint32), ("pb_block_log2", ctypes.c_uint32),
                 ("fsteal_remote_cost", ctypes.c_double), ("bfs_direction_opt", ctypes.c_int),
+                ("osteal_sync_edges", ctypes.c_double),
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
 
@@ -124,6 +125,7 @@ def load_library():
         "gum_fsteal_plan": (i32, [vp, i32, ctypes.c_double, vp, ctypes.POINTER(ctypes.c_double)]),
         "gum_version": (i32, []),
         "gum_mp_handshake": (i32, [ctypes.POINTER(gum_config), ctypes.POINTER(gum_mp_config)]),
+        "gum_osteal_plan": (i32, [vp, i32, ctypes.c_double, ctypes.c_double, vp, ctypes.POINTER(i32)]),
         "gum_create_mp": (i32, [ctypes.POINTER(gum_config), ctypes.POINTER(gum_mp_config), ctypes.POINTER(vp)]),
     }
     for name, (res, args) in sig.items():
@@ -188,7 +190,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
                 osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
-                use_torch_allocator=False, streams=None):
+                use_torch_allocator=False, streams=None, osteal_sync_edges=0.0):
     """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
     config points to and must live as long as the context."""
     lib = load_library()
@@ -203,7 +205,8 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
     cfg.fsteal = 2 if fsteal == "planned" else int(bool(fsteal))
     cfg.fsteal_remote_cost = float(fsteal_remote_cost)
     cfg.bfs_direction_opt = int(bool(bfs_direction_opt))
-    cfg.osteal = int(bool(osteal))
+    cfg.osteal = 2 if osteal == "cost" else int(bool(osteal))
+    cfg.osteal_sync_edges = float(osteal_sync_edges)
     cfg.t1_min_max_edges = int(t1)
     cfg.t2_min_spread_edges = int(t2)
     cfg.osteal_active_threshold = int(osteal_threshold)
@@ -376,6 +379,18 @@ def mp_handshake(rank, world, exchange, **kw):
     fn = exchange if isinstance(exchange, EXCHANGE_FN) else EXCHANGE_FN(exchange)
     mpc = gum_mp_config(int(rank), int(world), 0, fn, None)
     return int(load_library().gum_mp_handshake(ctypes.byref(cfg), ctypes.byref(mpc)))
+
+
+def osteal_plan(loads, remote_cost=1.0, p=0.0):
+    """NEXT-3 planner (host helper of the device routine): returns (m, [E(1..n)]) of Alg. 2 / Eq. (4)."""
+    n = len(loads)
+    l = np.ascontiguousarray(loads, dtype=np.uint64)
+    cost = np.zeros(n, dtype=np.float64)
+    m = ctypes.c_int()
+    st = load_library().gum_osteal_plan(_ptr(l), n, float(remote_cost), float(p), _ptr(cost), ctypes.byref(m))
+    if st != GUM_OK:
+        raise GumError(st, "gum_osteal_plan: bad arguments")
+    return m.value, cost
 
 
 def fsteal_plan(loads, remote_cost=1.0):

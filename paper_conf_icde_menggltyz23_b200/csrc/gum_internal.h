@@ -163,6 +163,7 @@ struct DevCtx {
     unsigned int num_vertices;  // |V|
     int fsteal, osteal;         // fsteal: 0 off, 1 steal queue, 2 planned (Eq. 1 / Alg. 1)
     double remote_cost;         // planned FSteal: cost of a remote edge relative to a local one
+    double os_p;                // OSteal cost model (osteal = 2): p of Eq. (4) in edges
     unsigned long long t1, t2, os_thresh, os_epw;
     unsigned int max_iter;
     int pr_iters;

@@ -607,7 +607,12 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         // ownership is given back. Fragment f is owned by f when f < m', else by f mod m'.
         if (c.osteal && c.P > 1) {
             unsigned mp = (unsigned)c.P;
-            if (active < c.os_thresh) {
+            if (c.osteal == 2) {
+                // NEXT-3: Alg. 2 with Eq. (4) on this iteration's per-fragment active edges
+                unsigned long long lf[kMaxW];
+                for (int f = 0; f < c.P; f++) lf[f] = vload(&c.f[f].ctl->qedges);
+                mp = (unsigned)osteal_choose(lf, c.P, c.remote_cost, c.os_p, nullptr);
+            } else if (active < c.os_thresh) {
                 mp = 1;
                 if (c.os_epw) {
                     const unsigned long long want = (total_edges + c.os_epw - 1) / c.os_epw;

@@ -57,4 +57,51 @@ GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double
     return z;
 }
 
+// OSteal cost model (§IV-A/B, Eq. (4), Alg. 2).
+// For a cluster size m the reduction tree on a uniform fabric keeps workers R(m) = {0..m-1} (DESIGN.md
+// reading #13); the revised Eq. (1) lets only R(m) process (x_ij = 0 for j outside R(m)): an evicted
+// fragment's edges are all processed remotely at cost b, a survivor keeps its own at cost 1 and trades
+// with the other survivors as in fsteal_waterfill. The LP relaxation again has a closed form: z solves
+//     sum_{j<m} max(l_j - z, 0) + sum_{i>=m} l_i = sum_{j<m} max(z - l_j, 0) / b.
+GUM_HD inline double osteal_makespan(const unsigned long long* l, int n, int m, double b) {
+    if (n <= 0 || m <= 0) return 0.0;
+    if (m > n) m = n;
+    if (b < 1.0) b = 1.0;
+    double evicted = 0.0, hi = 0.0;
+    for (int i = 0; i < n; i++) {
+        if (i >= m) evicted += (double)l[i];
+        hi = (double)l[i] > hi ? (double)l[i] : hi;
+    }
+    hi += evicted * b;  // z <= max own load + all evicted work on one survivor
+    double lo = 0.0;
+    for (int it = 0; it < 200; it++) {
+        const double z = 0.5 * (lo + hi);
+        double give = evicted, take = 0.0;
+        for (int j = 0; j < m; j++) {
+            const double lj = (double)l[j];
+            if (lj > z) give += lj - z;
+            else take += (z - lj) / b;
+        }
+        if (give > take) lo = z;
+        else hi = z;
+    }
+    return hi;
+}
+
+// Alg. 2: enumerate m = 1..n, E(m) = z(m) + p*m (Eq. 4), keep the first strict minimum. cost[m-1] =
+// E(m) when cost is non-null. Returns the chosen m.
+GUM_HD inline int osteal_choose(const unsigned long long* l, int n, double b, double p, double* cost) {
+    int best_m = n;
+    double best = 0.0;
+    for (int m = 1; m <= n; m++) {
+        const double e = osteal_makespan(l, n, m, b) + p * (double)m;
+        if (cost) cost[m - 1] = e;
+        if (m == 1 || e < best) {
+            best = e;
+            best_m = m;
+        }
+    }
+    return best_m;
+}
+
 }  // namespace gum

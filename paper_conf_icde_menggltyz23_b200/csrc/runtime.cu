@@ -361,6 +361,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.fsteal = c->cfg.fsteal;
     d.remote_cost = c->cfg.fsteal_remote_cost > 0.0 ? c->cfg.fsteal_remote_cost : 1.0;
     d.osteal = c->cfg.osteal;
+    d.os_p = c->cfg.osteal_sync_edges > 0.0 ? c->cfg.osteal_sync_edges : 500000.0;
     d.t1 = c->cfg.t1_min_max_edges;
     d.t2 = c->cfg.t2_min_spread_edges;
     d.os_thresh = c->cfg.osteal_active_threshold;
@@ -962,7 +963,7 @@ static unsigned long long config_hash(const gum_config* cfg) {
     GUM_HC(num_gpus); GUM_HC(fsteal); GUM_HC(t1_min_max_edges); GUM_HC(t2_min_spread_edges); GUM_HC(osteal);
     GUM_HC(osteal_active_threshold); GUM_HC(osteal_edges_per_worker); GUM_HC(chunk_edges); GUM_HC(pr_iterations);
     GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
-    GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt);
+    GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt); GUM_HC(osteal_sync_edges);
 #undef GUM_HC
     return h;
 }
@@ -1582,6 +1583,14 @@ gum_status gum_fsteal_plan(const uint64_t* loads, int n, double remote_cost, dou
     for (int i = 0; i < n; i++) l[i] = loads[i];
     const double zz = fsteal_waterfill(l, n, remote_cost > 0.0 ? remote_cost : 1.0, X);
     if (z) *z = zz;
+    return GUM_OK;
+}
+
+gum_status gum_osteal_plan(const uint64_t* loads, int n, double remote_cost, double p, double* cost, int* m_out) {
+    if (!loads || !m_out || n < 1 || n > kMaxW || p < 0.0) return GUM_EINVAL;
+    unsigned long long l[kMaxW];
+    for (int i = 0; i < n; i++) l[i] = loads[i];
+    *m_out = osteal_choose(l, n, remote_cost > 0.0 ? remote_cost : 1.0, p, cost);
     return GUM_OK;
 }
 

@@ -299,3 +299,18 @@ def test_wcc_blocked_first_iteration(monkeypatch, P):
     csr = csr_of(g)
     for kw in (dict(), dict(part="random", seed=2), dict(tail_vertices=0), dict(split_units=P > 1)):
         check(g, "wcc", 0, csr=csr, ref=ref, num_gpus=P, **kw)
+
+
+@pytest.mark.parametrize("alg", ALGS)
+@pytest.mark.parametrize("p", [0.0, 2e4, 1e12])
+def test_osteal_cost_model(alg, p):
+    """NEXT-3: OSteal by Alg. 2 / Eq. (4) (osteal='cost'): outputs unchanged for any p; p -> inf keeps one
+    owner, p = 0 keeps all of them (z(m) is non-increasing in m)."""
+    g = inputs.rmat(13, 16, seed=33)
+    s = inputs.pick_source(g, 33)
+    _, st, _ = check(g, alg, s, num_gpus=4, part="random", seed=3, osteal="cost", osteal_sync_edges=p,
+                     tail_vertices=0)
+    if p == 1e12:
+        assert st.final_owners == 1
+    if p == 0.0 and alg == "pr":
+        assert st.final_owners == 4

@@ -80,3 +80,66 @@ def test_carve_whole_adjacency_lists():
     assert planner.carve([4, 4, 4, 4], [6, 10]) == [(0, 1), (1, 4)]
     assert planner.carve([4, 4, 4, 4], [8, 8]) == [(0, 2), (2, 4)]
     assert planner.carve([4, 4, 4, 4], [16, 0]) == [(0, 4), None]
+
+
+# ------------------------------------------------------------------------------- NEXT-3 OSteal model
+GOLDEN3 = os.path.join(os.path.dirname(__file__), "golden", "example3_osteal.json")
+
+
+def test_example3_golden_oracle():
+    g = json.load(open(GOLDEN3))
+    C = uniform_costs(2, g["remote_cost"])
+    for m, zexp in enumerate(g["expected_z_by_m"], start=1):
+        assert planner.osteal_milp_bruteforce(g["loads"], C, m)[0] == zexp
+        assert abs(planner.osteal_lp(g["loads"], C, m)[0] - zexp) < 1e-9
+    th = g["p_threshold"]
+    assert planner.osteal_alg2(g["loads"], C, th - 0.5)[0] == 2
+    assert planner.osteal_alg2(g["loads"], C, th)[0] == 1  # tie: the first (smaller) m is kept
+    assert planner.osteal_alg2(g["loads"], C, th + 0.5)[0] == 1
+
+
+def test_example3_golden_product():
+    g = json.load(open(GOLDEN3))
+    th = g["p_threshold"]
+    for p, mexp in ((0.0, 2), (th - 0.5, 2), (th + 0.5, 1), (1e9, 1)):
+        m, cost = gum.osteal_plan(g["loads"], g["remote_cost"], p)
+        assert m == mexp, (p, m, cost)
+        assert np.allclose(cost, [z + p * (k + 1) for k, z in enumerate(g["expected_z_by_m"])], rtol=1e-9)
+
+
+@settings(max_examples=40, deadline=None)
+@given(st.lists(st.integers(0, 3), min_size=2, max_size=3), st.sampled_from([1.0, 2.0]))
+def test_osteal_lp_lower_bounds_milp(loads, b):
+    C = uniform_costs(len(loads), b)
+    for m in range(1, len(loads) + 1):
+        z_milp = planner.osteal_milp_bruteforce(loads, C, m)[0]
+        z_lp = planner.osteal_lp(loads, C, m)[0]
+        assert z_lp <= z_milp + 1e-9
+        assert z_milp <= z_lp + b * len(loads) + 1e-9  # integrality gap bounded by one edge per row
+
+
+@settings(max_examples=60, deadline=None)
+@given(st.lists(st.integers(0, 10**7), min_size=1, max_size=8), st.sampled_from([1.0, 1.3, 2.0, 5.0]),
+       st.sampled_from([0.0, 1.0, 1e4, 1e6, 1e9]))
+def test_product_osteal_matches_oracle_alg2(loads, b, p):
+    n = len(loads)
+    C = uniform_costs(n, b)
+    m_ora, cost_ora = planner.osteal_alg2(loads, C, p)
+    m, cost = gum.osteal_plan(loads, b, p)
+    scale = max(1.0, max(cost_ora))
+    assert np.allclose(cost, cost_ora, atol=1e-6 * scale, rtol=1e-7)
+    # the same choice unless two cluster sizes tie within rounding
+    if m != m_ora:
+        assert abs(cost[m - 1] - cost[m_ora - 1]) <= 1e-6 * scale
+
+
+def test_osteal_special_cases():
+    # m = n is the FSteal plan; m = 1 puts every other fragment's work on worker 0 at the remote cost;
+    # more survivors never increase the makespan
+    loads = [700, 50, 3000, 0, 12]
+    for b in (1.0, 2.5):
+        z_f, _ = gum.fsteal_plan(loads, b)
+        m, cost = gum.osteal_plan(loads, b, 0.0)
+        assert abs(cost[-1] - z_f) < 1e-6 * z_f
+        assert abs(cost[0] - (loads[0] + b * sum(loads[1:]))) < 1e-6 * cost[0]
+        assert all(cost[i + 1] <= cost[i] + 1e-6 for i in range(len(loads) - 1))
