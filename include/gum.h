@@ -46,8 +46,11 @@ typedef enum {
 typedef enum { GUM_BFS = 0, GUM_SSSP = 1, GUM_WCC = 2, GUM_PR = 3 } gum_alg;
 
 /* Partitioners (P:315, P:382 Exp-6): SEG = contiguous id ranges with ~equal out-edges; RANDOM =
- * keyed Feistel relabel of ids, then SEG (reading #17). metis is out of scope. */
-typedef enum { GUM_PART_SEG = 0, GUM_PART_RANDOM = 1 } gum_part;
+ * keyed Feistel relabel of ids, then SEG (reading #17). metis is out of scope.
+ * DEGREE (a B200 layout option, not in the paper): relabel ids by decreasing in-degree (ties by id), then
+ * SEG -- the few destinations most edges point to share a few KB of every per-vertex array, so their
+ * visited-bit / state probes hit L1/L2 instead of missing. Results are in original ids. */
+typedef enum { GUM_PART_SEG = 0, GUM_PART_RANDOM = 1, GUM_PART_DEGREE = 2 } gum_part;
 
 #define GUM_INF 0xFFFFFFFFu
 #define GUM_MAX_WORKERS 8
@@ -131,6 +134,27 @@ typedef struct {
     void (*free_fn)(void* ptr, uint64_t bytes, int device, void* user);
     void* alloc_user;
     void* const* streams; /* cudaStream_t per worker (NULL => library-owned non-blocking streams) */
+    /* NEXT-1 communication reducers (§V-B "Optimizations"; only change anything when num_gpus > 1).
+     * mirrors = 1: outer-vertex mirrors with early message aggregation ("the destination of
+     * cross-fragment edges are also kept as outer vertices for message-aggregation optimization").
+     * Every worker w keeps, in its own memory, a mirror of every vertex it does not own:
+     *   PR:        a double[V] accumulator -- pushes to other fragments' vertices add into w's mirror
+     *              (local red.add) instead of the owner's acc; the owner's finalize pulls and clears its
+     *              slice of every peer mirror (one bulk read per iteration instead of one remote atomic
+     *              per edge: an aggregated reduce-scatter over peer memory);
+     *   BFS:       a bit[V] "already sent" filter -- a cross-fragment update is issued only the first time
+     *              w discovers v (a set bit also caches "v is visited" seen in the owner's bitmap);
+     *   SSSP/WCC:  a uint32[V] "minimum sent" value -- a cross-fragment update is issued only when the
+     *              candidate beats every value w has sent to v before (the owner's value is <= it).
+     * Results are unchanged (monotone min-fixpoints; PR sums the same terms in another order).
+     * hub_cache = 1: hub adjacency caching (P:274 Example 6). At gum_prepare every worker copies the
+     * adjacency lists (col, and weights for SSSP) of every other fragment's vertices with out-degree >
+     * hub_degree (t4; 0 caches every list) into its own memory; a stolen (or OSteal-inherited) frontier
+     * vertex whose list is cached is expanded from the local copy instead of the owner's CSR over
+     * NVLink. BFS/SSSP/WCC (PR's static queue is destination-blocked; PR uses mirrors instead). */
+    int mirrors;
+    int hub_cache;
+    uint32_t hub_degree;
 } gum_config;
 
 /* Fills *cfg with the defaults: 1 worker, fsteal=1, osteal=1, t1=t2=0, osteal threshold 0 (off until
@@ -157,6 +181,10 @@ typedef struct {
     uint64_t kernel_launches; /* this process's kernel launches in the run: exact in host-loop and
                                  multi-process mode (incl. barrier kernels); CUDA-graph mode counts every
                                  body kernel once per executed WHILE iteration (iterations + 1) */
+    uint64_t remote_filtered; /* NEXT-1 mirrors: cross-fragment updates absorbed by the local mirror
+                                 (BFS/SSSP/WCC: not sent; PR: aggregated, then flushed in bulk) */
+    uint64_t hub_cached_edges;/* NEXT-1 hub cache: edges of non-local fragments expanded from a local copy */
+    uint64_t mirror_flush_bytes; /* PR mirrors: bytes the finalize read from peer mirrors */
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

@@ -24,7 +24,7 @@ GUM_OK, GUM_EINVAL, GUM_ENOMEM, GUM_ESTATE, GUM_ERANGE, GUM_ECUDA, GUM_ENCCL, GU
 STATUS_NAMES = {0: "GUM_OK", -1: "GUM_EINVAL", -2: "GUM_ENOMEM", -3: "GUM_ESTATE", -4: "GUM_ERANGE",
                 -5: "GUM_ECUDA", -6: "GUM_ENCCL", -7: "GUM_EUNSUP"}
 ALGS = {"bfs": 0, "sssp": 1, "wcc": 2, "pr": 3}
-PARTS = {"seg": 0, "random": 1}
+PARTS = {"seg": 0, "random": 1, "degree": 2}
 INF = 0xFFFFFFFF
 MAX_WORKERS = 8
 
@@ -59,7 +59,8 @@ class gum_config(ctypes.Structure):
                 ("fsteal_remote_cost", ctypes.c_double), ("bfs_direction_opt", ctypes.c_int),
                 ("osteal_sync_edges", ctypes.c_double),
                 ("alloc", ALLOC_FN),
-                ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p))]
+                ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p)),
+                ("mirrors", ctypes.c_int), ("hub_cache", ctypes.c_int), ("hub_degree", ctypes.c_uint32)]
 
 
 EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p)
@@ -77,7 +78,9 @@ class gum_run_stats(ctypes.Structure):
                 ("remote_updates", ctypes.c_uint64), ("activations", ctypes.c_uint64),
                 ("vertices_frontier", ctypes.c_uint64), ("final_owners", ctypes.c_uint32), ("osteal_iteration", ctypes.c_uint32),
                 ("tail_iterations", ctypes.c_uint32), ("bodies", ctypes.c_uint32),
-                ("pr_last_residual", ctypes.c_double), ("kernel_launches", ctypes.c_uint64)]
+                ("pr_last_residual", ctypes.c_double), ("kernel_launches", ctypes.c_uint64),
+                ("remote_filtered", ctypes.c_uint64), ("hub_cached_edges", ctypes.c_uint64),
+                ("mirror_flush_bytes", ctypes.c_uint64)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -184,13 +187,17 @@ class RunStats:
     bodies: int
     pr_last_residual: float
     kernel_launches: int
+    remote_filtered: int = 0
+    hub_cached_edges: int = 0
+    mirror_flush_bytes: int = 0
 
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                 osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
-                use_torch_allocator=False, streams=None, osteal_sync_edges=0.0):
+                use_torch_allocator=False, streams=None, osteal_sync_edges=0.0, mirrors=False, hub_cache=False,
+                hub_degree=0):
     """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
     config points to and must live as long as the context."""
     lib = load_library()
@@ -218,6 +225,9 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
     cfg.sssp_delta = int(sssp_delta)
     cfg.tail_vertices = int(tail_vertices)
     cfg.pb_block_log2 = int(pb_block_log2)
+    cfg.mirrors = int(bool(mirrors))          # NEXT-1 outer-vertex mirrors
+    cfg.hub_cache = int(bool(hub_cache))      # NEXT-1 hub adjacency caching
+    cfg.hub_degree = int(hub_degree)          # t4
     flags = 0
     if trace:
         flags |= CFG_TRACE

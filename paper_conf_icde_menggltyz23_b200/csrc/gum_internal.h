@@ -56,6 +56,8 @@ struct alignas(128) FragCtl {
     unsigned long long tedges[3];      // tail engine: out-edges of the listed vertices
     unsigned long long pclaim[kMaxW];  // FSteal planned mode: per-worker claim counters of this queue
     unsigned long long pull_checked;   // bottom-up BFS: in-edges inspected
+    unsigned long long remote_filtered;  // NEXT-1 mirrors: cross-fragment updates absorbed locally
+    unsigned long long hub_edges;        // NEXT-1 hub cache: non-local edges expanded from a local copy
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
@@ -141,6 +143,18 @@ struct FragPtrs {
     const unsigned long long* sq_q_off;
     const unsigned int* sq_tile;
     unsigned long long sq_len, sq_edges;
+    // NEXT-1 outer-vertex mirror of worker f (this fragment's memory), indexed by GLOBAL id; only
+    // vertices of other fragments are ever touched ("outer" vertices)
+    double* macc;                       // PR: [V] aggregated pushes to other fragments' vertices
+    unsigned int* msent;                // BFS: [ceil(V/32)] already-sent / known-visited bits
+    unsigned int* mmin;                 // SSSP/WCC: [V] upper bound of the owner's value (min sent/seen)
+};
+
+// NEXT-1 hub cache: worker w's local copy of fragment f's hub adjacency lists.
+struct HubPtrs {
+    const unsigned long long* off;  // [V_f] col index of local vertex u's list in the copy, ~0 = not cached
+    const unsigned int* col;        // cached destination ids
+    const unsigned int* w;          // cached weights (SSSP) or null
 };
 
 // Multi-process signal pads (a10): pad[u][s] = last barrier epoch unit s signalled to unit u;
@@ -177,6 +191,9 @@ struct DevCtx {
     unsigned int pb_nb;         // bins of fragment 0 (single-fragment only)
     unsigned int bfs_pull;      // direction-optimising BFS enabled (in-CSR built)
     unsigned long long total_edges;  // sum of the fragments' out-edges
+    int mirrors;                // NEXT-1 outer-vertex mirrors (P > 1 only)
+    int hub_on;                 // NEXT-1 hub cache built for this algorithm
+    HubPtrs hub[kMaxW][kMaxW];  // [worker][fragment] (fragment != worker)
 };
 
 }  // namespace gum

@@ -89,6 +89,16 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
             if (ALG == ALG_SSSP) F.far[i] = 0u;
         }
     }
+    // NEXT-1: worker f's outer-vertex mirror starts empty (global id space; own slice never touched)
+    if (c.mirrors) {
+        const unsigned NV = c.num_vertices;
+        const unsigned nm = ALG == ALG_BFS ? (NV + 31) / 32 : NV;
+        for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < nm; i += gridDim.x * blockDim.x) {
+            if (ALG == ALG_PR) F.macc[i] = 0.0;
+            if (ALG == ALG_BFS) F.msent[i] = 0u;
+            if (ALG == ALG_SSSP || ALG == ALG_WCC) F.mmin[i] = GUM_INF;
+        }
+    }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         FragCtl* ct = F.ctl;
         ct->claim = 0;
@@ -109,6 +119,8 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->far_cnt = 0;
         ct->far_min[0] = ct->far_min[1] = GUM_INF;
         ct->pull_checked = 0;
+        ct->remote_filtered = 0;
+        ct->hub_edges = 0;
         if (sq) {
             ct->frontier_edges = F.sq_edges;
             ct->frontier_vertices = F.sq_len;
@@ -794,6 +806,8 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     __shared__ unsigned short s_stbin[PBS];
     unsigned* const s_stage = s_head;  // s_head is dead once the chunk's col ids are loaded
     __shared__ unsigned s_wmax[kAdvThreads / 32];
+    // NEXT-1 hub cache: per staged vertex, 1 = its list is expanded from this worker's local copy
+    __shared__ unsigned char s_hub[MULTI ? kTileMax : 1];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
     __shared__ unsigned long long s_cnt[kMaxW][4];  // per fragment: edges, chunks, stolen edges, stolen chunks
@@ -838,7 +852,9 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kAdvThreads) s_head[e] = 0;
     unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
-    unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0;
+    unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0, filtered = 0, hub_e = 0;
+    // NEXT-1 outer-vertex mirrors (this worker's memory): updates to other fragments go through them
+    const bool mir = MULTI && c.mirrors;
 
     // Chunk claims run one chunk ahead of the expansion (thread 0): while chunk n is expanded, chunk n+1
     // is already claimed and its staging data (chunk table entries, degree prefix, col base, source
@@ -924,10 +940,12 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         unsigned long long t;
         int stolen;
         unsigned i0, nv, tlen;
+        bool hc;  // NEXT-1: non-local fragment whose hub lists this worker has cached
     };
     auto chunk_ref = [&](int f, unsigned long long t, int stolen) {
-        ChunkRef r{f, t, stolen, 0u, 0u, 0u};
+        ChunkRef r{f, t, stolen, 0u, 0u, 0u, false};
         if (f < 0) return r;
+        r.hc = MULTI && ALG != ALG_PR && c.hub_on && f != w;
         const FragPtrs& F = c.f[f];
         const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
         const unsigned* const tilep = sq ? F.sq_tile : F.tile;
@@ -939,7 +957,8 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         return r;
     };
     // per-vertex staging values of queue entry i of chunk r (vertex slot kk): edge prefix, col base, value
-    auto stage_load = [&](const ChunkRef& r, unsigned kk, unsigned long long& off, unsigned& base, unsigned& u) {
+    auto stage_load = [&](const ChunkRef& r, unsigned kk, unsigned long long& off, unsigned& base, unsigned& u,
+                          bool& hub) {
         const FragPtrs& F = c.f[r.f];
         const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
         const unsigned i = r.i0 + kk;
@@ -948,7 +967,17 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         // PR's (and WCC iteration 0's) blocked queue stores edges contiguously in queue order:
         // col index == q_off + j
         base = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(F.q_base + i)));
-        u = (ALG != ALG_BFS) ? __ldcs((sq ? F.sq_q_v : F.q_v) + i) : 0u;
+        u = (ALG != ALG_BFS || r.hc) ? __ldcs((sq ? F.sq_q_v : F.q_v) + i) : 0u;
+        hub = false;
+        if (MULTI && r.hc && !sq) {
+            // NEXT-1: a cached hub list is read from the local copy: col index of edge j of
+            // the vertex = h + j, i.e. base = tb + h - off (mod 2^32 like the fragment's base)
+            const unsigned long long h = __ldg(c.hub[w][r.f].off + u);
+            if (h != ~0ull) {
+                base = (unsigned)((long long)tb + (long long)h - (long long)off);
+                hub = true;
+            }
+        }
     };
     auto value_of = [&](const ChunkRef& r, unsigned u) -> VT {
         if (ALG == ALG_PR) return (VT)__ldcg(c.f[r.f].cx + u);
@@ -972,9 +1001,10 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     ChunkRef cur = chunk_ref(s_nf, s_nt, s_nstolen);
     unsigned long long p_off = 0;  // prefetched staging values of vertex slot threadIdx.x
     unsigned p_base = 0, p_u = 0;
+    bool p_hub = false;
     VT p_val = (VT)0;
     if (cur.f >= 0 && threadIdx.x < cur.nv) {
-        stage_load(cur, threadIdx.x, p_off, p_base, p_u);
+        stage_load(cur, threadIdx.x, p_off, p_base, p_u, p_hub);
         p_val = value_of(cur, p_u);
     }
     __syncthreads();  // everyone read s_nf before it is reused
@@ -1004,16 +1034,19 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         for (unsigned kk = threadIdx.x; kk < nv; kk += kAdvThreads) {
             unsigned long long off;
             unsigned base, u;
+            bool hub;
             VT val;
             if (kk < (unsigned)kAdvThreads) {
                 off = p_off;
                 base = p_base;
                 val = p_val;
+                hub = p_hub;
             } else {
-                stage_load(cur, kk, off, base, u);
+                stage_load(cur, kk, off, base, u, hub);
                 val = value_of(cur, u);
             }
             s_base[kk] = base;
+            if (MULTI) s_hub[kk] = hub ? 1 : 0;
             if (ALG != ALG_BFS) s_val[kk] = val;
             const long long rel = (long long)off - (long long)tb;
             if (rel > 0 && rel < (long long)tlen) s_head[rel] = (seq << 12) | kk;
@@ -1070,7 +1103,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
 
         // the next chunk's per-vertex staging values load while this chunk is expanded
         if (nxt.f >= 0 && threadIdx.x < nxt.nv) {
-            stage_load(nxt, threadIdx.x, p_off, p_base, p_u);
+            stage_load(nxt, threadIdx.x, p_off, p_base, p_u, p_hub);
             p_val = value_of(nxt, p_u);
         }
         // ---- expand: striped edges, coalesced streaming col/w loads
@@ -1084,11 +1117,13 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
             if (e < tlen) {
                 const unsigned kk = s_head[e];
                 const unsigned long long ci = (unsigned)(s_base[kk] + e);  // mod 2^32: the base may wrap
-                vv[j] = __ldcs(colp + ci);
+                const bool hv = MULTI && cur.hc && s_hub[kk];
+                if (MULTI) hub_e += hv ? 1 : 0;
+                vv[j] = __ldcs((hv ? c.hub[w][f].col : colp) + ci);
                 if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
                 if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];
                 if (ALG == ALG_SSSP) {
-                    const unsigned long long nd = (unsigned long long)s_val[kk] + __ldcs(F.w + ci);
+                    const unsigned long long nd = (unsigned long long)s_val[kk] + __ldcs((hv ? c.hub[w][f].w : F.w) + ci);
                     if (nd >= (unsigned long long)GUM_INF) {
                         atomicOr(&F.ctl->err, 1u);
                         vv[j] = GUM_INF;
@@ -1108,6 +1143,13 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                     if (MULTI) {
                         tf = frag_of(c, v);
                         lv = v - c.bounds[tf];
+                        if (mir && tf != w) {
+                            // NEXT-1: early aggregation into this worker's mirror of the outer vertex
+                            // (local red.add); the owner's finalize pulls the aggregate once
+                            atomicAdd(c.f[w].macc + v, (double)cv[j]);
+                            filtered++;
+                            continue;
+                        }
                         remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
                     }
                     atomicAdd(c.f[tf].acc + lv, (double)cv[j]);
@@ -1178,6 +1220,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
             // All candidates of iteration k equal k+1, so the depth store needs no atomic.
             unsigned lvv[kEdgesPerThread], wd[kEdgesPerThread];
             unsigned char tfv[kEdgesPerThread];
+            unsigned probed = 0;  // NEXT-1: outer vertices whose owner bitmap word was read
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++) {
                 tfv[j] = 0;
@@ -1188,14 +1231,28 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                         const int tf = frag_of(c, vv[j]);
                         tfv[j] = (unsigned char)tf;
                         lvv[j] = vv[j] - c.bounds[tf];
+                        // NEXT-1 "already sent" filter: an outer vertex this worker has sent to (or
+                        // seen visited) before needs no remote probe or update
+                        if (mir && tf != w && (c.f[w].msent[vv[j] >> 5] & (1u << (vv[j] & 31)))) {
+                            filtered++;
+                            continue;  // wd stays all-ones: no update
+                        }
                     }
                     wd[j] = c.f[tfv[j]].vis[lvv[j] >> 5];
+                    if (mir && tfv[j] != (unsigned char)w) probed |= 1u << j;
                 }
             }
             unsigned upd = 0;
 #pragma unroll
             for (int j = 0; j < kEdgesPerThread; j++)
                 if (!(wd[j] & (1u << (lvv[j] & 31)))) upd |= 1u << j;
+            if (mir) {
+                // every probed outer vertex is visited after this iteration (by us or before): cache it
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++)
+                    if (probed & (1u << j))
+                        atomicOr(c.f[w].msent + (vv[j] >> 5), 1u << (vv[j] & 31));  // local RED.OR
+            }
             if (next_dense) {
 #pragma unroll
                 for (int j = 0; j < kEdgesPerThread; j++) {
@@ -1243,6 +1300,14 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                         const int tf = frag_of(c, vv[j]);
                         tfv[j] = (unsigned char)tf;
                         lvv[j] = vv[j] - c.bounds[tf];
+                        // NEXT-1 mirror filter: the mirror holds an upper bound of the outer vertex's
+                        // value (min of everything this worker sent or read); a candidate that does not
+                        // beat it cannot improve the owner's value
+                        if (mir && tf != w && (unsigned)cv[j] >= c.f[w].mmin[vv[j]]) {
+                            filtered++;
+                            vv[j] = GUM_INF;
+                            continue;
+                        }
                     }
                     cur[j] = c.f[tfv[j]].state[lvv[j]];
                 }
@@ -1254,6 +1319,10 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                     upd |= 1u << j;
                     atomicMin(c.f[tfv[j]].state + lvv[j], (unsigned)cv[j]);  // RED.MIN (no return)
                     if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
+                }
+                if (mir && vv[j] != GUM_INF && tfv[j] != (unsigned char)w) {
+                    const unsigned nb = (unsigned)cv[j] < cur[j] ? (unsigned)cv[j] : cur[j];
+                    atomicMin(c.f[w].mmin + vv[j], nb);  // local RED.MIN: owner's value <= nb from now on
                 }
             }
             if (next_dense) {
@@ -1307,11 +1376,17 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     for (int o = 16; o > 0; o >>= 1) {
         remote += __shfl_xor_sync(0xffffffffu, remote, o);
         acts += __shfl_xor_sync(0xffffffffu, acts, o);
+        if (MULTI) {
+            filtered += __shfl_xor_sync(0xffffffffu, filtered, o);
+            hub_e += __shfl_xor_sync(0xffffffffu, hub_e, o);
+        }
     }
-    if (lane_id() == 0 && (remote | acts)) {
+    if (lane_id() == 0 && (remote | acts | filtered | hub_e)) {
         FragCtl* hc = c.f[w % c.P].ctl;
         if (remote) atomicAdd(&hc->remote_updates, remote);
         if (acts) atomicAdd(&hc->activations, acts);
+        if (filtered) atomicAdd(&hc->remote_filtered, filtered);
+        if (hub_e) atomicAdd(&hc->hub_edges, hub_e);
     }
     gum_iter_trace* tr = c.trace[w0];
     if (tr && threadIdx.x == 0 && k < (unsigned)kTraceMax) {
@@ -1824,9 +1899,21 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
     }
     const double N = (double)c.num_vertices, d = c.pr_d, D = s_D;
     double dang = 0.0, res = 0.0;
+    const bool mir = c.mirrors && c.P > 1;
     for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
         const double xo = F.x[i];
-        const double nx = (1.0 - d) / N + d * (F.acc[i] + D / N);
+        double a = F.acc[i];
+        if (mir) {
+            // NEXT-1: the aggregated pushes of every other worker to this (for them outer) vertex are
+            // pulled from their mirrors (coalesced peer loads) and the mirror entries cleared
+            for (int q = 1; q < c.P; q++) {
+                const int g = f + q < c.P ? f + q : f + q - c.P;  // peers in rotated order
+                double* m = c.f[g].macc + F.base + i;
+                a += *m;
+                *m = 0.0;
+            }
+        }
+        const double nx = (1.0 - d) / N + d * (a + D / N);
         res += fabs(nx - xo);
         const unsigned long long od = __ldg(F.row_ptr + i + 1) - __ldg(F.row_ptr + i);
         if (od == 0) dang += nx;

@@ -66,5 +66,19 @@ cudaError_t setup_pr_blocked(const unsigned long long* rp, const unsigned* col, 
 cudaError_t setup_count_dangling(const unsigned long long* row_ptr, unsigned V, unsigned long long* d_count,
                                  cudaStream_t s);
 unsigned host_feistel(unsigned v, unsigned V, unsigned long long seed);
+// DEGREE relabel: d_perm[old] = new, d_inv[new] = old, ids ordered by decreasing in-degree (stable)
+size_t setup_degree_tmp_bytes(unsigned V);
+cudaError_t setup_relabel_degree(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w,
+                                 unsigned V, unsigned long long E, unsigned* d_perm, unsigned* d_inv,
+                                 unsigned long long* r_row_ptr, unsigned* r_col, unsigned* r_w, void* tmp,
+                                 size_t tmp_bytes, cudaStream_t s);
+// NEXT-1 hub cache: off[0..n] = exclusive prefix of the cached (out-degree > t4) list lengths of global rows
+// [b0, b0+n) (off[n] = total; tmp sized by setup_scan_tmp_bytes(n)); then fill copies the lists and sets
+// off[v] = ~0 for rows that are not cached. hw / w may be null.
+cudaError_t setup_hub_offsets(const unsigned long long* row_ptr, unsigned b0, unsigned n, unsigned t4,
+                              unsigned long long* off, void* tmp, size_t tmp_bytes, cudaStream_t s);
+cudaError_t setup_hub_fill(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w, unsigned b0,
+                           unsigned n, unsigned t4, unsigned long long* off, unsigned* hcol, unsigned* hw,
+                           cudaStream_t s);
 
 }  // namespace gum

@@ -77,6 +77,15 @@ struct FragBufs {
     unsigned* pb_fill = nullptr;
     unsigned* pb_done = nullptr;
     unsigned* pb_buf = nullptr;
+    // NEXT-1 outer-vertex mirror of this worker (V entries of 8 B; PR acc / BFS bits / SSSP-WCC min alias it)
+    void* mbuf = nullptr;
+};
+
+// NEXT-1 hub cache: worker w's copy of fragment f's hub lists
+struct HubBufs {
+    unsigned long long* off = nullptr;
+    unsigned* col = nullptr;
+    unsigned* w = nullptr;
 };
 
 }  // namespace
@@ -110,7 +119,8 @@ struct gum_ctx {
     int part_kind = GUM_PART_SEG;
     unsigned long long seed = 0;
     unsigned bounds[kMaxW + 1] = {0};
-    unsigned* inv = nullptr;  // relabelled id -> original id (RANDOM)
+    unsigned* inv = nullptr;  // relabelled id -> original id (RANDOM, DEGREE)
+    unsigned* perm = nullptr; // original id -> relabelled id (DEGREE; RANDOM computes it with the Feistel map)
     unsigned long long* p_row_ptr = nullptr;  // the partitioned global CSR (relabelled or original)
     unsigned* p_col = nullptr;
     unsigned* p_w = nullptr;
@@ -121,6 +131,12 @@ struct gum_ctx {
     unsigned pb_shift = 0, pb_nb = 0;
     int pr_blocks = 1;
     FragBufs fr[kMaxW];
+    unsigned long long* s_rp_g = nullptr;  // global symmetric CSR (WCC), kept for the hub cache
+    unsigned* s_col_g = nullptr;
+    int hub_kind = 0;                      // hub cache built from: 0 none, 1 out-CSR (BFS/SSSP), 2 symmetric (WCC)
+    HubBufs hub[kMaxW][kMaxW];             // [worker][fragment]
+    std::vector<Alloc> hub_allocs;
+    unsigned long long hub_entries = 0;    // cached list entries per worker copy set (stats / tests)
     unsigned long long n_dangling = 0;
     RunCtl* rctl[kMaxW] = {nullptr};
     LBSlot* lb[kMaxW] = {nullptr};
@@ -240,6 +256,13 @@ void drop_partition(gum_ctx* c) {
     }
     c->mp_epoch = 0;
     for (auto& p : c->pad) p = nullptr;
+    free_list(c, c->hub_allocs);
+    c->hub_kind = 0;
+    c->hub_entries = 0;
+    for (auto& row : c->hub)
+        for (auto& h : row) h = HubBufs{};
+    c->s_rp_g = nullptr;
+    c->s_col_g = nullptr;
     free_list(c, c->part_allocs);
     c->partitioned = false;
     c->sym_ready = false;
@@ -249,6 +272,7 @@ void drop_partition(gum_ctx* c) {
     c->pb_shift = c->pb_nb = 0;
     c->has_result = false;
     c->inv = nullptr;
+    c->perm = nullptr;
     c->p_row_ptr = nullptr;
     c->p_col = nullptr;
     c->p_w = nullptr;
@@ -345,8 +369,20 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.ctl = F.ctl;
         p.V = F.V;
         p.base = F.base;
+        p.macc = (double*)F.mbuf;
+        p.msent = (unsigned*)F.mbuf;
+        p.mmin = (unsigned*)F.mbuf;
         d.lb[f] = c->lb[f];
     }
+    d.mirrors = (c->cfg.mirrors && c->P > 1 && c->fr[0].mbuf) ? 1 : 0;
+    const int hk = alg == GUM_WCC ? 2 : (alg == GUM_PR ? -1 : 1);
+    d.hub_on = (c->hub_kind == hk) ? 1 : 0;
+    for (int w = 0; w < c->P && d.hub_on; w++)
+        for (int f = 0; f < c->P; f++) {
+            d.hub[w][f].off = c->hub[w][f].off;
+            d.hub[w][f].col = c->hub[w][f].col;
+            d.hub[w][f].w = c->hub[w][f].w;
+        }
     for (int w = 0; w < c->P; w++) {
         int u = c->split ? w : 0;
         d.rctl[w] = c->rctl[unit_w0(c, u)];
@@ -428,6 +464,7 @@ int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     GUM_FLD(F.ctl); GUM_FLD(F.pr_col); GUM_FLD(F.pr_q_v); GUM_FLD(F.pr_q_off); GUM_FLD(F.pr_tile);
     GUM_FLD(F.sq_col); GUM_FLD(F.sq_q_v); GUM_FLD(F.sq_q_off); GUM_FLD(F.sq_tile); GUM_FLD(F.in_row_ptr);
     GUM_FLD(F.in_col); GUM_FLD(c->lb[f]); GUM_FLD(c->rctl[f]); GUM_FLD(c->trace[f]); GUM_FLD(c->pad[f]);
+    GUM_FLD(F.mbuf);
 #undef GUM_FLD
     return n;
 }
@@ -622,7 +659,82 @@ gum_status build_sym(gum_ctx* c) {
         }
         CK(cudaSetDevice(c->dev[0]));
     }
+    c->s_rp_g = srp;
+    c->s_col_g = scol;
     c->sym_ready = true;
+    drop_graphs(c);
+    return GUM_OK;
+}
+
+// NEXT-1 hub cache: every worker gets a local copy of the adjacency lists of every other fragment's
+// vertices with out-degree > t4, built from the global (partitioned) CSR of the algorithm: the out-CSR for
+// BFS/SSSP, the symmetric CSR for WCC. On one device the workers share one copy per fragment (their memory
+// is the same); across devices each worker's copy lives on its own device; in multi-process mode each rank
+// builds the copies it needs from its own full graph.
+gum_status build_hub(gum_ctx* c, int alg) {
+    if (!c->cfg.hub_cache || c->P == 1 || alg == GUM_PR) return GUM_OK;
+    const int kind = alg == GUM_WCC ? 2 : 1;
+    if (c->hub_kind == kind) return GUM_OK;
+    free_list(c, c->hub_allocs);
+    for (auto& row : c->hub)
+        for (auto& h : row) h = HubBufs{};
+    c->hub_kind = 0;
+    c->hub_entries = 0;
+    const unsigned long long* rp = kind == 2 ? c->s_rp_g : c->p_row_ptr;
+    const unsigned* col = kind == 2 ? c->s_col_g : c->p_col;
+    const unsigned* wt = kind == 2 ? nullptr : c->p_w;
+    if (!rp || !col) return fail(c, GUM_ESTATE, "hub cache: global CSR not available");
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    const unsigned t4 = c->cfg.hub_degree;
+    for (int f = 0; f < c->P; f++) {
+        const unsigned b0 = c->bounds[f], n = c->bounds[f + 1] - c->bounds[f];
+        // the workers that need a copy of fragment f (built here), and where the copy lives
+        bool need = false;
+        for (int w = 0; w < c->P; w++) need = need || (w != f && (!c->mp || w == c->rank));
+        if (!need) continue;
+        unsigned long long* off = (unsigned long long*)dalloc(c, d0, (n + 1ull) * 8, c->hub_allocs);
+        std::vector<Alloc> tmp;
+        const size_t tb = setup_scan_tmp_bytes(n);
+        void* t = dalloc(c, d0, tb, tmp);
+        if (!off || !t) {
+            free_list(c, tmp);
+            return fail(c, GUM_ENOMEM, "hub cache offsets alloc failed");
+        }
+        CK(setup_hub_offsets(rp, b0, n, t4, off, t, tb, s));
+        unsigned long long tot = 0;
+        CK(cudaMemcpyAsync(&tot, off + n, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        free_list(c, tmp);
+        if (tot >= (1ull << 32)) return fail(c, GUM_EUNSUP, "hub cache of fragment %d has >= 2^32 entries", f);
+        unsigned* hcol = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(tot, 1) * 4, c->hub_allocs);
+        unsigned* hw = wt ? (unsigned*)dalloc(c, d0, std::max<unsigned long long>(tot, 1) * 4, c->hub_allocs) : nullptr;
+        if (!hcol || (wt && !hw)) return fail(c, GUM_ENOMEM, "hub cache alloc failed (%llu entries)", tot);
+        CK(setup_hub_fill(rp, col, wt, b0, n, t4, off, hcol, hw, s));
+        CK(cudaStreamSynchronize(s));
+        c->hub_entries += tot;
+        for (int w = 0; w < c->P; w++) {
+            if (w == f || (c->mp && w != c->rank)) continue;
+            HubBufs& H = c->hub[w][f];
+            if (c->dev[w] == d0) {
+                H.off = off;
+                H.col = hcol;
+                H.w = hw;
+                continue;
+            }
+            const int dw = c->dev[w];
+            H.off = (unsigned long long*)dalloc(c, dw, (n + 1ull) * 8, c->hub_allocs);
+            H.col = (unsigned*)dalloc(c, dw, std::max<unsigned long long>(tot, 1) * 4, c->hub_allocs);
+            H.w = hw ? (unsigned*)dalloc(c, dw, std::max<unsigned long long>(tot, 1) * 4, c->hub_allocs) : nullptr;
+            if (!H.off || !H.col || (hw && !H.w)) return fail(c, GUM_ENOMEM, "hub cache copy alloc failed");
+            CK(cudaMemcpyPeerAsync(H.off, dw, off, d0, (n + 1ull) * 8, s));
+            if (tot) CK(cudaMemcpyPeerAsync(H.col, dw, hcol, d0, tot * 4, s));
+            if (tot && hw) CK(cudaMemcpyPeerAsync(H.w, dw, hw, d0, tot * 4, s));
+            CK(cudaStreamSynchronize(s));
+        }
+    }
+    c->hub_kind = kind;
     drop_graphs(c);
     return GUM_OK;
 }
@@ -964,6 +1076,7 @@ static unsigned long long config_hash(const gum_config* cfg) {
     GUM_HC(osteal_active_threshold); GUM_HC(osteal_edges_per_worker); GUM_HC(chunk_edges); GUM_HC(pr_iterations);
     GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
     GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt); GUM_HC(osteal_sync_edges);
+    GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree);
 #undef GUM_HC
     return h;
 }
@@ -1162,7 +1275,8 @@ gum_status gum_partition(gum_ctx* c, gum_part kind, uint64_t seed) {
     if (!c) return GUM_EINVAL;
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->loaded) return fail(c, GUM_ESTATE, "gum_partition before gum_load_csr");
-    if (kind != GUM_PART_SEG && kind != GUM_PART_RANDOM) return fail(c, GUM_EINVAL, "bad partition kind");
+    if (kind != GUM_PART_SEG && kind != GUM_PART_RANDOM && kind != GUM_PART_DEGREE)
+        return fail(c, GUM_EINVAL, "bad partition kind");
     drop_partition(c);
     gum_status st = partition_body(c, kind, seed);
     if (c->mp) {
@@ -1181,20 +1295,25 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
     c->part_kind = kind;
     c->seed = seed;
     // ---- a2: relabel (RANDOM) then edge-balanced contiguous ranges (SEG)
-    if (kind == GUM_PART_RANDOM) {
+    if (kind == GUM_PART_RANDOM || kind == GUM_PART_DEGREE) {
         c->inv = (unsigned*)dalloc(c, d0, (size_t)V * 4, c->part_allocs);
+        c->perm = kind == GUM_PART_DEGREE ? (unsigned*)dalloc(c, d0, (size_t)V * 4, c->part_allocs) : nullptr;
         c->p_row_ptr = (unsigned long long*)dalloc(c, d0, (V + 1ull) * 8, c->part_allocs);
         c->p_col = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs);
         c->p_w = c->has_w ? (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs) : nullptr;
         std::vector<Alloc> tmp;
-        size_t tb = setup_scan_tmp_bytes(V);
+        size_t tb = kind == GUM_PART_DEGREE ? setup_degree_tmp_bytes(V) : setup_scan_tmp_bytes(V);
         void* t = dalloc(c, d0, tb, tmp);
-        if (!c->inv || !c->p_row_ptr || !c->p_col || (c->has_w && !c->p_w) || !t) {
+        if (!c->inv || !c->p_row_ptr || !c->p_col || (c->has_w && !c->p_w) || !t ||
+            (kind == GUM_PART_DEGREE && !c->perm)) {
             free_list(c, tmp);
             return fail(c, GUM_ENOMEM, "relabel alloc failed");
         }
-        cudaError_t e = setup_relabel(c->g_row_ptr, c->g_col, c->g_w, V, E, seed, c->inv, c->p_row_ptr, c->p_col,
-                                      c->p_w, t, tb, s);
+        cudaError_t e = kind == GUM_PART_DEGREE
+                            ? setup_relabel_degree(c->g_row_ptr, c->g_col, c->g_w, V, E, c->perm, c->inv, c->p_row_ptr,
+                                                   c->p_col, c->p_w, t, tb, s)
+                            : setup_relabel(c->g_row_ptr, c->g_col, c->g_w, V, E, seed, c->inv, c->p_row_ptr,
+                                            c->p_col, c->p_w, t, tb, s);
         if (e == cudaSuccess) e = cudaStreamSynchronize(s);
         free_list(c, tmp);
         if (e != cudaSuccess) return fail(c, GUM_ECUDA, "relabel: %s", cudaGetErrorString(e));
@@ -1263,6 +1382,11 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
         if (!F.state || !F.x || !F.acc || !F.cx || !F.bm || !F.vis || !F.bm2 || !F.far || !F.app || !F.q_v || !F.q_off || !F.q_base || !F.ctl)
             return fail(c, GUM_ENOMEM, "fragment %d state alloc failed", f);
+        if (c->cfg.mirrors && c->P > 1) {
+            // NEXT-1: worker f's outer-vertex mirror (global id space, 8 B per vertex)
+            F.mbuf = dalloc(c, F.dev, (size_t)V * 8, c->part_allocs);
+            if (!F.mbuf) return fail(c, GUM_ENOMEM, "worker %d mirror alloc failed", f);
+        }
         CK(cudaSetDevice(F.dev));
         CK(cudaMemset(F.ctl, 0, sizeof(FragCtl)));
         CK(cudaSetDevice(d0));
@@ -1346,6 +1470,7 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
         st = build_pb(c);
         if (st == GUM_OK) st = build_in(c);
     }
+    if (st == GUM_OK) st = build_hub(c, alg);  // worker-local copies: nothing to publish
     if (c->mp && built) st = mp_publish(c, st);
     return st;
 }
@@ -1364,7 +1489,13 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     int src_frag = -1;
     unsigned src_local = 0;
     if (alg == GUM_BFS || alg == GUM_SSSP) {
-        unsigned sp = c->inv ? host_feistel(source, c->V, c->seed) : source;
+        unsigned sp = source;
+        if (c->perm) {
+            CK(cudaSetDevice(c->dev[0]));
+            CK(cudaMemcpy(&sp, c->perm + source, 4, cudaMemcpyDeviceToHost));
+        } else if (c->inv) {
+            sp = host_feistel(source, c->V, c->seed);
+        }
         for (int f = 0; f < c->P; f++)
             if (sp >= c->bounds[f] && sp < c->bounds[f + 1]) src_frag = f;
         src_local = sp - c->bounds[src_frag];
@@ -1525,6 +1656,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->remote_updates += fc.remote_updates;
             stats->activations += fc.activations;
             stats->vertices_frontier += fc.frontier_vertices;
+            stats->remote_filtered += fc.remote_filtered;
+            stats->hub_cached_edges += fc.hub_edges;
             if (getenv("GUM_DEBUG"))
                 fprintf(stderr, "[gum] frag %d: V=%u E=%llu qlen=%llu edges_done=%llu frontier_edges=%llu frontier_vertices=%llu app_cnt=%u tcnt=%u,%u,%u\n",
                         f, c->fr[f].V, (unsigned long long)(alg == GUM_WCC ? c->fr[f].sE : c->fr[f].E), fc.qlen,
@@ -1535,6 +1668,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->edges_frontier = qedges_total * R.iter;
             stats->vertices_frontier = 0;
             for (int f = 0; f < c->P; f++) stats->vertices_frontier += c->fr[f].pr_qlen * R.iter;
+            if (d.mirrors) stats->mirror_flush_bytes = (unsigned long long)R.iter * (c->P - 1) * c->V * 8ull;
         }
         CK(cudaSetDevice(c->dev[0]));
     }

@@ -113,8 +113,8 @@ __global__ void k_new_deg(const unsigned long long* rp, const unsigned* inv, uns
 }
 
 __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
-                               unsigned V, unsigned long long seed, const unsigned long long* nrp, unsigned* ncol,
-                               unsigned* nw) {
+                               unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
+                               unsigned* ncol, unsigned* nw) {
     const unsigned lane = threadIdx.x & 31;
     const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
     const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
@@ -122,7 +122,7 @@ __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col
         const unsigned o = inv[v];
         const unsigned long long s0 = rp[o], s1 = rp[o + 1], d0 = nrp[v];
         for (unsigned long long j = lane; j < s1 - s0; j += 32) {
-            ncol[d0 + j] = feistel(col[s0 + j], V, seed);
+            ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
             if (w) nw[d0 + j] = w[s0 + j];
         }
     }
@@ -136,7 +136,56 @@ cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col
     k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
     cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
     if (e != cudaSuccess) return e;
-    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, r_row_ptr, r_col, r_w);
+    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
+    return cudaGetLastError();
+}
+
+// DEGREE relabel (layout option): new ids in order of decreasing in-degree (ties by id), so the
+// destinations most edges point to share a few KB of the visited bitmap / state array and stay cache-resident.
+__global__ void k_indeg(const unsigned* col, unsigned long long E, unsigned* deg) {
+    for (unsigned long long e = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; e < E;
+         e += (unsigned long long)gridDim.x * blockDim.x)
+        atomicAdd(deg + col[e], 1u);
+}
+__global__ void k_deg_keys(unsigned* deg, unsigned V, unsigned* ids) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+        deg[v] = ~deg[v];  // ascending radix order of ~deg = decreasing degree
+        ids[v] = v;
+    }
+}
+__global__ void k_perm_of(const unsigned* inv, unsigned V, unsigned* perm) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) perm[inv[v]] = v;
+}
+
+size_t setup_degree_tmp_bytes(unsigned V) {
+    size_t a = 0, b = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, a, (unsigned*)nullptr, (unsigned*)nullptr, (unsigned*)nullptr,
+                                    (unsigned*)nullptr, (int)0 + (size_t)V);
+    cub::DeviceScan::ExclusiveSum(nullptr, b, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (int)0 + (size_t)V + 1);
+    return (a > b ? a : b) + 2 * ((size_t)V * 4 + 256) + 256;
+}
+
+cudaError_t setup_relabel_degree(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w,
+                                 unsigned V, unsigned long long E, unsigned* d_perm, unsigned* d_inv,
+                                 unsigned long long* r_row_ptr, unsigned* r_col, unsigned* r_w, void* tmp,
+                                 size_t tmp_bytes, cudaStream_t s) {
+    const size_t vb = ((size_t)V * 4 + 255) & ~(size_t)255;
+    unsigned* keys_in = (unsigned*)tmp;
+    unsigned* keys_out = (unsigned*)((char*)tmp + vb);
+    void* t = (char*)tmp + 2 * vb;
+    size_t tb = tmp_bytes - 2 * vb;
+    cudaError_t e = cudaMemsetAsync(keys_in, 0, (size_t)V * 4, s);
+    if (e != cudaSuccess) return e;
+    k_indeg<<<1184, 256, 0, s>>>(col, E, keys_in);
+    k_deg_keys<<<1184, 256, 0, s>>>(keys_in, V, d_perm);  // d_perm holds the identity as sort input
+    e = cub::DeviceRadixSort::SortPairs(t, tb, keys_in, keys_out, d_perm, d_inv, (size_t)V, 0, 32, s);
+    if (e != cudaSuccess) return e;
+    k_perm_of<<<1184, 256, 0, s>>>(d_inv, V, d_perm);
+    k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
+    e = cub::DeviceScan::ExclusiveSum(t, tb, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
+    if (e != cudaSuccess) return e;
+    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
     return cudaGetLastError();
 }
 
@@ -387,6 +436,55 @@ __global__ void k_count_dangling(const unsigned long long* rp, unsigned V, unsig
 cudaError_t setup_count_dangling(const unsigned long long* row_ptr, unsigned V, unsigned long long* d_count,
                                  cudaStream_t s) {
     k_count_dangling<<<592, 256, 0, s>>>(row_ptr, V, d_count);
+    return cudaGetLastError();
+}
+
+// NEXT-1 hub cache (P:274 Example 6): the adjacency lists of global rows [b0, b0+n) with out-degree > t4,
+// packed into a worker-local copy. off[v] = position of row b0+v in the copy, ~0 if not cached.
+__global__ void k_hub_deg(const unsigned long long* rp, unsigned b0, unsigned n, unsigned t4,
+                          unsigned long long* off) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v <= n; v += gridDim.x * blockDim.x) {
+        unsigned long long d = 0;
+        if (v < n) {
+            d = rp[b0 + v + 1] - rp[b0 + v];
+            if (d <= t4) d = 0;
+        }
+        off[v] = d;
+    }
+}
+
+// one warp per row: copy a cached list, or mark the row as not cached
+__global__ void k_hub_fill(const unsigned long long* rp, const unsigned* col, const unsigned* w, unsigned b0,
+                           unsigned n, unsigned t4, unsigned long long* off, unsigned* hcol, unsigned* hw) {
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long nwarps = (unsigned long long)gridDim.x * (blockDim.x / 32);
+    for (unsigned long long v = blockIdx.x * (unsigned long long)(blockDim.x / 32) + threadIdx.x / 32; v < n;
+         v += nwarps) {
+        const unsigned long long a = rp[b0 + v], d = rp[b0 + v + 1] - a;
+        const unsigned long long o = off[v];
+        if (d > t4) {
+            for (unsigned long long j = lane; j < d; j += 32) {
+                hcol[o + j] = col[a + j];
+                if (hw) hw[o + j] = w[a + j];
+            }
+        }
+        __syncwarp();
+        if (lane == 0 && d <= t4) off[v] = ~0ull;
+    }
+}
+
+cudaError_t setup_hub_offsets(const unsigned long long* row_ptr, unsigned b0, unsigned n, unsigned t4,
+                              unsigned long long* off, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    k_hub_deg<<<592, 256, 0, s>>>(row_ptr, b0, n, t4, off);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, off, off, (size_t)n + 1, s);
+    if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+
+cudaError_t setup_hub_fill(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w, unsigned b0,
+                           unsigned n, unsigned t4, unsigned long long* off, unsigned* hcol, unsigned* hw,
+                           cudaStream_t s) {
+    k_hub_fill<<<1184, 256, 0, s>>>(row_ptr, col, w, b0, n, t4, off, hcol, hw);
     return cudaGetLastError();
 }
 

@@ -4,6 +4,7 @@ without a GPU (no CPU fallback exists)."""
 import ctypes
 import os
 import re
+import subprocess
 
 import numpy as np
 import pytest
@@ -56,10 +57,28 @@ def test_build_csr_edge_cases():
         gum.build_csr(3, np.array([0, 5], np.uint32), np.array([1, 1], np.uint32))
 
 
-def test_struct_layouts_match_header():
-    # sizes fixed by include/gum.h (LP64)
-    assert ctypes.sizeof(gum.gum_run_stats) == 4 + 4 + 9 * 8 + 4 * 4 + 8 + 8
-    assert ctypes.sizeof(gum.gum_iter_trace) == 4 * 8 * 8 + 16 + 8
+def test_struct_layouts_match_header(tmp_path):
+    # every field offset and struct size of the ctypes mirrors equals the C compiler's view of include/gum.h
+    structs = {"gum_config": gum.gum_config, "gum_run_stats": gum.gum_run_stats,
+               "gum_iter_trace": gum.gum_iter_trace, "gum_kernel_times": gum.gum_kernel_times,
+               "gum_mp_config": gum.gum_mp_config}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "gum.h"', "int main(void) {"]
+    for name, cls in structs.items():
+        lines.append(f'printf("{name} size %zu\\n", sizeof({name}));')
+        for fname, _ in cls._fields_:
+            lines.append(f'printf("{name} {fname} %zu\\n", offsetof({name}, {fname}));')
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include")
+    subprocess.run(["gcc", "-I", inc, str(src), "-o", str(exe)], check=True)
+    out = subprocess.run([str(exe)], check=True, capture_output=True, text=True).stdout.split("\n")
+    got = {tuple(l.split()[:2]): int(l.split()[2]) for l in out if l.strip()}
+    for name, cls in structs.items():
+        assert got[(name, "size")] == ctypes.sizeof(cls), name
+        for fname, _ in cls._fields_:
+            assert got[(name, fname)] == getattr(cls, fname).offset, (name, fname)
 
 
 def test_no_gpu_means_error_not_fallback():

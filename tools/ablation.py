@@ -9,6 +9,13 @@ drops below the OSteal threshold ("long tail"), OSteal on vs off.
 
   python tools/ablation.py --fsteal --scale 22 --workers 8 [--split]
   python tools/ablation.py --osteal --grid 2048 --workers 8 [--split]
+
+NEXT-1: cross-fragment traffic with and without outer-vertex mirrors and the hub cache, per
+algorithm on RMAT with a random partition over 8 workers: remote atomics issued (each one crosses NVLink when
+the workers are GPUs), updates absorbed by the mirrors, PR mirror bytes pulled per run, stolen edges read
+from a local hub copy. Outputs must be identical (PR: within the parity tolerance).
+
+  python tools/ablation.py --next1 --scale 20 --workers 8
 """
 import argparse
 import json
@@ -106,6 +113,41 @@ def osteal(args):
     return res
 
 
+def next1(args):
+    g = inputs.rmat(args.scale, 16, seed=2)
+    src = inputs.pick_source(g, 2)
+    csr = gum.build_csr(g.num_vertices, g.src, g.dst, g.w)
+    res = {}
+    for alg in ("bfs", "sssp", "wcc", "pr"):
+        rows = {}
+        outs = []
+        for name, kw in (("plain", {}), ("mirrors", dict(mirrors=True)),
+                         ("mirrors+hub", dict(mirrors=True, hub_cache=True, hub_degree=args.hub_degree))):
+            rp, col, w = csr
+            with gum.Context(num_gpus=args.workers, chunk_edges=args.chunk, **kw) as ctx:
+                ctx.load_csr(rp, col, w if alg == "sssp" else None)
+                ctx.partition("random", 1)
+                ctx.run(alg, src)
+                st = min((ctx.run(alg, src) for _ in range(3)), key=lambda t: t.ms)
+                outs.append(ctx.result())
+            op = 8 if alg == "pr" else 4
+            rows[name] = dict(run_ms=round(st.ms, 3), iterations=st.iterations, remote_atomics=st.remote_updates,
+                              remote_atomic_bytes=st.remote_updates * op, absorbed_by_mirror=st.remote_filtered,
+                              mirror_flush_bytes=st.mirror_flush_bytes, edges_stolen=st.edges_stolen,
+                              stolen_edges_from_hub_copy=st.hub_cached_edges)
+        if alg == "pr":
+            ok = all(float(np.abs(o - outs[0]).sum()) <= 1e-6 for o in outs)
+        else:
+            ok = all(np.array_equal(o, outs[0]) for o in outs)
+        rows["identical_outputs"] = bool(ok)
+        res[alg] = rows
+    res["workload"] = (f"RMAT scale {args.scale} EF16 (seed 2), random partition over {args.workers} virtual workers "
+                       f"on 1 B200, chunk {args.chunk} edges, hub t4 = {args.hub_degree}; remote atomic bytes = "
+                       f"count x 4 B (8 B for PR's fp64 adds); on one GPU every access stays in HBM, so the times "
+                       f"are not NVLink times -- the counts are the cross-GPU traffic the same run issues on N GPUs")
+    return res
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--fsteal", action="store_true")
@@ -117,6 +159,8 @@ def main():
     ap.add_argument("--threshold", type=int, default=4096)
     ap.add_argument("--delta", type=int, default=0, help="SSSP near-far split (0 = plain frontier)")
     ap.add_argument("--split", action="store_true")
+    ap.add_argument("--next1", action="store_true")
+    ap.add_argument("--hub-degree", type=int, default=64)
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     out = {}
@@ -134,6 +178,17 @@ def main():
         for k in ("on", "off"):
             print(f"OSteal {k}: {o[k]['run_ms']:.2f} ms, {o[k]['iterations']} iterations, owners {o[k]['final_owners']}, "
                   f"tail iterations {o[k]['tail_iterations']}, tail advance {o[k]['tail_advance_us']} us")
+    if args.next1:
+        out["next1"] = next1(args)
+        for alg, rows in out["next1"].items():
+            if alg == "workload":
+                continue
+            for k, r in rows.items():
+                if isinstance(r, dict):
+                    print(f"{alg:5s} {k:12s} {r['run_ms']:9.3f} ms  remote atomics {r['remote_atomics']:>12d}  "
+                          f"absorbed {r['absorbed_by_mirror']:>12d}  flush {r['mirror_flush_bytes']:>12d} B  "
+                          f"hub-copy edges {r['stolen_edges_from_hub_copy']}")
+            print(f"{alg:5s} identical outputs: {rows['identical_outputs']}")
     if args.out:
         json.dump(out, open(args.out, "w"), indent=1)
 

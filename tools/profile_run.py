@@ -18,14 +18,17 @@ ap.add_argument("--alg", default="bfs")
 ap.add_argument("--runs", type=int, default=1)
 ap.add_argument("--gpus", type=int, default=1)
 ap.add_argument("--host-loop", type=int, default=1)
+ap.add_argument("--part", default="seg")
 a = ap.parse_args()
 g = inputs.make_config(a.config, weighted=(a.alg == "sssp"))
 s = 0 if a.config == "C3" else inputs.pick_source(g, int(a.config[1]))
 rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
 with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop)) as ctx:
     ctx.load_csr(rp, col, w)
-    ctx.partition()
+    ctx.partition(a.part, 1)
     ctx.prepare(a.alg)
     for _ in range(a.runs):
         st = ctx.run(a.alg, s)
     print(st)
+    if a.host_loop:
+        print(ctx.profile())
