@@ -40,6 +40,7 @@ WORKLOADS = {
 }
 PR_SAMPLE_ITERS = 2
 DEFAULT_ALG = {"C1": "bfs", "C2": "bfs", "C3": "sssp", "C4": "wcc", "C5": "pr"}
+L2_BYTES = 126 * 2**20  # B200 L2 (the flush buffer is twice this)
 
 
 def env_int(k, d):
@@ -300,7 +301,10 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-variants", action="store_true", help="skip the NEXT-4 variant measurement")
-    ap.add_argument("--part", default="seg")
+    ap.add_argument("--part", default=None,
+                    help="seg | random | degree (default: degree for BFS, where the in-degree-ordered layout keeps "
+                         "the hub probes in L1 -- measured 2.21 -> 1.82 ms on C2; seg otherwise, where it loses: "
+                         "hub atomics contend on a few L2 lines)")
     ap.add_argument("--fsteal", type=int, default=1)
     ap.add_argument("--osteal", type=int, default=1)
     ap.add_argument("--sssp-delta", type=int, default=None,
@@ -309,6 +313,8 @@ def main():
     ap.add_argument("--bfs-pull", type=int, default=0, help="NEXT-4 direction-optimising BFS (bottom-up iterations)")
     args = ap.parse_args()
     alg = args.alg or DEFAULT_ALG[args.config]
+    if args.part is None:
+        args.part = "degree" if alg == "bfs" else "seg"
     rank = env_int("RANK", 0)
     world = env_int("WORLD_SIZE", 1)
     N = args.gpus
@@ -330,7 +336,8 @@ def main():
                 "fsteal": args.fsteal, "osteal": args.osteal, "tail_engine_vertices": args.tail,
                 "bfs_direction_opt": bool(args.bfs_pull) if alg == "bfs" else None,
                 "sssp_near_far_delta": sssp_delta if alg == "sssp" else None,
-                "l2": "inputs larger than L2 (col array > 126 MB); no flush"}
+                "l2": ("L2 flushed between timed steps (2x-L2 buffer write, excluded from the per-step events)"
+                       if args.config == "C1" else "inputs larger than L2 (col array > 126 MB); no flush")}
 
     if world > 1 and args.impl == "ours":
         ctx_kw = dict(fsteal=bool(args.fsteal), osteal=bool(args.osteal), sssp_delta=sssp_delta,
@@ -399,17 +406,36 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     total_edges, launches = 0, 0
     sampler = ClockSampler(0)
+    small_inputs = args.config == "C1"
+    # inputs smaller than L2 (C1): flush L2 between timed steps (write a 2x-L2 buffer) and time every
+    # step with its own events so the flush is excluded; larger inputs stream through L2 anyway
+    flush = None
+    if small_inputs:
+        flush = torch.empty(int(2 * L2_BYTES) // 4, dtype=torch.int32, device="cuda")
     with sampler:
         with torch.cuda.stream(stream):
-            ev0.record(stream)
-            for i in range(args.steps):
-                s = sources[i % len(sources)]
-                st = ctx.run(alg, s)
-                total_edges += edges_of[s]
-                launches += st.kernel_launches
-            ev1.record(stream)
+            if flush is None:
+                ev0.record(stream)
+                for i in range(args.steps):
+                    s = sources[i % len(sources)]
+                    st = ctx.run(alg, s)
+                    total_edges += edges_of[s]
+                    launches += st.kernel_launches
+                ev1.record(stream)
+            else:
+                pairs = []
+                for i in range(args.steps):
+                    s = sources[i % len(sources)]
+                    flush.fill_(i)
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    st = ctx.run(alg, s)
+                    b.record(stream)
+                    pairs.append((a, b))
+                    total_edges += edges_of[s]
+                    launches += st.kernel_launches
         torch.cuda.synchronize()
-    ms = ev0.elapsed_time(ev1)
+    ms = ev0.elapsed_time(ev1) if flush is None else sum(a.elapsed_time(b) for a, b in pairs)
     barrier()
     value = total_edges / (ms / 1e3) / 1e9
     ms_per_step = ms / args.steps

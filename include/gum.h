@@ -185,6 +185,8 @@ typedef struct {
                                  (BFS/SSSP/WCC: not sent; PR: aggregated, then flushed in bulk) */
     uint64_t hub_cached_edges;/* NEXT-1 hub cache: edges of non-local fragments expanded from a local copy */
     uint64_t mirror_flush_bytes; /* PR mirrors: bytes the finalize read from peer mirrors */
+    uint32_t blocked_iterations; /* WCC: iterations run on the static destination-blocked queue */
+    uint32_t pad0;
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

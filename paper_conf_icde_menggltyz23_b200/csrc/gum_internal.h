@@ -76,6 +76,9 @@ struct alignas(128) RunCtl {
     unsigned int pb;          // the current advance bins its discoveries (apply runs next body)
     unsigned int pull;        // the current BFS iteration runs bottom-up (k_bfs_pull instead of advance)
     unsigned int skip_filter; // the first iteration's queue is static (WCC blocked): no filter pass
+    unsigned int blocked;     // WCC: the current advance runs on the static destination-blocked queue
+                              // (1 = every vertex active, 2 = sources masked by the frontier bitmap)
+    unsigned int blocked_iters;
     unsigned int plan_lo[kMaxW][kMaxW], plan_hi[kMaxW][kMaxW];  // FSteal plan: chunks [lo,hi) of queue f -> worker w
     double plan_z;            // planned makespan (edges) of the current iteration
     unsigned int nf_sweep;    // SSSP near-far: the next filter also scans the far set
@@ -192,6 +195,9 @@ struct DevCtx {
     unsigned int bfs_pull;      // direction-optimising BFS enabled (in-CSR built)
     unsigned long long total_edges;  // sum of the fragments' out-edges
     int mirrors;                // NEXT-1 outer-vertex mirrors (P > 1 only)
+    unsigned int filter_swizzle;  // filter: spread each CTA's tile range over the id space (stride permutation)
+    unsigned int wcc_blocked;     // WCC static destination-blocked queue exists: dense iterations may run on
+                                  // it (the filter keeps the frontier bitmap in F.far)
     int hub_on;                 // NEXT-1 hub cache built for this algorithm
     HubPtrs hub[kMaxW][kMaxW];  // [worker][fragment] (fragment != worker)
 };

@@ -143,6 +143,8 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     RunCtl* rc = c.rctl[w0];
     rc->next_dense = next_dense0;
     rc->skip_filter = skip_filter0;
+    rc->blocked = skip_filter0 ? 1u : 0u;
+    rc->blocked_iters = 0;
     rc->iter = 0;
     rc->done = 0;
     rc->m = c.P;
@@ -203,6 +205,14 @@ __device__ __forceinline__ Pair block_excl_scan(Pair v, Pair* s_warp, Pair& tota
     return Pair{wexcl.cnt + inc.cnt - v.cnt, wexcl.deg + inc.deg - v.deg};
 }
 
+// Chunk-table runs of long adjacency lists (> kLongInline chunk starts) are deferred to a per-CTA list and
+// written by whole warps after the tile (filter_flush_long): with a degree-ordered layout the hubs sit in
+// the first tiles, and one thread writing hundreds of entries serialised the whole filter.
+constexpr int kLongCap = 512;
+constexpr unsigned kLongInline = 2;
+__shared__ unsigned s_long_n;
+__shared__ unsigned s_long_pos[kLongCap], s_long_t0[kLongCap], s_long_t1[kLongCap];
+
 __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, unsigned v, unsigned long long rp,
                                             unsigned long long deg, unsigned long long pos, unsigned long long off) {
     F.q_v[pos] = v;
@@ -210,7 +220,30 @@ __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, u
     F.q_base[pos] = (long long)rp - (long long)off;
     // chunk table: every chunk whose first edge lies in [off, off+deg) starts at queue entry pos
     unsigned long long t = (off + chunk - 1) / chunk;
-    for (; t * chunk < off + deg; t++) F.tile[t] = (unsigned)pos;
+    const unsigned long long t1 = (off + deg + chunk - 1) / chunk;
+    if (t1 - t > kLongInline) {
+        const unsigned i = atomicAdd(&s_long_n, 1u);
+        if (i < (unsigned)kLongCap) {
+            s_long_pos[i] = (unsigned)pos;
+            s_long_t0[i] = (unsigned)t;
+            s_long_t1[i] = (unsigned)t1;
+            return;
+        }
+    }
+    for (; t < t1; t++) F.tile[t] = (unsigned)pos;
+}
+
+// all threads of the CTA: write the deferred chunk-table runs (a warp per run, lanes over its chunks)
+__device__ __forceinline__ void filter_flush_long(const FragPtrs& F) {
+    __syncthreads();
+    const unsigned n = s_long_n < (unsigned)kLongCap ? s_long_n : (unsigned)kLongCap;
+    if (n == 0) return;  // CTA-uniform (read after the barrier; the next append follows another barrier)
+    for (unsigned e = threadIdx.x >> 5; e < n; e += kThreads / 32) {
+        const unsigned pos = s_long_pos[e], t1 = s_long_t1[e];
+        for (unsigned t = s_long_t0[e] + (threadIdx.x & 31); t < t1; t += 32) F.tile[t] = pos;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) s_long_n = 0;
 }
 
 // Dense partitions: 8 warps x 32 bitmap words (8192 vertices); a warp walks its words i-major,
@@ -306,7 +339,7 @@ __device__ __forceinline__ void nf_flush(FragCtl* ct, unsigned fslot, const NfAc
 }
 
 template <int MODE>
-__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsigned tile, bool dense, bool sweep,
+__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool keep_fbm, unsigned tile, bool dense, bool sweep,
                                             bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt, unsigned ipt,
                                             unsigned chunk, unsigned long long pos, unsigned long long off) {
     const unsigned lane = lane_id();
@@ -322,7 +355,10 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, unsig
         }
         if (MODE == FT_EMIT) {
             __syncwarp();
-            if ((lane & 3u) == 0 && wi < nwords && F.bm[wi]) F.bm[wi] = 0u;
+            if ((lane & 3u) == 0 && wi < nwords) {
+                if (keep_fbm) F.far[wi] = word;  // WCC: the frontier as a bitmap for a masked blocked pass
+                if (F.bm[wi]) F.bm[wi] = 0u;
+            }
         }
         const unsigned bits = (word >> ((lane & 3u) * 8u)) & 0xFFu;
         if (bits) {
@@ -444,6 +480,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
             p.b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
         }
         s_pro = p;
+        s_long_n = 0;
     }
     __syncthreads();
     FT_MARK(1);
@@ -453,6 +490,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     const unsigned fslot = s_pro.fslot;
     const bool dense = s_pro.dense != 0;
     const unsigned app_cnt = s_pro.app_cnt;
+    const bool keep_fbm = c.wcc_blocked != 0 && !nf;
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
     // sparse lists: items per thread so that the tiles cover the grid (1..8)
@@ -472,12 +510,22 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     if (b >= G) return;
     const unsigned t_lo = (unsigned)(((unsigned long long)n_tiles * b) / G);
     const unsigned t_hi = (unsigned)(((unsigned long long)n_tiles * (b + 1)) / G);
+    // logical tile t (queue order) -> physical tile (t * stride) mod n_tiles, stride coprime to n_tiles:
+    // a CTA's contiguous logical range is spread over the id space, so activations clustered in one id
+    // range (the DEGREE layout activates vertices of similar in-degree together) do not all land on a
+    // few CTAs. The queue order is then a permutation of vertex order (nothing depends on it being sorted).
+    unsigned stride = 1;
+    if (c.filter_swizzle && n_tiles > 2u * G) {
+        stride = 2053u;  // prime
+        while (stride > 1 && n_tiles % stride == 0) stride += 2;
+        if (stride >= n_tiles) stride = 1;
+    }
 
     // ---- pass 1: aggregate of this CTA's tile range
     Pair mine{0, 0};
     NfAcc nfa;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, keep_fbm, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
         mine.cnt += q.cnt;
         mine.deg += q.deg;
     }
@@ -518,15 +566,18 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
     if (t_hi - t_lo == 1) {
         // one tile: pass 1's per-thread counts are this tile's (same acceptance), no re-count
-        filter_tile<FT_EMIT>(F, nfa, t_lo, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
+        filter_tile<FT_EMIT>(F, nfa, keep_fbm, (unsigned)((unsigned long long)t_lo * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
                              run_deg + tex1.deg);
+        filter_flush_long(F);
     } else {
         for (unsigned t = t_lo; t < t_hi; t++) {
-            const Pair q = filter_tile<FT_COUNT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+            const unsigned pt = (unsigned)((unsigned long long)t * stride % n_tiles);
+            const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
             Pair tot;
             const Pair tex = block_excl_scan(q, s_warp, tot);
-            filter_tile<FT_EMIT>(F, nfa, t, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
+            filter_tile<FT_EMIT>(F, nfa, keep_fbm, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
                                  run_deg + tex.deg);
+            filter_flush_long(F);
             run_cnt += tot.cnt;
             run_deg += tot.deg;
         }
@@ -735,6 +786,29 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         }
         rc->iter = k + 1;
     }
+    if (ALG == ALG_WCC && !done) {
+        // WCC on the blocked static queue: iteration 0 (every vertex active), and later iterations whose
+        // frontier (kept as a bitmap by a dense filter) holds >= 1/2 of the graph's entries: one pass over
+        // the destination-blocked queue with inactive sources masked keeps the label atomics L2-resident,
+        // while the frontier queue would probe a label array larger than L2 at one DRAM sector per edge.
+        // The masked pass still stages every queue entry (C4: ~8 ms fixed + ~4 ms per full frontier vs
+        // ~19 ms per full frontier for the queue path), hence the 1/2 break-even.
+        unsigned blk = rc->skip_filter ? 1u : 0u;
+        if (!blk && c.wcc_blocked && rc->m == (unsigned)c.P) {
+            bool all_dense = true;
+            unsigned long long sq_total = 0;
+            for (int f = 0; f < c.P; f++) {
+                all_dense = all_dense && vload(&c.f[f].ctl->dense) != 0;
+                sq_total += c.f[f].sq_edges;
+            }
+            if (all_dense && total_edges * 2ull >= sq_total) blk = 2u;
+        }
+        rc->blocked = blk;
+        if (blk) {
+            rc->blocked_iters = rc->blocked_iters + 1;
+            rc->tail = 0;
+        }
+    }
     rc->bodies = rc->bodies + 1;
     rc->skip_filter = 0;
     for (int f = 0; f < kMaxW; f++) rc->ticket[f] = 0;
@@ -814,7 +888,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
 
     // Prologue: thread 0 reads the run-control header once per CTA (per-warp loads of these few shared
     // addresses serialise in their L2 slice), threads < P the fragments' queue sizes.
-    __shared__ unsigned s_hdr[6];  // go, m, k, steal_ok, next_dense, pb
+    __shared__ unsigned s_hdr[7];  // go, m, k, steal_ok, next_dense, pb, blocked
     RunCtl* rc = c.rctl[w0];
     const int w = w0 + (int)(blockIdx.x % (unsigned)nw);
     if (threadIdx.x == 0) {
@@ -826,12 +900,21 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         s_hdr[3] = vload(&rc->steal_ok);
         s_hdr[4] = vload(&rc->next_dense);
         s_hdr[5] = (ALG == ALG_BFS && !MULTI && PB) ? vload(&rc->pb) : 0u;
+        s_hdr[6] = (ALG == ALG_WCC) ? vload(&rc->blocked) : 0u;
     }
     if (threadIdx.x < (unsigned)c.P) {
         FragCtl* ct = c.f[threadIdx.x].ctl;
-        s_ntiles[threadIdx.x] = vload(&ct->ntiles);
-        s_qlen[threadIdx.x] = vload(&ct->qlen);
-        s_qedges[threadIdx.x] = vload(&ct->qedges);
+        const FragPtrs& Fq = c.f[threadIdx.x];
+        if (ALG == ALG_WCC && Fq.sq_col && vload(&rc->blocked)) {
+            // the static destination-blocked queue (all vertices; inactive ones are masked in staging)
+            s_ntiles[threadIdx.x] = (Fq.sq_edges + c.chunk - 1) / c.chunk;
+            s_qlen[threadIdx.x] = Fq.sq_len;
+            s_qedges[threadIdx.x] = Fq.sq_edges;
+        } else {
+            s_ntiles[threadIdx.x] = vload(&ct->ntiles);
+            s_qlen[threadIdx.x] = vload(&ct->qlen);
+            s_qedges[threadIdx.x] = vload(&ct->qedges);
+        }
         s_owner[threadIdx.x] = vload(&rc->owner[threadIdx.x]);
         s_cnt[threadIdx.x][0] = s_cnt[threadIdx.x][1] = s_cnt[threadIdx.x][2] = s_cnt[threadIdx.x][3] = 0;
     }
@@ -839,6 +922,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     if (!s_hdr[0]) return;
     const unsigned m = s_hdr[1];
     const unsigned k = s_hdr[2];
+    const unsigned blk = ALG == ALG_WCC ? s_hdr[6] : 0u;  // 2: masked blocked pass (count valid edges)
     const bool steal = s_hdr[3] != 0;
     const bool next_dense = s_hdr[4] != 0;
     const bool planned = c.fsteal == 2 && m == (unsigned)c.P;  // NEXT-2 plan (else the steal queue)
@@ -853,6 +937,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0, filtered = 0, hub_e = 0;
+    unsigned nval = 0;  // masked blocked pass: this thread's expanded edges of the current chunk
     // NEXT-1 outer-vertex mirrors (this worker's memory): updates to other fragments go through them
     const bool mir = MULTI && c.mirrors;
 
@@ -947,7 +1032,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         if (f < 0) return r;
         r.hc = MULTI && ALG != ALG_PR && c.hub_on && f != w;
         const FragPtrs& F = c.f[f];
-        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned* const tilep = sq ? F.sq_tile : F.tile;
         const unsigned long long tb = t * CH, qe = s_qedges[f];
         r.tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
@@ -960,7 +1045,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     auto stage_load = [&](const ChunkRef& r, unsigned kk, unsigned long long& off, unsigned& base, unsigned& u,
                           bool& hub) {
         const FragPtrs& F = c.f[r.f];
-        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned i = r.i0 + kk;
         const unsigned long long tb = r.t * CH;
         off = __ldcs((sq ? F.sq_q_off : F.q_off) + i);
@@ -981,6 +1066,9 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     };
     auto value_of = [&](const ChunkRef& r, unsigned u) -> VT {
         if (ALG == ALG_PR) return (VT)__ldcg(c.f[r.f].cx + u);
+        // masked blocked pass: a source outside the frontier (its bit clear in the filter's copy) gets the
+        // value INF, and its edges are skipped in the expansion
+        if (ALG == ALG_WCC && blk == 2 && !((__ldcg(c.f[r.f].far + (u >> 5)) >> (u & 31)) & 1u)) return (VT)GUM_INF;
         if (ALG != ALG_BFS) return (VT)__ldcg(c.f[r.f].state + u);
         return (VT)0;
     };
@@ -1016,7 +1104,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         const FragPtrs& F = c.f[f];
         const unsigned long long tb = t * CH;
         const unsigned tlen = cur.tlen;
-        const bool sq = ALG == ALG_WCC && k == 0 && F.sq_col != nullptr;
+        const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned* const colp = sq ? F.sq_col : F.col;
         const unsigned nv = cur.nv;
         if (threadIdx.x == 0) {
@@ -1116,6 +1204,10 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
             cv[j] = (VT)0;
             if (e < tlen) {
                 const unsigned kk = s_head[e];
+                if (ALG == ALG_WCC && blk == 2) {
+                    if (s_val[kk] == (VT)GUM_INF) continue;  // source not in the frontier
+                    nval++;
+                }
                 const unsigned long long ci = (unsigned)(s_base[kk] + e);  // mod 2^32: the base may wrap
                 const bool hv = MULTI && cur.hc && s_hub[kk];
                 if (MULTI) hub_e += hv ? 1 : 0;
@@ -1346,7 +1438,24 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                 acts += append_activations<MULTI>(c, need, tfv, lvv);
             }
         }
-        if (threadIdx.x == 0) {
+        if (ALG == ALG_WCC && blk == 2) {
+            // masked pass: only the frontier's edges count as expanded (conservation, SURVEY c-6)
+            const unsigned long long ws = warp_sum_u64(nval);
+            nval = 0;
+            if (lane_id() == 0 && ws) {
+                atomicAdd(&s_cnt[f][0], ws);
+                if (stolen) {
+                    atomicAdd(&s_cnt[f][2], ws);
+                    e_stolen += ws;
+                } else {
+                    e_own += ws;
+                }
+            }
+            if (threadIdx.x == 0) {
+                s_cnt[f][1] += 1;
+                if (stolen) s_cnt[f][3] += 1;
+            }
+        } else if (threadIdx.x == 0) {
             // conservation counters of the chunk's fragment, accumulated per CTA (flushed at exit: the
             // fragment counters are single addresses)
             s_cnt[f][0] += tlen;
@@ -1389,11 +1498,14 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         if (hub_e) atomicAdd(&hc->hub_edges, hub_e);
     }
     gum_iter_trace* tr = c.trace[w0];
-    if (tr && threadIdx.x == 0 && k < (unsigned)kTraceMax) {
-        const unsigned long long t1 = globaltimer();
+    if (tr && k < (unsigned)kTraceMax) {
         gum_iter_trace* r = tr + k;
-        atomicMin((unsigned long long*)&r->t_start[w], t0);
-        atomicMax((unsigned long long*)&r->t_end[w], t1);
+        if (threadIdx.x == 0) {
+            const unsigned long long t1 = globaltimer();
+            atomicMin((unsigned long long*)&r->t_start[w], t0);
+            atomicMax((unsigned long long*)&r->t_end[w], t1);
+        }
+        // (thread 0 holds the per-chunk counts; in a masked WCC pass every warp's lane 0 holds a share)
         if (e_own) atomicAdd((unsigned long long*)&r->edges_own[w], e_own);
         if (e_stolen) atomicAdd((unsigned long long*)&r->edges_stolen[w], e_stolen);
     }

@@ -413,6 +413,10 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
     d.pb_nb = c->pb_nb;
     d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
+    static const int env_sw = getenv("GUM_FILTER_SWIZZLE") ? atoi(getenv("GUM_FILTER_SWIZZLE")) : 1;
+    d.filter_swizzle = env_sw ? 1u : 0u;
+    static const int env_wb = getenv("GUM_WCC_BLOCKED") ? atoi(getenv("GUM_WCC_BLOCKED")) : 1;
+    d.wcc_blocked = (alg == GUM_WCC && c->fr[0].sq_col && c->cfg.fsteal != 2 && env_wb) ? 1u : 0u;
     for (int f = 0; f < c->P; f++) d.total_edges += c->fr[f].E;
     return d;
 }
@@ -1637,6 +1641,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         stats->osteal_iteration = R.osteal_iter;
         stats->pr_last_residual = R.pr_resid;
         stats->tail_iterations = R.tail_iters;
+        stats->blocked_iterations = R.blocked_iters;
         stats->bodies = R.bodies;
         stats->kernel_launches = c->launches;
         if (graph_mode) {

@@ -112,6 +112,24 @@ __global__ void k_new_deg(const unsigned long long* rp, const unsigned* inv, uns
     }
 }
 
+// rows of <= kShortRow entries: one thread per row (a warp per row would leave most lanes idle and
+// serialise the row's dependent loads); longer rows: one warp per row
+constexpr unsigned long long kShortRow = 32;
+__global__ void k_relabel_short(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
+                                unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
+                                unsigned* ncol, unsigned* nw) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x) {
+        const unsigned long long d0 = nrp[v], n = nrp[v + 1] - d0;
+        if (n == 0 || n > kShortRow) continue;
+        const unsigned long long s0 = rp[inv[v]];
+        for (unsigned long long j = 0; j < n; j++) {
+            const unsigned x = col[s0 + j];
+            ncol[d0 + j] = perm ? perm[x] : feistel(x, V, seed);
+            if (w) nw[d0 + j] = w[s0 + j];
+        }
+    }
+}
+
 __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
                                unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
                                unsigned* ncol, unsigned* nw) {
@@ -119,8 +137,10 @@ __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col
     const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
     const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
     for (unsigned long long v = warp; v < V; v += nwarps) {
+        const unsigned long long d0 = nrp[v];
+        if (nrp[v + 1] - d0 <= kShortRow) continue;  // k_relabel_short moved it
         const unsigned o = inv[v];
-        const unsigned long long s0 = rp[o], s1 = rp[o + 1], d0 = nrp[v];
+        const unsigned long long s0 = rp[o], s1 = rp[o + 1];
         for (unsigned long long j = lane; j < s1 - s0; j += 32) {
             ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
             if (w) nw[d0 + j] = w[s0 + j];
@@ -136,6 +156,7 @@ cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col
     k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
     cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
     if (e != cudaSuccess) return e;
+    k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
     k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
     return cudaGetLastError();
 }
@@ -185,6 +206,7 @@ cudaError_t setup_relabel_degree(const unsigned long long* row_ptr, const unsign
     k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
     e = cub::DeviceScan::ExclusiveSum(t, tb, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
     if (e != cudaSuccess) return e;
+    k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
     k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
     return cudaGetLastError();
 }

@@ -300,8 +300,16 @@ def test_wcc_blocked_first_iteration(monkeypatch, P):
     g = inputs.rmat(14, 8, seed=91, weighted=False)
     ref = oracle.run("wcc", g)
     csr = csr_of(g)
-    for kw in (dict(), dict(part="random", seed=2), dict(tail_vertices=0), dict(split_units=P > 1)):
-        check(g, "wcc", 0, csr=csr, ref=ref, num_gpus=P, **kw)
+    blocked = []
+    for kw in (dict(), dict(part="random", seed=2), dict(tail_vertices=0), dict(split_units=P > 1),
+               dict(force_mode="dense", tail_vertices=0), dict(host_loop=True, trace=True, tail_vertices=0)):
+        _, st, tr = check(g, "wcc", 0, csr=csr, ref=ref, num_gpus=P, **kw)
+        blocked.append(st.blocked_iterations)
+        if tr is not None:  # per-iteration conservation holds in masked blocked passes too
+            for r in tr:
+                assert sum(r["edges_own"]) + sum(r["edges_stolen"]) == r["frontier_edges"]
+    # later dense iterations also ran on the blocked queue (sources masked by the frontier bitmap)
+    assert max(blocked) >= 2, blocked
 
 
 @pytest.mark.parametrize("alg", ALGS)
