@@ -27,6 +27,7 @@ constexpr int kFilterAppPerThread = 8;                            // sparse filt
 constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;
 constexpr int kPbMaxBins = 1024;       // propagation blocking: max destination blocks per fragment
+constexpr unsigned kPrPiece = 64;      // PR warp-task path: max edges per queue entry
 
 // Per-fragment control block (fragment memory, peer-visible). Counters that thieves touch
 // (claim) and that the filter publishes (qlen, qedges, ntiles) live here.
@@ -140,6 +141,10 @@ struct FragPtrs {
     unsigned int base;                  // global id of local vertex 0
     unsigned long long E;
     unsigned long long pr_qlen, pr_qedges;  // PR's static destination-blocked queue (gum_prepare)
+    // PR single fragment: the same queue with entries cut to <= kPrPiece edges, expanded by k_pr_push
+    const unsigned int* pr2_q_v;
+    const unsigned long long* pr2_q_off;  // [pr2_len + 1]; col index of edge j of entry i = q_off[i] + j
+    unsigned long long pr2_len;
     // WCC: static destination-blocked queue of the symmetric graph for iteration 0 (all vertices active)
     const unsigned int* sq_col;
     const unsigned int* sq_q_v;

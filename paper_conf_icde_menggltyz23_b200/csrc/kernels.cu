@@ -1609,6 +1609,78 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
     return acts;
 }
 
+// Phase-1 variant: the warp holds kTailVPW listed vertices at once, kTailG lanes each (gl = lane in the
+// group); every group walks its own vertex's edges [s0, s1) kTailG at a time. Low-degree frontiers (road-like
+// grids: out-degree <= 4) would otherwise leave 28 of 32 lanes idle and serialise one vertex's dependent
+// loads per warp. Appends keep the warp-aggregated reservation of tail_expand.
+constexpr unsigned kTailG = 8;
+constexpr unsigned kTailVPW = 32 / kTailG;
+template <int ALG, bool MULTI>
+__device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtrs& F, bool go, unsigned sval,
+                                                  unsigned long long s0, unsigned long long s1, unsigned k,
+                                                  unsigned it, unsigned ns, unsigned gl) {
+    const unsigned lane = lane_id();
+    unsigned acts = 0;
+    const unsigned long long d = go ? s1 - s0 : 0ull;
+    const unsigned rounds = __reduce_max_sync(0xffffffffu, (unsigned)((d + kTailG - 1) / kTailG));
+    for (unsigned r = 0; r < rounds; r++) {
+        const unsigned long long e = s0 + (unsigned long long)r * kTailG + gl;
+        bool need = false;
+        int tf = 0;
+        unsigned lu = 0;
+        if (go && e < s1) {
+            const unsigned u = __ldg(F.col + e);
+            tf = MULTI ? frag_of(c, u) : 0;
+            lu = MULTI ? u - c.bounds[tf] : u;
+            const FragPtrs& T = c.f[tf];
+            const unsigned bit = 1u << (lu & 31);
+            if (ALG == ALG_BFS) {
+                if (!(vload(T.vis + (lu >> 5)) & bit)) {
+                    const unsigned ob = atomicOr(T.vis + (lu >> 5), bit);
+                    if (!(ob & bit)) {
+                        T.state[lu] = k + 1;
+                        need = true;
+                    }
+                }
+            } else {
+                unsigned cand = sval;
+                bool ok = true;
+                if (ALG == ALG_SSSP) {
+                    const unsigned long long nd = (unsigned long long)sval + __ldg(F.w + e);
+                    if (nd >= (unsigned long long)GUM_INF) {
+                        atomicOr(&F.ctl->err, 1u);
+                        ok = false;
+                    }
+                    cand = (unsigned)nd;
+                }
+                if (ok && cand < vload(T.state + lu)) {
+                    atomicMin(T.state + lu, cand);
+                    const unsigned ob = atomicOr(((it & 1) ? T.bm2 : T.bm) + (lu >> 5), bit);
+                    need = !(ob & bit);
+                }
+            }
+        }
+        const unsigned key = need ? (unsigned)tf : 0xFFFFFFFFu;
+        const unsigned grp = MULTI ? __match_any_sync(0xffffffffu, key) : __ballot_sync(0xffffffffu, need);
+        if (need) {
+            const FragPtrs& T = c.f[tf];
+            const unsigned leader = __ffs(grp) - 1;
+            unsigned base = 0;
+            if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
+            base = __shfl_sync(grp, base, leader);
+            unsigned* nxt = (it & 1) ? T.q_v : T.app;
+            nxt[base + __popc(grp & lanemask_lt())] = lu;
+            acts++;
+        }
+        const unsigned long long deg = need ? __ldg(c.f[tf].row_ptr + lu + 1) - __ldg(c.f[tf].row_ptr + lu) : 0ull;
+        if (need) {
+            const unsigned hi = __reduce_add_sync(grp, (unsigned)(deg >> 16)), lo = __reduce_add_sync(grp, (unsigned)(deg & 0xFFFFu));
+            if (lane == __ffs(grp) - 1) atomicAdd(&c.f[tf].ctl->tedges[ns], ((unsigned long long)hi << 16) + lo);
+        }
+    }
+    return acts;
+}
+
 template <int ALG, bool MULTI>
 __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
     __shared__ unsigned s_n[kMaxW], s_nsplit, s_go;
@@ -1650,20 +1722,25 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         if (threadIdx.x < (unsigned)nfrag)
             s_n[threadIdx.x] = it == 0 ? (unsigned)vload(&c.f[threadIdx.x].ctl->qlen) : vload(&c.f[threadIdx.x].ctl->tcnt[cs]);
         __syncthreads();
-        // ---- phase 1: one warp per listed vertex; high-degree vertices go to the split list
+        // ---- phase 1: kTailG lanes per listed vertex (kTailVPW vertices per warp); high-degree vertices
+        // go to the split list
+        const unsigned sub = lane / kTailG, gl = lane % kTailG, src = sub * kTailG;
         for (int f = 0; f < nfrag; f++) {
             const FragPtrs& F = c.f[f];
             const unsigned* cur = (it & 1) ? F.app : F.q_v;
             const unsigned n = s_n[f];
             n_all += n;
             if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
-            for (unsigned i = gw; i < n; i += nwarps) {
-                const unsigned v = cur[i];
-                const unsigned long long s0 = __ldg(F.row_ptr + v), s1 = __ldg(F.row_ptr + v + 1);
+            for (unsigned i0 = gw * kTailVPW; i0 < n; i0 += nwarps * kTailVPW) {  // warp-uniform trip count
+                const unsigned i = i0 + sub;
+                const bool have = i < n;
+                const unsigned v = have ? cur[i] : 0u;
+                const unsigned long long s0 = have ? __ldg(F.row_ptr + v) : 0ull;
+                const unsigned long long s1 = have ? __ldg(F.row_ptr + v + 1) : 0ull;
                 unsigned sval = (ALG == ALG_BFS) ? k : 0u;
                 unsigned slot = 0xFFFFFFFFu;
-                bool park = false;
-                if (lane == 0) {
+                bool park = !have;
+                if (have && gl == 0) {
                     if (ALG != ALG_BFS) {
                         // release the cur list's dedupe bit (reused two iterations later); any
                         // improvement of v from now on appends it to the NEXT list (other parity)
@@ -1692,15 +1769,15 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                         }
                     }
                 }
-                park = __shfl_sync(0xffffffffu, park ? 1u : 0u, 0) != 0;
-                if (park) continue;
-                slot = __shfl_sync(0xffffffffu, slot, 0);
-                if (slot < kTailSplitCap) continue;  // expanded cooperatively in phase 2
-                sval = __shfl_sync(0xffffffffu, sval, 0);
-                a_sum += tail_expand<ALG, MULTI>(c, F, sval, s0, s1, k, it, ns);
+                park = __shfl_sync(0xffffffffu, park ? 1u : 0u, src) != 0;
+                slot = __shfl_sync(0xffffffffu, slot, src);
+                sval = __shfl_sync(0xffffffffu, sval, src);
+                // split vertices are expanded cooperatively in phase 2
+                a_sum += tail_expand_g<ALG, MULTI>(c, F, !park && slot >= kTailSplitCap, sval, s0, s1, k, it, ns, gl);
             }
         }
         if (tr && k < (unsigned)kTraceMax) {
+            it_edges = warp_sum_u64(it_edges);  // (group leaders hold the counts)
             if (lane == 0 && it_edges) {
                 if (it > 0) atomicAdd((unsigned long long*)&tr[k].frontier_edges, it_edges);
                 atomicAdd((unsigned long long*)&tr[k].edges_own[0], it_edges);  // the tail's single owner
@@ -1781,6 +1858,8 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
             break;
     }
     for (int f = 0; f < nfrag; f++) {
+        e_done[f] = warp_sum_u64(e_done[f]);  // group leaders (lanes 0, kTailG, ...) hold the counts
+        e_front[f] = warp_sum_u64(e_front[f]);
         if (lane == 0 && e_done[f]) {
             atomicAdd(&c.f[f].ctl->edges_done, e_done[f]);
             if (e_front[f]) atomicAdd(&c.f[f].ctl->frontier_edges, e_front[f]);
@@ -1989,6 +2068,97 @@ __global__ void __launch_bounds__(kThreads) k_pb_apply(const __grid_constant__ D
     }
 }
 
+// ------------------------------------------------------------------------------------------ PR push (P = 1)
+// The advance of PR's static frontier on one fragment, without CTA barriers: the destination-blocked queue
+// is cut at gum_prepare into entries of <= kPrPiece edges, and each warp task takes 32 consecutive entries
+// (one per lane: x/outdeg of its source, its col range), scans their lengths with shuffles and walks the
+// task's edges 32 at a time -- a warp-level merge path: lane e finds its entry by a 5-step shuffle binary
+// search over the lanes' prefixes, loads col (consecutive edges are consecutive in the blocked col array,
+// so every round is one coalesced 128-byte load) and issues red.add.f64 of the entry's value into acc.
+// The CTA-level merge path of k_advance spends ~27% of its stalls on the per-chunk barriers here (the PR
+// push has only 8 edges of work per thread per chunk); warps here are independent. Same sums as k_advance.
+// Measured on C5 (opt-in, GUM_PR_PUSH=1): 12.0 ms per iteration vs 10.8 ms for k_advance -- the 8 dependent
+// shuffles per 32 edges make it MIO-bound (short_sb 33% + mio 17% of stalls); a static task split was
+// worse still (19.1 ms: warps drifted over several acc blocks and thrashed L2).
+__global__ void __launch_bounds__(kThreads) k_pr_push(const __grid_constant__ DevCtx c, int w0, int nw) {
+    RunCtl* rc = c.rctl[w0];
+    __shared__ unsigned s_go;
+    if (threadIdx.x == 0) s_go = !vload(&rc->done) && (unsigned)w0 < vload(&rc->m);
+    __syncthreads();
+    if (!s_go) return;
+    const unsigned long long t0 = globaltimer();
+    const FragPtrs& F = c.f[0];
+    const unsigned lane = lane_id();
+    const unsigned long long n = F.pr2_len;
+    const unsigned long long tasks = (n + 31) / 32;
+    unsigned long long edges = 0;
+    // dynamic claims of kPrClaim tasks (one atomic per ~1K edges): every warp works in the same narrow
+    // window of the destination-blocked queue, so only the current acc block is live in L2 (a static
+    // task split let warps drift over several blocks and thrash L2: 7.5 GB of acc write-backs per launch)
+    constexpr unsigned kPrClaim = 4;
+    unsigned long long nxt = 0;
+    if (lane == 0) nxt = atomicAdd(&F.ctl->claim, (unsigned long long)kPrClaim);
+    nxt = __shfl_sync(0xffffffffu, nxt, 0);
+    for (;;) {
+        const unsigned long long cl = nxt;
+        if (cl >= tasks) break;
+        if (lane == 0) nxt = atomicAdd(&F.ctl->claim, (unsigned long long)kPrClaim);  // one claim ahead
+        nxt = __shfl_sync(0xffffffffu, nxt, 0);
+        const unsigned long long tend = cl + kPrClaim < tasks ? cl + kPrClaim : tasks;
+    for (unsigned long long task = cl; task < tend; task++) {
+        const unsigned long long i = task * 32 + lane;
+        unsigned long long off = 0, len = 0;
+        double val = 0.0;
+        if (i < n) {
+            off = __ldcs(F.pr2_q_off + i);
+            len = __ldcs(F.pr2_q_off + i + 1) - off;
+            val = __ldcg(F.cx + __ldcs(F.pr2_q_v + i));
+        }
+        // inclusive prefix of the entry lengths over the lanes (len <= kPrPiece: 32-bit sums)
+        unsigned inc = (unsigned)len;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned x = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= (unsigned)o) inc += x;
+        }
+        const unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
+        const unsigned excl = inc - (unsigned)len;
+        for (unsigned b = 0; b < tot; b += 32) {
+            const unsigned e = b + lane;
+            // entry of edge e: the last lane j with excl_j <= e (lanes with len 0 share their successor's
+            // excl and are never selected past it: the search takes the largest such j)
+            unsigned j = 0;
+#pragma unroll
+            for (unsigned step = 16; step > 0; step >>= 1) {
+                const unsigned x = __shfl_sync(0xffffffffu, excl, j + step);
+                if (x <= e) j += step;
+            }
+            const unsigned long long oj = __shfl_sync(0xffffffffu, off, j);
+            const double vj = __shfl_sync(0xffffffffu, val, j);
+            const unsigned ej = __shfl_sync(0xffffffffu, excl, j);
+            if (e < tot) {
+                const unsigned v = __ldcs(F.col + oj + (e - ej));
+                atomicAdd(F.acc + v, vj);  // RED.ADD.F64
+            }
+        }
+        edges += tot;
+    }
+    }
+    // conservation counters (lane 0 holds the per-task totals) and the worker's busy window
+    if (lane == 0 && edges) atomicAdd(&F.ctl->edges_done, edges);
+    gum_iter_trace* tr = c.trace[w0];
+    const unsigned k = vload(&rc->iter) - 1;
+    if (tr && threadIdx.x == 0 && k < (unsigned)kTraceMax) {
+        atomicMin((unsigned long long*)&tr[k].t_start[0], t0);
+        atomicMax((unsigned long long*)&tr[k].t_end[0], globaltimer());
+    }
+    if (tr && lane == 0 && edges && k < (unsigned)kTraceMax) atomicAdd((unsigned long long*)&tr[k].edges_own[0], edges);
+}
+
+cudaError_t pr_push_occupancy(int* blocks_per_sm) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_pr_push, kThreads, 0);
+}
+
 // ------------------------------------------------------------------------------------------ PR finalize
 __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
@@ -2085,7 +2255,9 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
         case KER_FILTER: k_filter<<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
         case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
         case KER_ADVANCE:
-            if (c.P > 1)
+            if (ALG == ALG_PR && c.P == 1 && c.f[0].pr2_q_v)
+                k_pr_push<<<L.adv_grid_pr, kThreads, 0, s>>>(c, L.w0, L.nw);
+            else if (c.P > 1)
                 k_advance<ALG, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             else
                 if (ALG == ALG_BFS && c.pb_shift)

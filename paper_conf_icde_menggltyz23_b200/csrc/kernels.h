@@ -16,6 +16,7 @@ struct LaunchCfg {
     int fin_grid;     // PR finalize CTAs per fragment
     int init_grid;
     int tail_grid;    // tail engine CTAs (cooperative; 0 = engine disabled)
+    int adv_grid_pr;  // PR warp-task push (single fragment): occupancy-sized grid
 };
 
 enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_APPLY = 6, KER_PULL = 7, KER_COUNT = 8 };
@@ -32,6 +33,14 @@ cudaError_t launch_mp_barrier(const MpPads& p, int P, int me, unsigned long long
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
 cudaError_t filter_occupancy(int* blocks_per_sm);
+cudaError_t pr_push_occupancy(int* blocks_per_sm);
+// PR single fragment: cut the destination-blocked queue's entries into pieces of <= piece edges
+// (q2_off gets n2 + 1 entries; *n2 = pieces). tmp sized by setup_scan_tmp_bytes(n).
+cudaError_t setup_pr_pieces_count(const unsigned long long* q_off, unsigned long long n, unsigned piece,
+                                  unsigned long long* cnt, void* tmp, size_t tmp_bytes, cudaStream_t s);
+cudaError_t setup_pr_pieces_emit(const unsigned* q_v, const unsigned long long* q_off, unsigned long long n,
+                                 unsigned piece, const unsigned long long* pos, unsigned* q2_v,
+                                 unsigned long long* q2_off, cudaStream_t s);
 // BFS propagation blocking: static per-block capacities (in-degree histogram of the blocks) -> pb_off
 cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,
                              unsigned long long* pb_off, void* tmp, size_t tmp_bytes, cudaStream_t s);

@@ -64,6 +64,9 @@ struct FragBufs {
     unsigned long long* pr_q_off = nullptr;
     unsigned* pr_tile = nullptr;
     unsigned long long pr_qlen = 0, pr_qedges = 0;
+    unsigned* pr2_q_v = nullptr;             // PR single fragment: pieces of <= kPrPiece edges (k_pr_push)
+    unsigned long long* pr2_q_off = nullptr;
+    unsigned long long pr2_len = 0;
     // WCC iteration-0 static destination-blocked queue over the symmetric graph
     unsigned* sq_col = nullptr;
     unsigned* sq_q_v = nullptr;
@@ -103,6 +106,7 @@ struct gum_ctx {
     int tail_occ = 1;
     int filter_occ = 2;
     int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
+    int pr_push_occ = 8;
     std::string err;
     bool poisoned = false;
     std::vector<Alloc> load_allocs, part_allocs, misc_allocs;
@@ -310,6 +314,7 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.tail_grid = (c->n_units == 1 && c->cfg.tail_vertices && alg != GUM_PR) ? c->nsm * c->tail_occ : 0;
+    L.adv_grid_pr = c->nsm * c->pr_push_occ;
     return L;
 }
 
@@ -365,6 +370,9 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
             p.tile = F.pr_tile;
             p.pr_qlen = F.pr_qlen;
             p.pr_qedges = F.pr_qedges;
+            p.pr2_q_v = F.pr2_q_v;
+            p.pr2_q_off = F.pr2_q_off;
+            p.pr2_len = F.pr2_len;
         }
         p.ctl = F.ctl;
         p.V = F.V;
@@ -823,6 +831,36 @@ gum_status build_pr(gum_ctx* c) {
         if (e != cudaSuccess) return fail(c, GUM_ECUDA, "PR blocked queue: %s", cudaGetErrorString(e));
         F.pr_qlen = Q;
         F.pr_qedges = F.E;
+        // opt-in (measured slower on C5: 12.0 vs 10.8 ms per iteration, the shuffle search is MIO-bound)
+        static const int env_pp = getenv("GUM_PR_PUSH") ? atoi(getenv("GUM_PR_PUSH")) : 0;
+        if (c->P == 1 && env_pp) {
+            // single fragment: the warp-task push (k_pr_push) runs on the same queue cut into pieces
+            std::vector<Alloc> t3;
+            unsigned long long* pos = (unsigned long long*)dalloc(c, F.dev, (Q + 1) * 8, t3);
+            const size_t tb3 = setup_scan_tmp_bytes((unsigned)std::min<unsigned long long>(Q, 0xFFFFFFF0ull));
+            void* tt = dalloc(c, F.dev, tb3 + (Q > 0xFFFFFFF0ull ? 0 : 0), t3);
+            if (!pos || !tt) {
+                free_list(c, t3);
+                return fail(c, GUM_ENOMEM, "PR pieces alloc failed");
+            }
+            unsigned long long n2 = 0;
+            cudaError_t e3 = setup_pr_pieces_count(F.pr_q_off, Q, kPrPiece, pos, tt, tb3, s);
+            if (e3 == cudaSuccess) e3 = cudaMemcpyAsync(&n2, pos + Q, 8, cudaMemcpyDeviceToHost, s);
+            if (e3 == cudaSuccess) e3 = cudaStreamSynchronize(s);
+            if (e3 == cudaSuccess) {
+                F.pr2_q_v = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(n2, 1) * 4, c->part_allocs);
+                F.pr2_q_off = (unsigned long long*)dalloc(c, F.dev, (n2 + 1) * 8, c->part_allocs);
+                if (!F.pr2_q_v || !F.pr2_q_off) {
+                    free_list(c, t3);
+                    return fail(c, GUM_ENOMEM, "PR pieces alloc failed (%llu pieces)", n2);
+                }
+                e3 = setup_pr_pieces_emit(F.pr_q_v, F.pr_q_off, Q, kPrPiece, pos, F.pr2_q_v, F.pr2_q_off, s);
+                if (e3 == cudaSuccess) e3 = cudaStreamSynchronize(s);
+            }
+            free_list(c, t3);
+            if (e3 != cudaSuccess) return fail(c, GUM_ECUDA, "PR pieces: %s", cudaGetErrorString(e3));
+            F.pr2_len = n2;
+        }
     }
     CK(cudaSetDevice(c->dev[0]));
     c->pr_ready = true;
@@ -974,6 +1012,7 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     if (cfg->num_gpus < 1 || cfg->num_gpus > kMaxW) return GUM_EINVAL;
     gum_ctx* c = new gum_ctx();
     c->cfg = *cfg;
+    if (const char* e = getenv("GUM_CHUNK")) c->cfg.chunk_edges = (uint32_t)atoi(e);  // tuning override
     if (c->cfg.chunk_edges == 0 || c->cfg.chunk_edges > (unsigned)kTileMax) c->cfg.chunk_edges = kTileMax;
     if (c->cfg.chunk_edges % 32 != 0) {
         delete c;
@@ -1060,6 +1099,9 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
         cudaGetLastError();
         occ = 0;
         if (filter_occupancy(&occ) == cudaSuccess && occ > 0) c->filter_occ = std::min(occ, 4);
+        occ = 0;
+        if (pr_push_occupancy(&occ) == cudaSuccess && occ > 0) c->pr_push_occ = occ;
+        if (const char* e = getenv("GUM_PR_PUSH_CTAS_PER_SM")) c->pr_push_occ = std::max(1, atoi(e));
         cudaGetLastError();
     }
     cudaEventCreate(&c->ev0);

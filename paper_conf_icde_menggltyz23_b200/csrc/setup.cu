@@ -130,6 +130,7 @@ __global__ void k_relabel_short(const unsigned long long* rp, const unsigned* co
     }
 }
 
+constexpr unsigned long long kHugeRow = 4096;  // rows longer than this: one CTA per row (k_relabel_huge)
 __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
                                unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
                                unsigned* ncol, unsigned* nw) {
@@ -137,14 +138,38 @@ __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col
     const unsigned long long warp = (blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x) >> 5;
     const unsigned long long nwarps = ((unsigned long long)gridDim.x * blockDim.x) >> 5;
     for (unsigned long long v = warp; v < V; v += nwarps) {
-        const unsigned long long d0 = nrp[v];
-        if (nrp[v + 1] - d0 <= kShortRow) continue;  // k_relabel_short moved it
-        const unsigned o = inv[v];
-        const unsigned long long s0 = rp[o], s1 = rp[o + 1];
-        for (unsigned long long j = lane; j < s1 - s0; j += 32) {
+        const unsigned long long d0 = nrp[v], n = nrp[v + 1] - d0;
+        if (n <= kShortRow || n > kHugeRow) continue;  // k_relabel_short / k_relabel_huge move those
+        const unsigned long long s0 = rp[inv[v]];
+        for (unsigned long long j = lane; j < n; j += 32) {
             ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
             if (w) nw[d0 + j] = w[s0 + j];
         }
+    }
+}
+
+// hub rows (the highest-degree rows hold up to ~0.15% of all edges each on RMAT): the whole CTA per row
+__global__ void k_relabel_huge(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
+                               unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
+                               unsigned* ncol, unsigned* nw) {
+    __shared__ unsigned s_rows[256];
+    __shared__ unsigned s_n;
+    for (unsigned long long b = (unsigned long long)blockIdx.x * blockDim.x; b < V;
+         b += (unsigned long long)gridDim.x * blockDim.x) {
+        if (threadIdx.x == 0) s_n = 0;
+        __syncthreads();
+        const unsigned long long v = b + threadIdx.x;
+        if (v < V && nrp[v + 1] - nrp[v] > kHugeRow) s_rows[atomicAdd(&s_n, 1u)] = (unsigned)v;
+        __syncthreads();
+        for (unsigned r = 0; r < s_n; r++) {
+            const unsigned hv = s_rows[r];
+            const unsigned long long d0 = nrp[hv], n = nrp[hv + 1] - d0, s0 = rp[inv[hv]];
+            for (unsigned long long j = threadIdx.x; j < n; j += blockDim.x) {
+                ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
+                if (w) nw[d0 + j] = w[s0 + j];
+            }
+        }
+        __syncthreads();
     }
 }
 
@@ -158,6 +183,7 @@ cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col
     if (e != cudaSuccess) return e;
     k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
     k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
+    k_relabel_huge<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
     return cudaGetLastError();
 }
 
@@ -208,6 +234,7 @@ cudaError_t setup_relabel_degree(const unsigned long long* row_ptr, const unsign
     if (e != cudaSuccess) return e;
     k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
     k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
+    k_relabel_huge<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
     return cudaGetLastError();
 }
 
@@ -507,6 +534,44 @@ cudaError_t setup_hub_fill(const unsigned long long* row_ptr, const unsigned* co
                            unsigned n, unsigned t4, unsigned long long* off, unsigned* hcol, unsigned* hw,
                            cudaStream_t s) {
     k_hub_fill<<<1184, 256, 0, s>>>(row_ptr, col, w, b0, n, t4, off, hcol, hw);
+    return cudaGetLastError();
+}
+
+// PR pieces: entry i (edges [q_off[i], q_off[i+1])) becomes ceil(len / piece) entries of <= piece edges
+__global__ void k_pr_piece_cnt(const unsigned long long* q_off, unsigned long long n, unsigned piece,
+                               unsigned long long* cnt) {
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i <= n;
+         i += (unsigned long long)gridDim.x * blockDim.x)
+        cnt[i] = i < n ? (q_off[i + 1] - q_off[i] + piece - 1) / piece : 0ull;
+}
+__global__ void k_pr_piece_emit(const unsigned* q_v, const unsigned long long* q_off, unsigned long long n,
+                                unsigned piece, const unsigned long long* pos, unsigned* q2_v,
+                                unsigned long long* q2_off) {
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i <= n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+        if (i == n) {
+            q2_off[pos[n]] = q_off[n];
+            continue;
+        }
+        const unsigned long long a = q_off[i], b = q_off[i + 1], p0 = pos[i];
+        const unsigned v = q_v[i];
+        for (unsigned long long k = 0; a + k * piece < b; k++) {
+            q2_v[p0 + k] = v;
+            q2_off[p0 + k] = a + k * piece;
+        }
+    }
+}
+cudaError_t setup_pr_pieces_count(const unsigned long long* q_off, unsigned long long n, unsigned piece,
+                                  unsigned long long* cnt, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    k_pr_piece_cnt<<<1184, 256, 0, s>>>(q_off, n, piece, cnt);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, cnt, cnt, (size_t)n + 1, s);
+    if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+cudaError_t setup_pr_pieces_emit(const unsigned* q_v, const unsigned long long* q_off, unsigned long long n,
+                                 unsigned piece, const unsigned long long* pos, unsigned* q2_v,
+                                 unsigned long long* q2_off, cudaStream_t s) {
+    k_pr_piece_emit<<<1184, 256, 0, s>>>(q_v, q_off, n, piece, pos, q2_v, q2_off);
     return cudaGetLastError();
 }
 
