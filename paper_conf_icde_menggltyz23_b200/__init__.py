@@ -197,7 +197,7 @@ class RunStats:
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
                 osteal_edges_per_worker=0, chunk_edges=2048, pr_iterations=20, pr_damping=0.85, max_iterations=0,
-                trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=8192,
+                trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=16384,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
                 use_torch_allocator=False, streams=None, osteal_sync_edges=0.0, mirrors=False, hub_cache=False,
                 hub_degree=0):

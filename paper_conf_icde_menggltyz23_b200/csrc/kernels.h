@@ -57,6 +57,7 @@ cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col
                           unsigned long long E, unsigned long long seed, unsigned* d_inv, unsigned long long* r_row_ptr,
                           unsigned* r_col, unsigned* r_w, void* tmp, size_t tmp_bytes, cudaStream_t s);
 size_t setup_scan_tmp_bytes(unsigned V);
+size_t setup_relabel_tmp_bytes(unsigned V);  // RANDOM relabel: scan temp + hub-row list
 // symmetric (out + in) CSR for WCC: sym row v = out-neighbours of v followed by in-neighbours of v.
 cudaError_t setup_symmetrize(const unsigned long long* row_ptr, const unsigned* col, unsigned V, unsigned long long E,
                              unsigned long long* s_row_ptr, unsigned* s_col, unsigned long long* cursor, void* tmp,

@@ -1000,7 +1000,7 @@ void gum_config_default(gum_config* cfg) {
     cfg->chunk_edges = 2048;
     cfg->pr_iterations = 20;
     cfg->pr_damping = 0.85;
-    cfg->tail_vertices = 8192;
+    cfg->tail_vertices = 16384;
     cfg->pb_block_log2 = 0;  // propagation blocking is opt-in (slower than the probe path)
 }
 
@@ -1348,7 +1348,7 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
         c->p_col = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs);
         c->p_w = c->has_w ? (unsigned*)dalloc(c, d0, std::max<unsigned long long>(E, 1) * 4, c->part_allocs) : nullptr;
         std::vector<Alloc> tmp;
-        size_t tb = kind == GUM_PART_DEGREE ? setup_degree_tmp_bytes(V) : setup_scan_tmp_bytes(V);
+        size_t tb = kind == GUM_PART_DEGREE ? setup_degree_tmp_bytes(V) : setup_relabel_tmp_bytes(V);
         void* t = dalloc(c, d0, tb, tmp);
         if (!c->inv || !c->p_row_ptr || !c->p_col || (c->has_w && !c->p_w) || !t ||
             (kind == GUM_PART_DEGREE && !c->perm)) {

@@ -95,6 +95,15 @@ size_t setup_scan_tmp_bytes(unsigned V) {
                                   (int)0 + (size_t)V + 1);
     return bytes + 256;
 }
+size_t setup_relabel_tmp_bytes(unsigned V) {
+    return (setup_scan_tmp_bytes(V) + 255) / 256 * 256 + ((size_t)V * 4 + 255) / 256 * 256 + 256;
+}
+
+// relabelled rows -> new col/w: short rows by threads, medium rows by warps, hub rows by CTAs
+static cudaError_t relabel_move(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w,
+                                const unsigned* d_inv, unsigned V, unsigned long long seed, const unsigned* perm,
+                                const unsigned long long* r_row_ptr, unsigned* r_col, unsigned* r_w, unsigned* list,
+                                unsigned* cnt, cudaStream_t s);
 
 __global__ void k_inv_perm(unsigned V, unsigned long long seed, unsigned* inv) {
     for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
@@ -148,28 +157,24 @@ __global__ void k_relabel_rows(const unsigned long long* rp, const unsigned* col
     }
 }
 
-// hub rows (the highest-degree rows hold up to ~0.15% of all edges each on RMAT): the whole CTA per row
+// hub rows (the highest-degree rows hold up to ~0.15% of all edges each on RMAT): collected into a list
+// first, then one CTA per listed row (CTAs take list entries round-robin, so the degree-ordered layout's
+// hub rows -- all in the first ids -- do not land on one CTA)
+__global__ void k_huge_list(const unsigned long long* nrp, unsigned V, unsigned* list, unsigned* cnt) {
+    for (unsigned v = blockIdx.x * blockDim.x + threadIdx.x; v < V; v += gridDim.x * blockDim.x)
+        if (nrp[v + 1] - nrp[v] > kHugeRow) list[atomicAdd(cnt, 1u)] = v;
+}
 __global__ void k_relabel_huge(const unsigned long long* rp, const unsigned* col, const unsigned* w, const unsigned* inv,
                                unsigned V, unsigned long long seed, const unsigned* perm, const unsigned long long* nrp,
-                               unsigned* ncol, unsigned* nw) {
-    __shared__ unsigned s_rows[256];
-    __shared__ unsigned s_n;
-    for (unsigned long long b = (unsigned long long)blockIdx.x * blockDim.x; b < V;
-         b += (unsigned long long)gridDim.x * blockDim.x) {
-        if (threadIdx.x == 0) s_n = 0;
-        __syncthreads();
-        const unsigned long long v = b + threadIdx.x;
-        if (v < V && nrp[v + 1] - nrp[v] > kHugeRow) s_rows[atomicAdd(&s_n, 1u)] = (unsigned)v;
-        __syncthreads();
-        for (unsigned r = 0; r < s_n; r++) {
-            const unsigned hv = s_rows[r];
-            const unsigned long long d0 = nrp[hv], n = nrp[hv + 1] - d0, s0 = rp[inv[hv]];
-            for (unsigned long long j = threadIdx.x; j < n; j += blockDim.x) {
-                ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
-                if (w) nw[d0 + j] = w[s0 + j];
-            }
+                               unsigned* ncol, unsigned* nw, const unsigned* list, const unsigned* cnt) {
+    const unsigned n = *cnt;
+    for (unsigned r = blockIdx.x; r < n; r += gridDim.x) {
+        const unsigned hv = list[r];
+        const unsigned long long d0 = nrp[hv], m = nrp[hv + 1] - d0, s0 = rp[inv[hv]];
+        for (unsigned long long j = threadIdx.x; j < m; j += blockDim.x) {
+            ncol[d0 + j] = perm ? perm[col[s0 + j]] : feistel(col[s0 + j], V, seed);
+            if (w) nw[d0 + j] = w[s0 + j];
         }
-        __syncthreads();
     }
 }
 
@@ -181,10 +186,9 @@ cudaError_t setup_relabel(const unsigned long long* row_ptr, const unsigned* col
     k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
     cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
     if (e != cudaSuccess) return e;
-    k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
-    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
-    k_relabel_huge<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w);
-    return cudaGetLastError();
+    unsigned* list = (unsigned*)((char*)tmp + (setup_scan_tmp_bytes(V) + 255) / 256 * 256);
+    unsigned* cnt = list + ((size_t)V * 4 + 255) / 256 * 64;
+    return relabel_move(row_ptr, col, w, d_inv, V, seed, nullptr, r_row_ptr, r_col, r_w, list, cnt, s);
 }
 
 // DEGREE relabel (layout option): new ids in order of decreasing in-degree (ties by id), so the
@@ -232,10 +236,8 @@ cudaError_t setup_relabel_degree(const unsigned long long* row_ptr, const unsign
     k_new_deg<<<1184, 256, 0, s>>>(row_ptr, d_inv, V, r_row_ptr);
     e = cub::DeviceScan::ExclusiveSum(t, tb, r_row_ptr, r_row_ptr, (size_t)V + 1, s);
     if (e != cudaSuccess) return e;
-    k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
-    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
-    k_relabel_huge<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w);
-    return cudaGetLastError();
+    // (both key buffers are free after the sort: the hub-row list and its counter go there)
+    return relabel_move(row_ptr, col, w, d_inv, V, 0, d_perm, r_row_ptr, r_col, r_w, keys_out, keys_in, s);
 }
 
 __global__ void k_sym_deg(const unsigned long long* rp, const unsigned* col, unsigned V, unsigned long long E,
@@ -461,6 +463,19 @@ size_t setup_pb_tmp_bytes(unsigned nb) {
     cub::DeviceScan::ExclusiveSum(nullptr, bytes, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
                                   (size_t)nb + 1);
     return bytes + 256;
+}
+
+static cudaError_t relabel_move(const unsigned long long* row_ptr, const unsigned* col, const unsigned* w,
+                                const unsigned* d_inv, unsigned V, unsigned long long seed, const unsigned* perm,
+                                const unsigned long long* r_row_ptr, unsigned* r_col, unsigned* r_w, unsigned* list,
+                                unsigned* cnt, cudaStream_t s) {
+    k_relabel_short<<<4736, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, perm, r_row_ptr, r_col, r_w);
+    k_relabel_rows<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, perm, r_row_ptr, r_col, r_w);
+    cudaError_t e = cudaMemsetAsync(cnt, 0, 4, s);
+    if (e != cudaSuccess) return e;
+    k_huge_list<<<1184, 256, 0, s>>>(r_row_ptr, V, list, cnt);
+    k_relabel_huge<<<1184, 256, 0, s>>>(row_ptr, col, w, d_inv, V, seed, perm, r_row_ptr, r_col, r_w, list, cnt);
+    return cudaGetLastError();
 }
 
 cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,

@@ -225,7 +225,7 @@ def test_sssp_near_far_split(delta):
 
 
 @pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
-@pytest.mark.parametrize("tail", [0, 1, 64, 8192])
+@pytest.mark.parametrize("tail", [0, 1, 64, 8192, 16384])
 def test_tail_engine_long_chains(alg, tail):
     """High-diameter inputs (the long-tail regime): a 3000-vertex path with shortcuts and a grid; the
     cooperative tail engine must give the oracle's answer whether it never runs, enters/leaves every
@@ -326,3 +326,19 @@ def test_osteal_cost_model(alg, p):
         assert st.final_owners == 1
     if p < 1.0 and alg == "pr":
         assert st.final_owners == 4
+
+
+@pytest.mark.parametrize("part", ["random", "degree"])
+def test_relabel_hub_rows(part):
+    """Relabelling moves rows of every length class (thread / warp / CTA-per-row paths of the relabel):
+    out-stars with 5000-20000 leaves next to short random rows."""
+    rng = np.random.default_rng(3)
+    n = 60000
+    pairs = [(c, int(x)) for c, k in ((7, 20000), (11, 5000), (40000, 9000)) for x in rng.integers(0, n, k)]
+    pairs += [(int(a), int(b)) for a, b in rng.integers(0, n, (200000, 2))]
+    g = inputs.from_pairs(n, pairs, rng.integers(1, 256, len(pairs)))
+    csr = csr_of(g)
+    for alg in ("bfs", "sssp", "wcc"):
+        ref = oracle.run(alg, g, 7)
+        for P in (1, 3):
+            check(g, alg, 7, csr=csr, ref=ref, num_gpus=P, part=part, seed=5)
