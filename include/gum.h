@@ -187,6 +187,11 @@ typedef struct {
     uint64_t mirror_flush_bytes; /* PR mirrors: bytes the finalize read from peer mirrors */
     uint32_t blocked_iterations; /* WCC: iterations run on the static destination-blocked queue */
     uint32_t pad0;
+    /* of edges_expanded / vertices_frontier (list entries) / activations: the share done inside the tail
+     * engine (k_tail), so per-kernel byte counts can be attributed (bench.py roofline) */
+    uint64_t tail_edges;
+    uint64_t tail_vertices;
+    uint64_t tail_activations;
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

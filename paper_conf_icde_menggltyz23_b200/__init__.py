@@ -81,7 +81,8 @@ class gum_run_stats(ctypes.Structure):
                 ("pr_last_residual", ctypes.c_double), ("kernel_launches", ctypes.c_uint64),
                 ("remote_filtered", ctypes.c_uint64), ("hub_cached_edges", ctypes.c_uint64),
                 ("mirror_flush_bytes", ctypes.c_uint64), ("blocked_iterations", ctypes.c_uint32),
-                ("pad0", ctypes.c_uint32)]
+                ("pad0", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
+                ("tail_activations", ctypes.c_uint64)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -193,6 +194,9 @@ class RunStats:
     mirror_flush_bytes: int = 0
     blocked_iterations: int = 0
     pad0: int = 0
+    tail_edges: int = 0
+    tail_vertices: int = 0
+    tail_activations: int = 0
 
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,

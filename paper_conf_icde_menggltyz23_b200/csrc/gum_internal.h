@@ -59,6 +59,7 @@ struct alignas(128) FragCtl {
     unsigned long long pull_checked;   // bottom-up BFS: in-edges inspected
     unsigned long long remote_filtered;  // NEXT-1 mirrors: cross-fragment updates absorbed locally
     unsigned long long hub_edges;        // NEXT-1 hub cache: non-local edges expanded from a local copy
+    unsigned long long tail_edges, tail_vertices, tail_acts;  // work done inside the tail engine (stats)
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and

@@ -121,6 +121,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->pull_checked = 0;
         ct->remote_filtered = 0;
         ct->hub_edges = 0;
+        ct->tail_edges = ct->tail_vertices = ct->tail_acts = 0;
         if (sq) {
             ct->frontier_edges = F.sq_edges;
             ct->frontier_vertices = F.sq_len;
@@ -1710,7 +1711,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
     TailSplit* split = c.tsplit[w0];
     // accounting: iteration k0's queue was already counted by the filter (frontier_*); later tail
     // iterations count their own lists. edges_done counts every expanded edge (conservation).
-    unsigned long long e_done[kMaxW], e_front[kMaxW], v_front[kMaxW], a_sum = 0;
+    unsigned long long e_done[kMaxW], e_front[kMaxW], v_front[kMaxW], a_sum = 0, tail_v = 0;
     for (int i = 0; i < kMaxW; i++) e_done[i] = e_front[i] = v_front[i] = 0;
     unsigned it = 0;
     for (;; it++) {
@@ -1731,6 +1732,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
             const unsigned n = s_n[f];
             n_all += n;
             if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
+            if (gw == 0 && lane == 0) tail_v += n;
             for (unsigned i0 = gw * kTailVPW; i0 < n; i0 += nwarps * kTailVPW) {  // warp-uniform trip count
                 const unsigned i = i0 + sub;
                 const bool have = i < n;
@@ -1862,13 +1864,18 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         e_front[f] = warp_sum_u64(e_front[f]);
         if (lane == 0 && e_done[f]) {
             atomicAdd(&c.f[f].ctl->edges_done, e_done[f]);
+            atomicAdd(&c.f[0].ctl->tail_edges, e_done[f]);
             if (e_front[f]) atomicAdd(&c.f[f].ctl->frontier_edges, e_front[f]);
         }
         if (gw == 0 && lane == 0 && v_front[f]) atomicAdd(&c.f[f].ctl->frontier_vertices, v_front[f]);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) a_sum += __shfl_xor_sync(0xffffffffu, a_sum, o);
-    if (lane == 0 && a_sum) atomicAdd(&c.f[0].ctl->activations, a_sum);
+    if (lane == 0 && a_sum) {
+        atomicAdd(&c.f[0].ctl->activations, a_sum);
+        atomicAdd(&c.f[0].ctl->tail_acts, a_sum);
+    }
+    if (tail_v) atomicAdd(&c.f[0].ctl->tail_vertices, tail_v);
     // hand the last produced list back to the regular path as the sparse activation list
     if (blockIdx.x == 0) {
         const unsigned ns = (it + 1) % 3;

@@ -1705,6 +1705,9 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->vertices_frontier += fc.frontier_vertices;
             stats->remote_filtered += fc.remote_filtered;
             stats->hub_cached_edges += fc.hub_edges;
+            stats->tail_edges += fc.tail_edges;
+            stats->tail_vertices += fc.tail_vertices;
+            stats->tail_activations += fc.tail_acts;
             if (getenv("GUM_DEBUG"))
                 fprintf(stderr, "[gum] frag %d: V=%u E=%llu qlen=%llu edges_done=%llu frontier_edges=%llu frontier_vertices=%llu app_cnt=%u tcnt=%u,%u,%u\n",
                         f, c->fr[f].V, (unsigned long long)(alg == GUM_WCC ? c->fr[f].sE : c->fr[f].E), fc.qlen,
