@@ -1616,10 +1616,21 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
 // loads per warp. Appends keep the warp-aggregated reservation of tail_expand.
 constexpr unsigned kTailG = 8;
 constexpr unsigned kTailVPW = 32 / kTailG;
+// single fragment: phase-1 appends go to a CTA-local buffer, reserved in the next list with ONE atomic per
+// CTA per iteration instead of one returning atomic per warp and round on the same counter address
+// (thousands per iteration, serialised in one L2 slice and each on a warp's critical path)
+constexpr unsigned kTailAppCap = 2048;
+struct TailApp {
+    unsigned* buf;
+    unsigned* n;
+    unsigned* lim;  // reservations past the capacity go to the global list; the first failing base bounds
+                    // the buffer's valid prefix (a straddling group leaves [base, cap) unwritten)
+    unsigned long long* edges;
+};
 template <int ALG, bool MULTI>
 __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtrs& F, bool go, unsigned sval,
                                                   unsigned long long s0, unsigned long long s1, unsigned k,
-                                                  unsigned it, unsigned ns, unsigned gl) {
+                                                  unsigned it, unsigned ns, unsigned gl, const TailApp& ta) {
     const unsigned lane = lane_id();
     unsigned acts = 0;
     const unsigned long long d = go ? s1 - s0 : 0ull;
@@ -1629,12 +1640,17 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
         bool need = false;
         int tf = 0;
         unsigned lu = 0;
+        unsigned long long rp0 = 0, rp1 = 0;
         if (go && e < s1) {
             const unsigned u = __ldg(F.col + e);
             tf = MULTI ? frag_of(c, u) : 0;
             lu = MULTI ? u - c.bounds[tf] : u;
             const FragPtrs& T = c.f[tf];
             const unsigned bit = 1u << (lu & 31);
+            // the neighbour's row bounds (its out-degree, for the next list's edge count) load together with
+            // its state instead of after the append decision (one dependent round trip less per round)
+            rp0 = __ldg(T.row_ptr + lu);
+            rp1 = __ldg(T.row_ptr + lu + 1);
             if (ALG == ALG_BFS) {
                 if (!(vload(T.vis + (lu >> 5)) & bit)) {
                     const unsigned ob = atomicOr(T.vis + (lu >> 5), bit);
@@ -1663,20 +1679,31 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
         }
         const unsigned key = need ? (unsigned)tf : 0xFFFFFFFFu;
         const unsigned grp = MULTI ? __match_any_sync(0xffffffffu, key) : __ballot_sync(0xffffffffu, need);
+        const unsigned long long deg = need ? rp1 - rp0 : 0ull;
         if (need) {
             const FragPtrs& T = c.f[tf];
             const unsigned leader = __ffs(grp) - 1;
-            unsigned base = 0;
-            if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
-            base = __shfl_sync(grp, base, leader);
-            unsigned* nxt = (it & 1) ? T.q_v : T.app;
-            nxt[base + __popc(grp & lanemask_lt())] = lu;
-            acts++;
-        }
-        const unsigned long long deg = need ? __ldg(c.f[tf].row_ptr + lu + 1) - __ldg(c.f[tf].row_ptr + lu) : 0ull;
-        if (need) {
             const unsigned hi = __reduce_add_sync(grp, (unsigned)(deg >> 16)), lo = __reduce_add_sync(grp, (unsigned)(deg & 0xFFFFu));
-            if (lane == __ffs(grp) - 1) atomicAdd(&c.f[tf].ctl->tedges[ns], ((unsigned long long)hi << 16) + lo);
+            const unsigned long long gdeg = ((unsigned long long)hi << 16) + lo;
+            unsigned base = 0;
+            bool local = false;
+            if (!MULTI && ta.buf) {
+                if (lane == leader) base = atomicAdd(ta.n, (unsigned)__popc(grp));
+                base = __shfl_sync(grp, base, leader);
+                local = base + (unsigned)__popc(grp) <= kTailAppCap;  // group-uniform
+                if (!local && lane == leader && base < kTailAppCap) atomicMin(ta.lim, base);
+            }
+            if (local) {
+                ta.buf[base + __popc(grp & lanemask_lt())] = lu;
+                if (lane == leader) atomicAdd(ta.edges, gdeg);
+            } else {
+                if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
+                base = __shfl_sync(grp, base, leader);
+                unsigned* nxt = (it & 1) ? T.q_v : T.app;
+                nxt[base + __popc(grp & lanemask_lt())] = lu;
+                if (lane == leader) atomicAdd(&T.ctl->tedges[ns], gdeg);
+            }
+            acts++;
         }
     }
     return acts;
@@ -1685,6 +1712,14 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
 template <int ALG, bool MULTI>
 __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
     __shared__ unsigned s_n[kMaxW], s_nsplit, s_go;
+    __shared__ unsigned s_app[MULTI ? 1 : kTailAppCap], s_app_n, s_app_lim, s_app_base;
+    __shared__ unsigned long long s_app_e;
+    const TailApp ta{MULTI ? nullptr : s_app, &s_app_n, &s_app_lim, &s_app_e};
+    if (threadIdx.x == 0) {
+        s_app_n = 0;
+        s_app_lim = kTailAppCap;
+        s_app_e = 0;
+    }
     __shared__ unsigned long long s_tn[kMaxW], s_te[kMaxW];
     RunCtl* rc = c.rctl[w0];
     __shared__ unsigned s_hdr[4];  // gen, k0, nfT, fslot
@@ -1748,6 +1783,9 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                         // improvement of v from now on appends it to the NEXT list (other parity)
                         if (it > 0) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
                         sval = vload(F.state + v);
+                        // v's far bit is only changed by v's own processing: read it with the state (one
+                        // round trip) instead of after the near/far decision
+                        const unsigned fw = (nf && s1 > s0) ? F.far[v >> 5] : 0u;
                         if (nf && s1 > s0) {  // like the filter, only vertices with out-edges are parked
                             const unsigned bit = 1u << (v & 31);
                             if (sval >= nfT) {
@@ -1755,7 +1793,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                                 const unsigned ob = atomicOr(F.far + (v >> 5), bit);
                                 if (!(ob & bit)) atomicAdd(&F.ctl->far_cnt, 1ull);
                                 atomicMin(&F.ctl->far_min[fslot], sval);
-                            } else if (F.far[v >> 5] & bit) {
+                            } else if (fw & bit) {
                                 const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
                                 if (ob & bit) atomicAdd(&F.ctl->far_cnt, ~0ull);
                             }
@@ -1775,7 +1813,27 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 slot = __shfl_sync(0xffffffffu, slot, src);
                 sval = __shfl_sync(0xffffffffu, sval, src);
                 // split vertices are expanded cooperatively in phase 2
-                a_sum += tail_expand_g<ALG, MULTI>(c, F, !park && slot >= kTailSplitCap, sval, s0, s1, k, it, ns, gl);
+                a_sum += tail_expand_g<ALG, MULTI>(c, F, !park && slot >= kTailSplitCap, sval, s0, s1, k, it, ns, gl, ta);
+            }
+        }
+        if (!MULTI) {
+            // the CTA's buffered appends: one reservation in the next list, then a coalesced copy
+            __syncthreads();
+            const unsigned na = s_app_n < s_app_lim ? s_app_n : s_app_lim;
+            if (threadIdx.x == 0 && na) {
+                s_app_base = atomicAdd(&c.f[0].ctl->tcnt[ns], na);
+                atomicAdd(&c.f[0].ctl->tedges[ns], s_app_e);
+            }
+            __syncthreads();
+            if (na) {
+                unsigned* nxt = (it & 1) ? c.f[0].q_v : c.f[0].app;
+                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base + i] = s_app[i];
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                s_app_n = 0;
+                s_app_lim = kTailAppCap;
+                s_app_e = 0;
             }
         }
         if (tr && k < (unsigned)kTraceMax) {

@@ -241,8 +241,11 @@ def test_tail_engine_long_chains(alg, tail):
             _, st, _ = check(g, alg, s, csr=csr, ref=ref, tail_vertices=tail, **kw)
             if tail == 8192 and alg != "wcc":
                 assert st.tail_iterations > 0
+                assert 0 < st.tail_edges <= st.edges_expanded and 0 < st.tail_vertices <= st.vertices_frontier
             if tail == 0:
                 assert st.tail_iterations == 0
+                assert st.tail_edges == st.tail_vertices == st.tail_activations == 0
+            assert st.tail_activations <= st.activations
         if alg == "sssp":
             check(g, alg, s, csr=csr, ref=ref, tail_vertices=tail, sssp_delta=20)
 
@@ -342,3 +345,22 @@ def test_relabel_hub_rows(part):
         ref = oracle.run(alg, g, 7)
         for P in (1, 3):
             check(g, alg, 7, csr=csr, ref=ref, num_gpus=P, part=part, seed=5)
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
+def test_tail_engine_append_overflow(alg):
+    """One CTA of the tail engine appends more vertices than its shared buffer holds (2048): 40 mid vertices
+    of out-degree 250 (below the 256-edge split threshold) discovered together, each with fresh leaves."""
+    rng = np.random.default_rng(11)
+    mids = list(range(1, 41))
+    pairs = [(0, m) for m in mids]
+    nxt = 41
+    for m in mids:
+        pairs += [(m, nxt + j) for j in range(250)]
+        nxt += 250
+    pairs += [(nxt - 1 - j, j % 41) for j in range(0, 2000, 7)]  # back edges (cycles for WCC/SSSP)
+    g = inputs.from_pairs(nxt, pairs, rng.integers(1, 30, len(pairs)))
+    ref = oracle.run(alg, g, 0)
+    csr = csr_of(g)
+    for kw in (dict(), dict(tail_vertices=1 << 16), dict(num_gpus=2, tail_vertices=1 << 16)):
+        _, st, _ = check(g, alg, 0, csr=csr, ref=ref, **kw)

@@ -31,8 +31,13 @@ import inputs  # noqa: E402
 import paper_conf_icde_menggltyz23_b200 as gum  # noqa: E402
 
 
+TAIL = None  # --tail: tail engine threshold override
+
+
 def run(csr, alg, src, reps=3, **kw):
     rp, col, w = csr
+    if TAIL is not None:
+        kw.setdefault("tail_vertices", TAIL)
     with gum.Context(trace=True, **kw) as ctx:
         ctx.load_csr(rp, col, w if alg == "sssp" else None)
         ctx.partition("seg")
@@ -160,9 +165,12 @@ def main():
     ap.add_argument("--delta", type=int, default=0, help="SSSP near-far split (0 = plain frontier)")
     ap.add_argument("--split", action="store_true")
     ap.add_argument("--next1", action="store_true")
+    ap.add_argument("--tail", type=int, default=None, help="tail engine threshold (default: the library's)")
     ap.add_argument("--hub-degree", type=int, default=64)
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
+    global TAIL
+    TAIL = args.tail
     out = {}
     if args.fsteal:
         out["fsteal"] = fsteal(args)

@@ -19,11 +19,13 @@ ap.add_argument("--runs", type=int, default=1)
 ap.add_argument("--gpus", type=int, default=1)
 ap.add_argument("--host-loop", type=int, default=1)
 ap.add_argument("--part", default="seg")
+ap.add_argument("--delta", type=int, default=None, help="SSSP near-far split (default: bench.py's, 4096 on C3)")
 a = ap.parse_args()
 g = inputs.make_config(a.config, weighted=(a.alg == "sssp"))
 s = 0 if a.config == "C3" else inputs.pick_source(g, int(a.config[1]))
 rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
-with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop)) as ctx:
+delta = a.delta if a.delta is not None else (4096 if a.config == "C3" and a.alg == "sssp" else 0)
+with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop), sssp_delta=delta) as ctx:
     ctx.load_csr(rp, col, w)
     ctx.partition(a.part, 1)
     ctx.prepare(a.alg)
