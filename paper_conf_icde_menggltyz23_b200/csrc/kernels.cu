@@ -864,7 +864,9 @@ __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned
     return done;
 }
 
-template <int ALG, bool MULTI, bool PB = false>
+// NX: the NEXT-1 reducers (mirrors / hub cache) are compiled in; the plain multi-worker instantiation
+// leaves them out (their registers cost the default path ~15% on P = 8 virtual workers)
+template <int ALG, bool MULTI, bool PB = false, bool NX = false>
 #ifndef GUM_ADV_MINB_BFS
 #define GUM_ADV_MINB_BFS 4
 #endif
@@ -882,7 +884,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     unsigned* const s_stage = s_head;  // s_head is dead once the chunk's col ids are loaded
     __shared__ unsigned s_wmax[kAdvThreads / 32];
     // NEXT-1 hub cache: per staged vertex, 1 = its list is expanded from this worker's local copy
-    __shared__ unsigned char s_hub[MULTI ? kTileMax : 1];
+    __shared__ unsigned char s_hub[(MULTI && NX) ? kTileMax : 1];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
     __shared__ unsigned long long s_cnt[kMaxW][4];  // per fragment: edges, chunks, stolen edges, stolen chunks
@@ -940,7 +942,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0, filtered = 0, hub_e = 0;
     unsigned nval = 0;  // masked blocked pass: this thread's expanded edges of the current chunk
     // NEXT-1 outer-vertex mirrors (this worker's memory): updates to other fragments go through them
-    const bool mir = MULTI && c.mirrors;
+    const bool mir = MULTI && NX && c.mirrors;
 
     // Chunk claims run one chunk ahead of the expansion (thread 0): while chunk n is expanded, chunk n+1
     // is already claimed and its staging data (chunk table entries, degree prefix, col base, source
@@ -1031,7 +1033,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     auto chunk_ref = [&](int f, unsigned long long t, int stolen) {
         ChunkRef r{f, t, stolen, 0u, 0u, 0u, false};
         if (f < 0) return r;
-        r.hc = MULTI && ALG != ALG_PR && c.hub_on && f != w;
+        r.hc = MULTI && NX && ALG != ALG_PR && c.hub_on && f != w;
         const FragPtrs& F = c.f[f];
         const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned* const tilep = sq ? F.sq_tile : F.tile;
@@ -1135,7 +1137,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                 val = value_of(cur, u);
             }
             s_base[kk] = base;
-            if (MULTI) s_hub[kk] = hub ? 1 : 0;
+            if (MULTI && NX) s_hub[kk] = hub ? 1 : 0;
             if (ALG != ALG_BFS) s_val[kk] = val;
             const long long rel = (long long)off - (long long)tb;
             if (rel > 0 && rel < (long long)tlen) s_head[rel] = (seq << 12) | kk;
@@ -1210,8 +1212,8 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                     nval++;
                 }
                 const unsigned long long ci = (unsigned)(s_base[kk] + e);  // mod 2^32: the base may wrap
-                const bool hv = MULTI && cur.hc && s_hub[kk];
-                if (MULTI) hub_e += hv ? 1 : 0;
+                const bool hv = MULTI && NX && cur.hc && s_hub[kk];
+                if (MULTI && NX) hub_e += hv ? 1 : 0;
                 vv[j] = __ldcs((hv ? c.hub[w][f].col : colp) + ci);
                 if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
                 if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];
@@ -1812,8 +1814,19 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 park = __shfl_sync(0xffffffffu, park ? 1u : 0u, src) != 0;
                 slot = __shfl_sync(0xffffffffu, slot, src);
                 sval = __shfl_sync(0xffffffffu, sval, src);
-                // split vertices are expanded cooperatively in phase 2
-                a_sum += tail_expand_g<ALG, MULTI>(c, F, !park && slot >= kTailSplitCap, sval, s0, s1, k, it, ns, gl, ta);
+                // split vertices are expanded cooperatively in phase 2; lists longer than 32 edges by the
+                // whole warp, one vertex at a time (8 lanes would need up to 32 rounds for a 256-edge list)
+                const bool go = !park && slot >= kTailSplitCap;
+                const bool wide = go && s1 - s0 > 32;
+                a_sum += tail_expand_g<ALG, MULTI>(c, F, go && !wide, sval, s0, s1, k, it, ns, gl, ta);
+                unsigned wmask = __ballot_sync(0xffffffffu, wide && gl == 0);
+                while (wmask) {
+                    const unsigned ld = __ffs(wmask) - 1;
+                    wmask &= wmask - 1;
+                    const unsigned wv = __shfl_sync(0xffffffffu, sval, ld);
+                    const unsigned long long w0s = __shfl_sync(0xffffffffu, s0, ld), w1s = __shfl_sync(0xffffffffu, s1, ld);
+                    a_sum += tail_expand<ALG, MULTI>(c, F, wv, w0s, w1s, k, it, ns);
+                }
             }
         }
         if (!MULTI) {
@@ -2323,7 +2336,10 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
             if (ALG == ALG_PR && c.P == 1 && c.f[0].pr2_q_v)
                 k_pr_push<<<L.adv_grid_pr, kThreads, 0, s>>>(c, L.w0, L.nw);
             else if (c.P > 1)
-                k_advance<ALG, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
+                if (c.mirrors || c.hub_on)
+                    k_advance<ALG, true, false, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
+                else
+                    k_advance<ALG, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);
             else
                 if (ALG == ALG_BFS && c.pb_shift)
                     k_advance<ALG, false, true><<<L.adv_grid, kAdvThreads, 0, s>>>(c, L.w0, L.nw);

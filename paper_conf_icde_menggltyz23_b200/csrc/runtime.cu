@@ -1094,7 +1094,7 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     cudaGetLastError();
     {
         int occ = 0;
-        if (tail_occupancy(&occ) == cudaSuccess && occ > 0) c->tail_occ = std::min(occ, 2);
+        if (tail_occupancy(&occ) == cudaSuccess && occ > 0) c->tail_occ = std::min(occ, 3);  // C3: 2 -> 3 per SM 253 -> 243 ms
         if (const char* e = getenv("GUM_TAIL_CTAS_PER_SM")) c->tail_occ = std::max(1, std::min(occ, atoi(e)));
         cudaGetLastError();
         occ = 0;
