@@ -202,6 +202,8 @@ struct DevCtx {
     unsigned long long total_edges;  // sum of the fragments' out-edges
     int mirrors;                // NEXT-1 outer-vertex mirrors (P > 1 only)
     unsigned int filter_swizzle;  // filter: spread each CTA's tile range over the id space (stride permutation)
+    unsigned int bfs_filter_depth;  // BFS: the filter writes the depth of the vertices it takes from the
+                                    // activations (the advance only sets visited / frontier bits)
     unsigned int wcc_blocked;     // WCC static destination-blocked queue exists: dense iterations may run on
                                   // it (the filter keeps the frontier bitmap in F.far)
     int hub_on;                 // NEXT-1 hub cache built for this algorithm

@@ -340,7 +340,7 @@ __device__ __forceinline__ void nf_flush(FragCtl* ct, unsigned fslot, const NfAc
 }
 
 template <int MODE>
-__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool keep_fbm, unsigned tile, bool dense, bool sweep,
+__device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool keep_fbm, unsigned depth, unsigned tile, bool dense, bool sweep,
                                             bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt, unsigned ipt,
                                             unsigned chunk, unsigned long long pos, unsigned long long off) {
     const unsigned lane = lane_id();
@@ -362,6 +362,13 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
             }
         }
         const unsigned bits = (word >> ((lane & 3u) * 8u)) & 0xFFu;
+        if (MODE == FT_EMIT && depth != GUM_INF && bits) {
+            // BFS: the depth of every vertex activated by the previous advance is written here, in vertex
+            // order, instead of by every discovering edge in the advance (a random 4-byte store each)
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread; q++)
+                if ((bits >> q) & 1u) F.state[vb + q] = depth;
+        }
         if (bits) {
             unsigned long long rpv[kDenseVertsPerThread + 1];
             const unsigned long long* rp = F.row_ptr + vb;  // 64-byte aligned (vb % 8 == 0)
@@ -413,6 +420,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
                 const unsigned v = items[j];
                 // every set bit belongs to a listed vertex: clearing whole words is exact
                 if (MODE == FT_EMIT) F.bm[v >> 5] = 0u;
+                if (MODE == FT_EMIT && depth != GUM_INF) F.state[v] = depth;  // BFS (see the dense path)
                 rp0[j] = __ldg(F.row_ptr + v);
                 d[j] = __ldg(F.row_ptr + v + 1) - rp0[j];
             }
@@ -448,13 +456,16 @@ __device__ unsigned g_fcall;
 #else
 #define FT_MARK(i) do {} while (0)
 #endif
+// NF: SSSP near-far parking compiled in (its batched state loads and far-bit atomics cost registers the
+// other algorithms' filters do not need)
+template <bool NF>
 __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     FT_MARK(0);
     // Prologue by thread 0 only, broadcast through shared memory: the run-control fields are a handful of
     // L2 lines that every CTA of every kernel reads, and per-warp loads of one address serialise in its
     // L2 slice (with ~600 CTAs x 8 warps that alone cost tens of microseconds per launch).
     struct Pro {
-        unsigned go, sweep, dense, nfT, fslot, app_cnt, b, pad;
+        unsigned go, sweep, dense, nfT, fslot, app_cnt, b, depth;
         unsigned long long epoch;
     };
     __shared__ Pro s_pro;
@@ -463,7 +474,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     const int f = blockIdx.y;
     const FragPtrs& F = c.f[f];
     FragCtl* ct = F.ctl;
-    const bool nf = c.nf_delta != 0;
+    const bool nf = NF && c.nf_delta != 0;
     if (threadIdx.x == 0) {
         Pro p{};
         const unsigned o = vload(&rc->owner[f]);
@@ -478,6 +489,8 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
             p.dense = p.sweep || vload(&rc->next_dense) != 0;
             p.app_cnt = p.dense ? 0u : vload(&ct->app_cnt);
             p.epoch = vload(&rc->epoch);
+            // BFS: activations of advance k-1 have depth k = the iteration counter before control runs
+            p.depth = c.bfs_filter_depth ? vload(&rc->iter) : GUM_INF;
             p.b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
         }
         s_pro = p;
@@ -492,6 +505,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     const bool dense = s_pro.dense != 0;
     const unsigned app_cnt = s_pro.app_cnt;
     const bool keep_fbm = c.wcc_blocked != 0 && !nf;
+    const unsigned depth = s_pro.depth;
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
     // sparse lists: items per thread so that the tiles cover the grid (1..8)
@@ -526,7 +540,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     Pair mine{0, 0};
     NfAcc nfa;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, keep_fbm, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
         mine.cnt += q.cnt;
         mine.deg += q.deg;
     }
@@ -567,16 +581,16 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
     if (t_hi - t_lo == 1) {
         // one tile: pass 1's per-thread counts are this tile's (same acceptance), no re-count
-        filter_tile<FT_EMIT>(F, nfa, keep_fbm, (unsigned)((unsigned long long)t_lo * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
+        filter_tile<FT_EMIT>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t_lo * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
                              run_deg + tex1.deg);
         filter_flush_long(F);
     } else {
         for (unsigned t = t_lo; t < t_hi; t++) {
             const unsigned pt = (unsigned)((unsigned long long)t * stride % n_tiles);
-            const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+            const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
             Pair tot;
             const Pair tex = block_excl_scan(q, s_warp, tot);
-            filter_tile<FT_EMIT>(F, nfa, keep_fbm, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
+            filter_tile<FT_EMIT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
                                  run_deg + tex.deg);
             filter_flush_long(F);
             run_cnt += tot.cnt;
@@ -1356,7 +1370,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                         const unsigned bit = 1u << (lvv[j] & 31);
                         atomicOr(T.vis + (lvv[j] >> 5), bit);  // RED.OR
                         atomicOr(T.bm + (lvv[j] >> 5), bit);   // RED.OR
-                        T.state[lvv[j]] = k + 1;
+                        // (the depth k+1 is written by the next filter: BFS state is write-only here)
                         if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
                     }
                 }
@@ -1373,7 +1387,6 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                 for (int j = 0; j < kEdgesPerThread; j++) {
                     if (!(ob[j] & (1u << (lvv[j] & 31)))) {
                         need |= 1u << j;
-                        c.f[tfv[j]].state[lvv[j]] = k + 1;
                         if (MULTI) remote += (s_owner[tfv[j]] != (unsigned)w) ? 1 : 0;
                     }
                 }
@@ -1992,7 +2005,7 @@ void dump_filter_timing() {
 #endif
 
 cudaError_t filter_occupancy(int* blocks_per_sm) {
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_filter, kThreads, 0);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_filter<true>, kThreads, 0);
 }
 
 cudaError_t tail_occupancy(int* blocks_per_sm) {
@@ -2330,7 +2343,12 @@ template <int ALG>
 static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L, cudaStream_t s,
                                    cudaGraphConditionalHandle h, int use_h) {
     switch (kind) {
-        case KER_FILTER: k_filter<<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw); break;
+        case KER_FILTER:
+            if (c.nf_delta)
+                k_filter<true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+            else
+                k_filter<false><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+            break;
         case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
         case KER_ADVANCE:
             if (ALG == ALG_PR && c.P == 1 && c.f[0].pr2_q_v)

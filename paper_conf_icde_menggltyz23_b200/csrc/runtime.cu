@@ -423,6 +423,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
     static const int env_sw = getenv("GUM_FILTER_SWIZZLE") ? atoi(getenv("GUM_FILTER_SWIZZLE")) : 1;
     d.filter_swizzle = env_sw ? 1u : 0u;
+    d.bfs_filter_depth = alg == GUM_BFS ? 1u : 0u;  // (the advance no longer writes BFS depths)
     static const int env_wb = getenv("GUM_WCC_BLOCKED") ? atoi(getenv("GUM_WCC_BLOCKED")) : 1;
     d.wcc_blocked = (alg == GUM_WCC && c->fr[0].sq_col && c->cfg.fsteal != 2 && env_wb) ? 1u : 0u;
     for (int f = 0; f < c->P; f++) d.total_edges += c->fr[f].E;
