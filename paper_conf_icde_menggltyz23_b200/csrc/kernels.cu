@@ -364,10 +364,27 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
         const unsigned bits = (word >> ((lane & 3u) * 8u)) & 0xFFu;
         if (MODE == FT_EMIT && depth != GUM_INF && bits) {
             // BFS: the depth of every vertex activated by the previous advance is written here, in vertex
-            // order, instead of by every discovering edge in the advance (a random 4-byte store each)
+            // order, instead of by every discovering edge in the advance (a random 4-byte store each):
+            // the thread's 8 consecutive states as two 16-byte read-modify-writes
+            if (vb + kDenseVertsPerThread <= F.V) {
+                uint4* sp = reinterpret_cast<uint4*>(F.state + vb);  // 32-byte aligned (vb % 8 == 0)
+                uint4 a = bits == 0xFFu ? make_uint4(0, 0, 0, 0) : __ldcg(sp);
+                uint4 b = bits == 0xFFu ? make_uint4(0, 0, 0, 0) : __ldcg(sp + 1);
+                if (bits & 1u) a.x = depth;
+                if (bits & 2u) a.y = depth;
+                if (bits & 4u) a.z = depth;
+                if (bits & 8u) a.w = depth;
+                if (bits & 16u) b.x = depth;
+                if (bits & 32u) b.y = depth;
+                if (bits & 64u) b.z = depth;
+                if (bits & 128u) b.w = depth;
+                if (bits & 0x0Fu) sp[0] = a;
+                if (bits & 0xF0u) sp[1] = b;
+            } else {
 #pragma unroll
-            for (int q = 0; q < kDenseVertsPerThread; q++)
-                if ((bits >> q) & 1u) F.state[vb + q] = depth;
+                for (int q = 0; q < kDenseVertsPerThread; q++)
+                    if ((bits >> q) & 1u) F.state[vb + q] = depth;
+            }
         }
         if (bits) {
             unsigned long long rpv[kDenseVertsPerThread + 1];
