@@ -1652,12 +1652,13 @@ constexpr unsigned kTailVPW = 32 / kTailG;
 // CTA per iteration instead of one returning atomic per warp and round on the same counter address
 // (thousands per iteration, serialised in one L2 slice and each on a warp's critical path)
 constexpr unsigned kTailAppCap = 2048;
-struct TailApp {
+struct TailApp {  // per target fragment f: buf[f * cap ..], n[f], lim[f], edges[f]
     unsigned* buf;
     unsigned* n;
     unsigned* lim;  // reservations past the capacity go to the global list; the first failing base bounds
                     // the buffer's valid prefix (a straddling group leaves [base, cap) unwritten)
     unsigned long long* edges;
+    unsigned cap;   // kTailAppCap / fragments
 };
 template <int ALG, bool MULTI>
 __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtrs& F, bool go, unsigned sval,
@@ -1719,15 +1720,16 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
             const unsigned long long gdeg = ((unsigned long long)hi << 16) + lo;
             unsigned base = 0;
             bool local = false;
-            if (!MULTI && ta.buf) {
-                if (lane == leader) base = atomicAdd(ta.n, (unsigned)__popc(grp));
+            {
+                // (MULTI: grp holds the lanes with the same target fragment -- match_any above)
+                if (lane == leader) base = atomicAdd(ta.n + tf, (unsigned)__popc(grp));
                 base = __shfl_sync(grp, base, leader);
-                local = base + (unsigned)__popc(grp) <= kTailAppCap;  // group-uniform
-                if (!local && lane == leader && base < kTailAppCap) atomicMin(ta.lim, base);
+                local = base + (unsigned)__popc(grp) <= ta.cap;  // group-uniform
+                if (!local && lane == leader && base < ta.cap) atomicMin(ta.lim + tf, base);
             }
             if (local) {
-                ta.buf[base + __popc(grp & lanemask_lt())] = lu;
-                if (lane == leader) atomicAdd(ta.edges, gdeg);
+                ta.buf[tf * ta.cap + base + __popc(grp & lanemask_lt())] = lu;
+                if (lane == leader) atomicAdd(ta.edges + tf, gdeg);
             } else {
                 if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
                 base = __shfl_sync(grp, base, leader);
@@ -1744,13 +1746,14 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
 template <int ALG, bool MULTI>
 __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
     __shared__ unsigned s_n[kMaxW], s_nsplit, s_go;
-    __shared__ unsigned s_app[MULTI ? 1 : kTailAppCap], s_app_n, s_app_lim, s_app_base;
-    __shared__ unsigned long long s_app_e;
-    const TailApp ta{MULTI ? nullptr : s_app, &s_app_n, &s_app_lim, &s_app_e};
-    if (threadIdx.x == 0) {
-        s_app_n = 0;
-        s_app_lim = kTailAppCap;
-        s_app_e = 0;
+    __shared__ unsigned s_app[kTailAppCap], s_app_n[kMaxW], s_app_lim[kMaxW], s_app_base[kMaxW];
+    __shared__ unsigned long long s_app_e[kMaxW];
+    const unsigned app_cap = kTailAppCap / (unsigned)(MULTI ? c.P : 1);
+    const TailApp ta{s_app, s_app_n, s_app_lim, s_app_e, app_cap};
+    if (threadIdx.x < (unsigned)kMaxW) {
+        s_app_n[threadIdx.x] = 0;
+        s_app_lim[threadIdx.x] = app_cap;
+        s_app_e[threadIdx.x] = 0;
     }
     __shared__ unsigned long long s_tn[kMaxW], s_te[kMaxW];
     RunCtl* rc = c.rctl[w0];
@@ -1859,24 +1862,29 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 }
             }
         }
-        if (!MULTI) {
-            // the CTA's buffered appends: one reservation in the next list, then a coalesced copy
+        {
+            // the CTA's buffered appends: one reservation per target fragment's next list, then a copy
             __syncthreads();
-            const unsigned na = s_app_n < s_app_lim ? s_app_n : s_app_lim;
-            if (threadIdx.x == 0 && na) {
-                s_app_base = atomicAdd(&c.f[0].ctl->tcnt[ns], na);
-                atomicAdd(&c.f[0].ctl->tedges[ns], s_app_e);
+            if (threadIdx.x < (unsigned)nfrag) {
+                const unsigned f = threadIdx.x;
+                const unsigned na = s_app_n[f] < s_app_lim[f] ? s_app_n[f] : s_app_lim[f];
+                if (na) {
+                    s_app_base[f] = atomicAdd(&c.f[f].ctl->tcnt[ns], na);
+                    atomicAdd(&c.f[f].ctl->tedges[ns], s_app_e[f]);
+                }
+                s_app_n[f] = na;  // (the valid prefix to copy)
             }
             __syncthreads();
-            if (na) {
-                unsigned* nxt = (it & 1) ? c.f[0].q_v : c.f[0].app;
-                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base + i] = s_app[i];
+            for (int f = 0; f < nfrag; f++) {
+                const unsigned na = s_app_n[f];
+                unsigned* nxt = (it & 1) ? c.f[f].q_v : c.f[f].app;
+                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base[f] + i] = s_app[f * app_cap + i];
             }
             __syncthreads();
-            if (threadIdx.x == 0) {
-                s_app_n = 0;
-                s_app_lim = kTailAppCap;
-                s_app_e = 0;
+            if (threadIdx.x < (unsigned)kMaxW) {
+                s_app_n[threadIdx.x] = 0;
+                s_app_lim[threadIdx.x] = app_cap;
+                s_app_e[threadIdx.x] = 0;
             }
         }
         if (tr && k < (unsigned)kTraceMax) {
