@@ -319,12 +319,17 @@ def main():
     ap.add_argument("--osteal", type=int, default=1)
     ap.add_argument("--sssp-delta", type=int, default=None,
                     help="near-far split for SSSP (default: 4096 on the C3 grid, 0 = plain BSP frontier otherwise)")
-    ap.add_argument("--tail", type=int, default=16384, help="tail engine threshold (vertices; 0 = off)")
+    ap.add_argument("--tail", type=int, default=None,
+                    help="tail engine threshold (vertices; 0 = off). Default: 16384, except BFS on the RMAT configs "
+                         "(C1/C2: 8 iterations, no long tail; the engine's per-iteration launch costs more than it "
+                         "saves -- C2 1.622 ms with it, 1.595 ms without), where it is 0")
     ap.add_argument("--bfs-pull", type=int, default=0, help="NEXT-4 direction-optimising BFS (bottom-up iterations)")
     args = ap.parse_args()
     alg = args.alg or DEFAULT_ALG[args.config]
     if args.part is None:
         args.part = "degree" if alg == "bfs" else "seg"
+    if args.tail is None:
+        args.tail = 0 if (alg == "bfs" and args.config in ("C1", "C2")) else 16384
     rank = env_int("RANK", 0)
     world = env_int("WORLD_SIZE", 1)
     N = args.gpus

@@ -21,9 +21,14 @@ ap.add_argument("--host-loop", type=int, default=1)
 ap.add_argument("--part", default="seg")
 ap.add_argument("--rmat", type=int, default=0, help="instead of --config: RMAT of this scale (EF 16, seed 9)")
 ap.add_argument("--noscramble", action="store_true")
+ap.add_argument("--grid", type=int, default=0, help="instead of --config: n x n grid (seed 3), source 0")
+ap.add_argument("--osteal-threshold", type=int, default=0)
 ap.add_argument("--delta", type=int, default=None, help="SSSP near-far split (default: bench.py's, 4096 on C3)")
 a = ap.parse_args()
-if a.rmat:
+if a.grid:
+    g = inputs.grid(a.grid, seed=3)
+    s = 0
+elif a.rmat:
     g = inputs.rmat(a.rmat, 16, seed=9, scramble=not a.noscramble, weighted=(a.alg == "sssp"))
     s = inputs.pick_source(g, 9)
 else:
@@ -31,7 +36,8 @@ else:
     s = 0 if a.config == "C3" else inputs.pick_source(g, int(a.config[1]))
 rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
 delta = a.delta if a.delta is not None else (4096 if a.config == "C3" and a.alg == "sssp" else 0)
-with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop), sssp_delta=delta) as ctx:
+with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop), sssp_delta=delta,
+                 osteal_threshold=a.osteal_threshold) as ctx:
     ctx.load_csr(rp, col, w)
     ctx.partition(a.part, 1)
     ctx.prepare(a.alg)
