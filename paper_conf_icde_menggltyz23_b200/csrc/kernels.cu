@@ -1646,8 +1646,13 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
 // group); every group walks its own vertex's edges [s0, s1) kTailG at a time. Low-degree frontiers (road-like
 // grids: out-degree <= 4) would otherwise leave 28 of 32 lanes idle and serialise one vertex's dependent
 // loads per warp. Appends keep the warp-aggregated reservation of tail_expand.
-constexpr unsigned kTailG = 8;
-constexpr unsigned kTailVPW = 32 / kTailG;
+// (multi-fragment runs keep a warp per vertex: their tails are small frontiers spread over fragments, where
+// the 8-lane groups measured slower -- SSSP 2048^2 grid on 8 virtual workers: 90 vs 123 ms of tail engine)
+template <bool MULTI>
+struct TailGroup {
+    static constexpr unsigned G = MULTI ? 32u : 8u;
+    static constexpr unsigned VPW = 32u / G;
+};
 // single fragment: phase-1 appends go to a CTA-local buffer, reserved in the next list with ONE atomic per
 // CTA per iteration instead of one returning atomic per warp and round on the same counter address
 // (thousands per iteration, serialised in one L2 slice and each on a warp's critical path)
@@ -1667,6 +1672,7 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
     const unsigned lane = lane_id();
     unsigned acts = 0;
     const unsigned long long d = go ? s1 - s0 : 0ull;
+    constexpr unsigned kTailG = TailGroup<MULTI>::G;
     const unsigned rounds = __reduce_max_sync(0xffffffffu, (unsigned)((d + kTailG - 1) / kTailG));
     for (unsigned r = 0; r < rounds; r++) {
         const unsigned long long e = s0 + (unsigned long long)r * kTailG + gl;
@@ -1746,7 +1752,7 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
 template <int ALG, bool MULTI>
 __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ DevCtx c, int w0) {
     __shared__ unsigned s_n[kMaxW], s_nsplit, s_go;
-    __shared__ unsigned s_app[kTailAppCap], s_app_n[kMaxW], s_app_lim[kMaxW], s_app_base[kMaxW];
+    __shared__ unsigned s_app[kTailAppCap], s_app_n[kMaxW], s_app_na[kMaxW], s_app_lim[kMaxW], s_app_base[kMaxW];
     __shared__ unsigned long long s_app_e[kMaxW];
     const unsigned app_cap = kTailAppCap / (unsigned)(MULTI ? c.P : 1);
     const TailApp ta{s_app, s_app_n, s_app_lim, s_app_e, app_cap};
@@ -1795,6 +1801,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         __syncthreads();
         // ---- phase 1: kTailG lanes per listed vertex (kTailVPW vertices per warp); high-degree vertices
         // go to the split list
+        constexpr unsigned kTailG = TailGroup<MULTI>::G, kTailVPW = TailGroup<MULTI>::VPW;
         const unsigned sub = lane / kTailG, gl = lane % kTailG, src = sub * kTailG;
         for (int f = 0; f < nfrag; f++) {
             const FragPtrs& F = c.f[f];
@@ -1865,6 +1872,10 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         {
             // the CTA's buffered appends: one reservation per target fragment's next list, then a copy
             __syncthreads();
+            unsigned any = 0;
+            for (int f = 0; f < nfrag; f++) any |= s_app_n[f];
+            if (any)  // CTA-uniform (read after the barrier); nothing buffered: no reservation, no copy
+        {
             if (threadIdx.x < (unsigned)nfrag) {
                 const unsigned f = threadIdx.x;
                 const unsigned na = s_app_n[f] < s_app_lim[f] ? s_app_n[f] : s_app_lim[f];
@@ -1872,11 +1883,11 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                     s_app_base[f] = atomicAdd(&c.f[f].ctl->tcnt[ns], na);
                     atomicAdd(&c.f[f].ctl->tedges[ns], s_app_e[f]);
                 }
-                s_app_n[f] = na;  // (the valid prefix to copy)
+                s_app_na[f] = na;  // (the valid prefix to copy; s_app_n stays as read by every thread above)
             }
             __syncthreads();
             for (int f = 0; f < nfrag; f++) {
-                const unsigned na = s_app_n[f];
+                const unsigned na = s_app_na[f];
                 unsigned* nxt = (it & 1) ? c.f[f].q_v : c.f[f].app;
                 for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base[f] + i] = s_app[f * app_cap + i];
             }
@@ -1886,6 +1897,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 s_app_lim[threadIdx.x] = app_cap;
                 s_app_e[threadIdx.x] = 0;
             }
+        }
         }
         if (tr && k < (unsigned)kTraceMax) {
             it_edges = warp_sum_u64(it_edges);  // (group leaders hold the counts)

@@ -23,6 +23,7 @@ ap.add_argument("--rmat", type=int, default=0, help="instead of --config: RMAT o
 ap.add_argument("--noscramble", action="store_true")
 ap.add_argument("--grid", type=int, default=0, help="instead of --config: n x n grid (seed 3), source 0")
 ap.add_argument("--osteal-threshold", type=int, default=0)
+ap.add_argument("--tail", type=int, default=None, help="tail engine threshold (default: bench.py's choice)")
 ap.add_argument("--delta", type=int, default=None, help="SSSP near-far split (default: bench.py's, 4096 on C3)")
 a = ap.parse_args()
 if a.grid:
@@ -36,8 +37,10 @@ else:
     s = 0 if a.config == "C3" else inputs.pick_source(g, int(a.config[1]))
 rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
 delta = a.delta if a.delta is not None else (4096 if a.config == "C3" and a.alg == "sssp" else 0)
+tail = a.tail if a.tail is not None else (0 if a.alg == "bfs" and a.config in ("C1", "C2") and not (a.rmat or a.grid)
+                                          else 16384)
 with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop), sssp_delta=delta,
-                 osteal_threshold=a.osteal_threshold) as ctx:
+                 osteal_threshold=a.osteal_threshold, tail_vertices=tail) as ctx:
     ctx.load_csr(rp, col, w)
     ctx.partition(a.part, 1)
     ctx.prepare(a.alg)
