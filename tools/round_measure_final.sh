@@ -19,7 +19,7 @@ for cfg in "C2 bfs degree" "C4 wcc seg" "C5 pr seg"; do set -- $cfg
   timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:k_advance --csv --log-file $O/traffic_$1_$2.csv $P --config $1 --alg $2 --part $3 > /dev/null 2>&1
 done
 echo "ncu lists done"
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_advance -s 2 -c 1 -o $O/adv_C2_bfs $P --config C2 --alg bfs --part degree > /dev/null 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_advance -s 3 -c 1 -o $O/adv_C2_bfs $P --config C2 --alg bfs --part degree > /dev/null 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_filter -s 2 -c 1 -o $O/filt_C2_bfs $P --config C2 --alg bfs --part degree > /dev/null 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_advance -s 10 -c 1 -o $O/adv_C5_pr $P --config C5 --alg pr > /dev/null 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_tail -s 40 -c 1 -o $O/tail_C3_sssp $P --config C3 --alg sssp > /dev/null 2>&1

@@ -11,5 +11,5 @@ for f in C1 C2 C3 C4; do python -c "import json; d=json.loads(open('$O/bench_$f.
 P="python tools/profile_run.py --runs 1"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_C2_bfs.csv $P --config C2 --alg bfs --part degree > /dev/null 2>&1
 timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:k_advance --csv --log-file $O/traffic_C2_bfs.csv $P --config C2 --alg bfs --part degree > /dev/null 2>&1
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_advance -s 2 -c 1 -o $O/adv_C2_bfs $P --config C2 --alg bfs --part degree > /dev/null 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_advance -s 3 -c 1 -o $O/adv_C2_bfs $P --config C2 --alg bfs --part degree > /dev/null 2>&1
 echo done
