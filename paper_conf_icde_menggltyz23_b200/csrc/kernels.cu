@@ -460,6 +460,89 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
     return mine;
 }
 
+// Pass 2 of one dense tile without the near-far split (acceptance = out-degree > 0): the count, the
+// block scan for the per-thread offsets and the emit in one walk of the tile (FT_COUNT + FT_EMIT read the
+// bitmap word and the row_ptr run twice). Only the 8-bit accepted mask stays live across the scan; the
+// row_ptr run is re-read after it from L1 (the same thread's lines). Returns the tile's totals.
+__device__ __forceinline__ Pair filter_tile_dense_fused(const FragPtrs& F, bool keep_fbm, unsigned depth, unsigned tile,
+                                                        unsigned nwords, unsigned chunk, unsigned long long pos,
+                                                        unsigned long long off, Pair* s_warp) {
+    const unsigned lane = lane_id();
+    const unsigned wbase = tile * kDenseWordsPerPart + (threadIdx.x >> 5) * kDenseWordsPerWarp;
+    const unsigned vb = wbase * 32u + lane * kDenseVertsPerThread;
+    const unsigned wi = wbase + (lane >> 2);
+    const bool full = vb + kDenseVertsPerThread <= F.V;
+    const unsigned word = wi < nwords ? F.bm[wi] : 0u;
+    __syncwarp();
+    if ((lane & 3u) == 0 && wi < nwords) {
+        if (keep_fbm) F.far[wi] = word;
+        if (word) F.bm[wi] = 0u;
+    }
+    const unsigned bits = (word >> ((lane & 3u) * 8u)) & 0xFFu;
+    if (depth != GUM_INF && bits) {
+        if (full) {
+            uint4* sp = reinterpret_cast<uint4*>(F.state + vb);
+            uint4 a = bits == 0xFFu ? make_uint4(0, 0, 0, 0) : __ldcg(sp);
+            uint4 b = bits == 0xFFu ? make_uint4(0, 0, 0, 0) : __ldcg(sp + 1);
+            if (bits & 1u) a.x = depth;
+            if (bits & 2u) a.y = depth;
+            if (bits & 4u) a.z = depth;
+            if (bits & 8u) a.w = depth;
+            if (bits & 16u) b.x = depth;
+            if (bits & 32u) b.y = depth;
+            if (bits & 64u) b.z = depth;
+            if (bits & 128u) b.w = depth;
+            if (bits & 0x0Fu) sp[0] = a;
+            if (bits & 0xF0u) sp[1] = b;
+        } else {
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread; q++)
+                if ((bits >> q) & 1u) F.state[vb + q] = depth;
+        }
+    }
+    const unsigned long long* rp = F.row_ptr + vb;
+    Pair mine{0, 0};
+    unsigned ok = 0;
+    if (bits) {
+        unsigned long long rpv[kDenseVertsPerThread + 1];
+        if (full) {
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread / 2; q++) {
+                const ulonglong2 t2 = __ldg(reinterpret_cast<const ulonglong2*>(rp) + q);
+                rpv[2 * q] = t2.x;
+                rpv[2 * q + 1] = t2.y;
+            }
+            rpv[kDenseVertsPerThread] = __ldg(rp + kDenseVertsPerThread);
+        } else {
+#pragma unroll
+            for (int q = 0; q <= kDenseVertsPerThread; q++) rpv[q] = (vb + q <= F.V) ? __ldg(rp + q) : 0ull;
+        }
+#pragma unroll
+        for (int q = 0; q < kDenseVertsPerThread; q++) {
+            if (((bits >> q) & 1u) && rpv[q + 1] != rpv[q]) {
+                ok |= 1u << q;
+                mine.cnt += 1;
+                mine.deg += rpv[q + 1] - rpv[q];
+            }
+        }
+    }
+    Pair tot;
+    const Pair tex = block_excl_scan(mine, s_warp, tot);
+    if (ok) {
+        unsigned long long p = pos + tex.cnt, o = off + tex.deg;
+#pragma unroll
+        for (int q = 0; q < kDenseVertsPerThread; q++) {
+            if ((ok >> q) & 1u) {
+                const unsigned long long r0 = __ldg(rp + q), r1 = __ldg(rp + q + 1);
+                emit_vertex(F, chunk, vb + q, r0, r1 - r0, p, o);
+                p += 1;
+                o += r1 - r0;
+            }
+        }
+    }
+    return tot;
+}
+
 // a4 filter / frontier generation (Example 4 Step 1; Alg. 1's degree prefix sum): the
 // fragment's activations (bitmap words when dense, the activation list when sparse) -> queue of
 // vertices with out-degree > 0 (q_v), exclusive out-degree prefix (q_off), col base (q_base) and the
@@ -604,6 +687,13 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     } else {
         for (unsigned t = t_lo; t < t_hi; t++) {
             const unsigned pt = (unsigned)((unsigned long long)t * stride % n_tiles);
+            if (dense && !nf) {
+                const Pair tot = filter_tile_dense_fused(F, keep_fbm, depth, pt, nwords, chunk, run_cnt, run_deg, s_warp);
+                filter_flush_long(F);
+                run_cnt += tot.cnt;
+                run_deg += tot.deg;
+                continue;
+            }
             const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
             Pair tot;
             const Pair tex = block_excl_scan(q, s_warp, tot);

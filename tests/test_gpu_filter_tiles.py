@@ -1,0 +1,36 @@
+"""Filter pass 2 over several tiles per CTA (kernels.cu k_filter, multi-tile branch; the fused dense
+tile of BFS/SSSP/WCC/PR without the near-far split). At the parity sizes of the other tests every filter
+CTA holds at most one tile; here the filter grid is cut to one CTA per SM (GUM_FILTER_CTAS_PER_SM=1, read
+once per process, hence the subprocess) so that a 2^20-vertex bitmap spans 512 dense tiles over 148 CTAs
+(stride-permuted), and the results must still equal the oracle's."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+CHILD = r"""
+import sys
+sys.path.insert(0, ROOT)
+import inputs
+from tests.gpu_helpers import check, csr_of
+g = inputs.rmat(20, 16, seed=33)
+s = inputs.pick_source(g, 33)
+csr = csr_of(g)
+for alg in ("bfs", "sssp", "wcc", "pr"):
+    for P, part in ((1, "seg"), (1, "degree"), (2, "random")):
+        check(g, alg, s, csr=csr, num_gpus=P, part=part)
+        print("ok", alg, P, part, flush=True)
+"""
+
+
+def test_filter_multi_tile_per_cta():
+    env = dict(os.environ, GUM_FILTER_CTAS_PER_SM="1")
+    r = subprocess.run([sys.executable, "-c", f"ROOT = {ROOT!r}\n" + CHILD], cwd=ROOT, env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert r.stdout.count("ok ") == 12, r.stdout

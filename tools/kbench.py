@@ -30,7 +30,7 @@ def child(a):
     out = {}
     with gum.Context(**kw) as ctx:
         ctx.load_csr(rp, col, w)
-        ctx.partition()
+        ctx.partition(a.part)
         ctx.prepare(a.alg)
         ref = {}
         for s in srcs:
@@ -43,7 +43,7 @@ def child(a):
         out["graph_ms_min"] = float(np.min(ms))
     with gum.Context(profile=True, **kw) as ctx:
         ctx.load_csr(rp, col, w)
-        ctx.partition()
+        ctx.partition(a.part)
         ctx.prepare(a.alg)
         ctx.run(a.alg, srcs[0])
         acc = {}
@@ -66,6 +66,7 @@ def main():
     ap.add_argument("--runs", type=int, default=8)
     ap.add_argument("--libs", default="")
     ap.add_argument("--kw", default="{}")
+    ap.add_argument("--part", default="seg")
     ap.add_argument("--child", action="store_true")
     a = ap.parse_args()
     if a.child:
@@ -74,7 +75,7 @@ def main():
     for lib in libs:
         env = dict(os.environ, GUM_LIB=os.path.abspath(lib))
         r = subprocess.run([sys.executable, __file__, "--child", "--config", a.config, "--alg", a.alg, "--runs",
-                            str(a.runs), "--kw", a.kw], env=env, capture_output=True, text=True)
+                            str(a.runs), "--kw", a.kw, "--part", a.part], env=env, capture_output=True, text=True)
         line = [x for x in r.stdout.splitlines() if x.startswith("KBENCH ")]
         print(os.path.basename(lib), line[0][7:] if line else ("FAILED " + r.stderr[-800:]), flush=True)
 
