@@ -22,7 +22,7 @@ inputs/libgen.so: inputs/gen.c
 	gcc -O3 -fopenmp -shared -fPIC -o $@ $<
 
 oracle/liboracle.so: oracle/oracle.c
-	gcc -O2 -shared -fPIC -o $@ $< -lm
+	gcc -O2 -fopenmp -shared -fPIC -o $@ $< -lm
 
 $(PKG)/libgum.so: $(GUM_SRCS) $(GUM_HDRS)
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(GUM_SRCS) -lgomp 2> build/ptxas.log || (cat build/ptxas.log; false)

@@ -42,6 +42,9 @@ def _load():
     lib.oracle_pagerank.restype = ctypes.c_int
     lib.oracle_pagerank.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_int, ctypes.c_double,
                                     pd, pd]
+    lib.oracle_pagerank_pull.restype = ctypes.c_int
+    lib.oracle_pagerank_pull.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_int, ctypes.c_double,
+                                         ctypes.c_int, pd, pd, ctypes.POINTER(ctypes.c_int)]
     _lib = lib
     return lib
 
@@ -122,6 +125,23 @@ def pagerank(V, src, dst, iterations=20, damping=0.85, return_residuals=False):
     if return_residuals:
         return x, r[:iterations]
     return x
+
+
+def pagerank_pull(V, src, dst, iterations=20, damping=0.85, threads=0, return_residuals=False):
+    """OpenMP pull variant of ``pagerank``: same x_K (same terms, same per-vertex sum
+    order); returns (x, threads_used) or (x, residuals, threads_used)."""
+    src, dst = _u32(src), _u32(dst)
+    x = np.empty(int(V), dtype=np.float64)
+    r = np.empty(max(iterations, 1), dtype=np.float64)
+    used = ctypes.c_int(0)
+    rc = _load().oracle_pagerank_pull(int(V), int(src.shape[0]), _p(src, ctypes.c_uint32), _p(dst, ctypes.c_uint32),
+                                      int(iterations), float(damping), int(threads), _p(x, ctypes.c_double),
+                                      _p(r, ctypes.c_double), ctypes.byref(used))
+    if rc != 0:
+        raise ValueError(f"oracle_pagerank_pull rc={rc}")
+    if return_residuals:
+        return x, r[:iterations], used.value
+    return x, used.value
 
 
 def run(alg: str, g, source: int = 0, pr_iterations: int = 20, pr_damping: float = 0.85):

@@ -25,12 +25,15 @@
  * networkx.pagerank, brute force (Floyd-Warshall, reachability powers, dense PR) on tiny graphs.
  * No function here is "parity unpinned".
  *
- * Build: gcc -O2 -shared -fPIC (single-threaded by design; SURVEY.md §8(d) "Oracle timing").
+ * Build: gcc -O2 -fopenmp -shared -fPIC. Every function is single-threaded by design (SURVEY.md §8(d)
+ * "Oracle timing") except oracle_pagerank_pull, the OpenMP variant §8(d) allows for full-size PR
+ * checks ("an optional OpenMP pull variant reports its thread count").
  */
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
 #include <math.h>
+#include <omp.h>
 
 #define ORACLE_INF 0xFFFFFFFFu
 
@@ -203,5 +206,74 @@ int oracle_pagerank(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t*
     free(outdeg);
     free(x);
     free(y);
+    return 0;
+}
+
+/* ---- c-4 PageRank, OpenMP pull variant ("an optional OpenMP pull variant reports its
+ * thread count"). The same recurrence as oracle_pagerank, computed per destination:
+ *   y[v] = sum over the in-edges (u, v) of x_k[u]/outdeg(u)
+ * with the in-edges of v taken from a STABLE counting sort of the raw edge list by destination, i.e. in
+ * increasing edge index -- the order in which oracle_pagerank's edge loop adds them into y[v]. Each term
+ * is the same double (x[u]/outdeg(u), one division) and each sum has the same order, so x_K is identical
+ * to oracle_pagerank's (D_k is summed serially in vertex order as there); only the residual is reduced
+ * in another order (pinned in tests/test_oracle.py). nthreads <= 0 => omp_get_max_threads(); *threads_used reports it.           */
+int oracle_pagerank_pull(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, int K, double d,
+                         int nthreads, double* x_out, double* resid, int* threads_used) {
+    if (V == 0) return 0;
+    const int T = nthreads > 0 ? nthreads : omp_get_max_threads();
+    if (threads_used) *threads_used = T;
+    uint64_t* outdeg = (uint64_t*)calloc((size_t)V, sizeof(uint64_t));
+    uint64_t* in_ptr = (uint64_t*)calloc((size_t)V + 1, sizeof(uint64_t));
+    uint32_t* in_src = (uint32_t*)malloc(sizeof(uint32_t) * (size_t)(E ? E : 1));
+    double* x = (double*)malloc(sizeof(double) * V);
+    double* cx = (double*)malloc(sizeof(double) * V);
+    double* y = (double*)malloc(sizeof(double) * V);
+    if (!outdeg || !in_ptr || !in_src || !x || !cx || !y) {
+        free(outdeg); free(in_ptr); free(in_src); free(x); free(cx); free(y);
+        return -2;
+    }
+    for (uint64_t i = 0; i < E; i++) {
+        if (src[i] >= V || dst[i] >= V) {
+            free(outdeg); free(in_ptr); free(in_src); free(x); free(cx); free(y);
+            return -1;
+        }
+        outdeg[src[i]]++;
+        in_ptr[dst[i] + 1]++;
+    }
+    for (uint32_t v = 0; v < V; v++) in_ptr[v + 1] += in_ptr[v];
+    {
+        uint64_t* fill = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)V);
+        if (!fill) {
+            free(outdeg); free(in_ptr); free(in_src); free(x); free(cx); free(y);
+            return -2;
+        }
+        memcpy(fill, in_ptr, sizeof(uint64_t) * (size_t)V);
+        for (uint64_t i = 0; i < E; i++) in_src[fill[dst[i]]++] = src[i]; /* stable: edge order per v */
+        free(fill);
+    }
+    for (uint32_t v = 0; v < V; v++) x[v] = 1.0 / (double)V;
+    for (int k = 0; k < K; k++) {
+        double D = 0.0; /* serial, in vertex order: the same D_k as oracle_pagerank */
+        for (uint32_t u = 0; u < V; u++)
+            if (outdeg[u] == 0) D += x[u];
+#pragma omp parallel for num_threads(T) schedule(static)
+        for (int64_t u = 0; u < (int64_t)V; u++) cx[u] = outdeg[u] ? x[u] / (double)outdeg[u] : 0.0;
+#pragma omp parallel for num_threads(T) schedule(dynamic, 4096)
+        for (int64_t v = 0; v < (int64_t)V; v++) {
+            double acc = 0.0;
+            for (uint64_t e = in_ptr[v]; e < in_ptr[v + 1]; e++) acc += cx[in_src[e]];
+            y[v] = acc;
+        }
+        double r = 0.0;
+#pragma omp parallel for num_threads(T) schedule(static) reduction(+ : r)
+        for (int64_t v = 0; v < (int64_t)V; v++) {
+            double nx = (1.0 - d) / (double)V + d * (y[v] + D / (double)V);
+            r += fabs(nx - x[v]);
+            x[v] = nx;
+        }
+        if (resid) resid[k] = r;
+    }
+    memcpy(x_out, x, sizeof(double) * V);
+    free(outdeg); free(in_ptr); free(in_src); free(x); free(cx); free(y);
     return 0;
 }

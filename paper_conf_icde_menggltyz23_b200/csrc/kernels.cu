@@ -726,7 +726,11 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
             }
             const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
             Pair tot;
-            const Pair tex = block_excl_scan_tile(q, s_warp, tot);  // one tile: <= 2048 entries
+#ifdef GUM_PACK2
+            const Pair tex = block_excl_scan_tile(q, s_warp, tot);  // A/B variant "pack2" (filter 0.390 ms/run on C2)
+#else
+            const Pair tex = block_excl_scan(q, s_warp, tot);  // "pack": packed scan in the fused dense tile only (0.384)
+#endif
             filter_tile<FT_EMIT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
                                  run_deg + tex.deg);
             filter_flush_long(F);

@@ -358,3 +358,32 @@ def test_pr_residuals_decrease_geometrically():
     g = inputs.rmat(11, 8, seed=7, weighted=False)
     _, r = oracle.pagerank(g.num_vertices, g.src, g.dst, 20, 0.85, return_residuals=True)
     assert np.all(r[1:] <= r[:-1] * 0.85 + 1e-15)
+
+
+# ---- OpenMP pull variant: pinned to the serial power iteration and to the matrix form
+def test_pr_pull_equals_serial_rmat16_k20():
+    g = inputs.rmat(16, 16, seed=1, weighted=False)
+    x, r, used = oracle.pagerank_pull(g.num_vertices, g.src, g.dst, 20, 0.85, threads=4, return_residuals=True)
+    xs, rs = oracle.pagerank(g.num_vertices, g.src, g.dst, 20, 0.85, return_residuals=True)
+    assert used == 4
+    # same terms summed in the same per-vertex order (stable in-edge sort): bit-identical x_K
+    assert np.array_equal(x, xs)
+    assert float(np.max(np.abs(x - xs) / xs)) <= 1e-13
+    assert np.allclose(r, rs, rtol=1e-10, atol=0)
+
+
+@settings(max_examples=20, deadline=None)
+@given(st.integers(1, 40), st.integers(0, 160), st.integers(0, 2**32 - 1), st.integers(0, 22), st.integers(1, 5))
+def test_pr_pull_vs_dense_matrix(V, E, seed, K, T):
+    rng = np.random.default_rng(seed)
+    g = random_graph(rng, V, E)
+    x, used = oracle.pagerank_pull(V, g.src, g.dst, K, 0.85, threads=T)
+    assert used == T
+    assert np.allclose(x, dense_pagerank(g, K, 0.85), rtol=1e-12, atol=1e-15)
+
+
+def test_pr_pull_torus_uniform():
+    g = inputs.torus(48)
+    x, _ = oracle.pagerank_pull(g.num_vertices, g.src, g.dst, 20, 0.85, threads=3)
+    assert np.allclose(x, 1.0 / g.num_vertices, rtol=1e-13, atol=0)
+    assert abs(x.sum() - 1.0) < 1e-12
