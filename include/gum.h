@@ -155,6 +155,12 @@ typedef struct {
     int mirrors;
     int hub_cache;
     uint32_t hub_degree;
+    /* PageRank advance (a8 for PR). 0 (default): pull -- every vertex sums x[u]/outdeg(u) over its in-edges,
+     * one pass per L2-sized block of sources, rows and edges balanced by merge path; the sum is the same
+     * set of terms as the push ("PR pull"). 1: push -- one red.add.f64 of x[u]/outdeg(u) per
+     * out-edge into the destination's accumulator (the GAS scatter of P:53; also used whenever mirrors = 1,
+     * whose aggregation is a push). Results agree within the PR tolerance either way. */
+    int pr_push;
 } gum_config;
 
 /* Fills *cfg with the defaults: 1 worker, fsteal=1, osteal=1, t1=t2=0, osteal threshold 0 (off until

@@ -60,7 +60,8 @@ class gum_config(ctypes.Structure):
                 ("osteal_sync_edges", ctypes.c_double),
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p)),
-                ("mirrors", ctypes.c_int), ("hub_cache", ctypes.c_int), ("hub_degree", ctypes.c_uint32)]
+                ("mirrors", ctypes.c_int), ("hub_cache", ctypes.c_int), ("hub_degree", ctypes.c_uint32),
+                ("pr_push", ctypes.c_int)]
 
 
 EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p)
@@ -204,7 +205,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=16384,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
                 use_torch_allocator=False, streams=None, osteal_sync_edges=0.0, mirrors=False, hub_cache=False,
-                hub_degree=0):
+                hub_degree=0, pr_push=False):
     """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
     config points to and must live as long as the context."""
     lib = load_library()
@@ -235,6 +236,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
     cfg.mirrors = int(bool(mirrors))          # NEXT-1 outer-vertex mirrors
     cfg.hub_cache = int(bool(hub_cache))      # NEXT-1 hub adjacency caching
     cfg.hub_degree = int(hub_degree)          # t4
+    cfg.pr_push = int(bool(pr_push))          # PR advance: pull over source blocks (default) or push
     flags = 0
     if trace:
         flags |= CFG_TRACE

@@ -28,6 +28,11 @@ constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;
 constexpr int kPbMaxBins = 1024;       // propagation blocking: max destination blocks per fragment
 constexpr unsigned kPrPiece = 64;      // PR warp-task path: max edges per queue entry
+#ifndef GUM_PULL_IPT
+#define GUM_PULL_IPT 8
+#endif
+constexpr int kPullIPT = GUM_PULL_IPT;              // PR pull: merge-path items (rows + edges) per thread
+constexpr int kPullTile = kThreads * kPullIPT;       // PR pull: merge-path items per CTA tile
 
 // Per-fragment control block (fragment memory, peer-visible). Counters that thieves touch
 // (claim) and that the filter publishes (qlen, qedges, ntiles) live here.
@@ -152,6 +157,15 @@ struct FragPtrs {
     const unsigned long long* sq_q_off;
     const unsigned int* sq_tile;
     unsigned long long sq_len, sq_edges;
+    // PR pull (default PR advance): the fragment's in-edges regrouped source-block-major.
+    // Pass b covers the sources [b*S, (b+1)*S) (an L2-sized block of x/outdeg); its rows are this fragment's
+    // vertices: row i = pl_col[pl_off[b*V + i] .. pl_off[b*V + i + 1]) (global source ids, absolute u32
+    // offsets). pl_tx[pl_tb[b] + t] = first row of merge-path tile t of pass b (pl_tb[b+1] - pl_tb[b] - 1
+    // tiles; the last entry is V).
+    const unsigned* pl_off;
+    const unsigned* pl_col;
+    const unsigned* pl_tx;
+    const unsigned long long* pl_tb;
     // NEXT-1 outer-vertex mirror of worker f (this fragment's memory), indexed by GLOBAL id; only
     // vertices of other fragments are ever touched ("outer" vertices)
     double* macc;                       // PR: [V] aggregated pushes to other fragments' vertices
@@ -206,6 +220,14 @@ struct DevCtx {
                                     // activations (the advance only sets visited / frontier bits)
     unsigned int wcc_blocked;     // WCC static destination-blocked queue exists: dense iterations may run on
                                   // it (the filter keeps the frontier bitmap in F.far)
+    // PR pull: pl_B source-block passes per iteration; every launch unit keeps a replica of the global
+    // x/outdeg vector, double-buffered by iteration parity ([2][num_vertices] doubles): the finalize of
+    // fragment f writes its slice into every replica (cxrep[0..n_rep)), the pull of worker w reads cxw[w]
+    // (its unit's replica). 0 passes = push (k_advance with red.add.f64).
+    unsigned pl_B;
+    int n_rep;
+    double* cxrep[kMaxW];
+    const double* cxw[kMaxW];
     int hub_on;                 // NEXT-1 hub cache built for this algorithm
     HubPtrs hub[kMaxW][kMaxW];  // [worker][fragment] (fragment != worker)
 };

@@ -49,6 +49,15 @@ __device__ __forceinline__ unsigned lanemask_lt() {
     return m;
 }
 
+__host__ __device__ __forceinline__ unsigned gcd_u32(unsigned a, unsigned b) {
+    while (b) {
+        const unsigned t = a % b;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
 // owner fragment of a global (relabelled) vertex id: <= 7 compares ("global to local id").
 __device__ __forceinline__ int frag_of(const DevCtx& c, unsigned v) {
     int f = 0;
@@ -75,6 +84,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
                 F.x[i] = x0;
                 F.acc[i] = 0.0;
                 F.cx[i] = od ? x0 / (double)od : 0.0;  // the contribution x/outdeg pushed along out-edges
+                for (int r = 0; r < c.n_rep; r++) c.cxrep[r][F.base + i] = F.cx[i];  // pull replicas, buffer 0
             }
         }
         if (i < nwords) {
@@ -209,6 +219,8 @@ __device__ __forceinline__ Pair block_excl_scan(Pair v, Pair* s_warp, Pair& tota
 // Block scan of one filter tile's (count, degree) pairs packed into one u64: a tile holds <= 2048
 // accepted vertices (12 bits) and a degree sum < 2^52 edges, so each step is one 64-bit shuffle instead
 // of two (C2 filter 0.396 -> 0.383 ms per run). Same contract as block_excl_scan.
+static_assert(kThreads * kDenseVertsPerThread < 4096 && kThreads * kFilterAppPerThread < 4096,
+              "block_excl_scan_tile keeps a tile's count in 12 bits");
 __device__ __forceinline__ Pair block_excl_scan_tile(Pair v, Pair* s_warp, Pair& total) {
     constexpr unsigned kCntShift = 52;
     constexpr unsigned long long kDegMask = (1ull << kCntShift) - 1;
@@ -661,8 +673,8 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     // few CTAs. The queue order is then a permutation of vertex order (nothing depends on it being sorted).
     unsigned stride = 1;
     if (c.filter_swizzle && n_tiles > 2u * G) {
-        stride = 2053u;  // prime
-        while (stride > 1 && n_tiles % stride == 0) stride += 2;
+        stride = 2053u;  // start at a prime; step until gcd(stride, n_tiles) == 1 (a bijection on the tiles)
+        while (stride < n_tiles && gcd_u32(stride, n_tiles) != 1u) stride++;
         if (stride >= n_tiles) stride = 1;
     }
 
@@ -1029,6 +1041,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     typedef typename ValT<ALG>::T VT;
     __shared__ unsigned s_base[kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
+    static_assert(kTileMax <= 4096, "s_head tags keep the vertex slot in 12 bits");
     __shared__ __align__(16) unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
     // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
     constexpr int PBB = (ALG == ALG_BFS && !MULTI && PB) ? kPbMaxBins : 1;  // (own instantiation:
@@ -2411,16 +2424,207 @@ cudaError_t pr_push_occupancy(int* blocks_per_sm) {
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_pr_push, kThreads, 0);
 }
 
+// ------------------------------------------------------------------------------------------ PR pull
+// a8 for PageRank as a pull: pass b gathers, for every vertex v of the fragment, the sum of
+// x[u]/outdeg(u) over v's in-edges whose source u lies in source block b (an L2-resident slice of the
+// unit's replica of x/outdeg) and adds it to acc[v]; the finalize then forms x' = (1-d)/V + d(acc + D/V)
+// as for the push (same terms, summed in another order). Rows and edges of a pass are balanced over CTAs
+// by merge path (Merrill & Garland's SpMV): a tile is kPullTile consecutive items of the merge of row ends
+// and edge indices. Per tile the CTA first stages, with coalesced loads and every gather of a thread in
+// flight at once, the tile's edge values x[u]/outdeg(u), its row ends and its rows' accumulators into
+// shared memory; then thread t walks kPullIPT items of the merge. A row that ends in a thread after that
+// thread's first row lies entirely inside the thread and is stored once (acc + sum); partial rows are
+// carried between threads by a block-wide segmented scan, and only rows that cross a tile boundary use a
+// global fp64 atomic: <= 2 atomics per tile instead of one red.add.f64 per edge.
+// (A three-stage cp.async pipeline -- ids, then 8-byte async gathers, then the reduction -- measured 2x
+// slower on C5: DESIGN.md §6.)
+__global__ void __launch_bounds__(kThreads) k_pr_pull(const __grid_constant__ DevCtx c, int w0, int nw, int pass) {
+    __shared__ unsigned s_re[kPullTile + 1];  // row ends (relative to the pass's first edge) of the tile's rows
+    __shared__ double s_val[kPullTile];       // x[u]/outdeg(u) of the tile's edges
+    __shared__ double s_acc[kPullTile + 1];   // acc of the tile's rows (rows x0 .. x1)
+    __shared__ unsigned s_key[kThreads];
+    __shared__ double s_inc[kThreads];
+    __shared__ unsigned s_wkey[kThreads / 32], s_ckey[kThreads / 32];
+    __shared__ double s_wval[kThreads / 32], s_cval[kThreads / 32];
+    __shared__ unsigned s_tx[3];
+    struct Pro {
+        unsigned go, buf, owner, k;
+        unsigned long long tb0, ntiles, t0;
+    };
+    __shared__ Pro s_pro;
+    RunCtl* rc = c.rctl[w0];
+    const int f = blockIdx.y;
+    const FragPtrs& F = c.f[f];
+    const unsigned Vf = F.V;
+    const unsigned* off = F.pl_off + (size_t)pass * Vf;
+    if (threadIdx.x == 0) {
+        Pro p{};
+        p.owner = vload(&rc->owner[f]);
+        p.go = !vload(&rc->done) && (int)p.owner >= w0 && (int)p.owner < w0 + nw;
+        if (p.go) {
+            p.k = vload(&rc->iter) - 1u;
+            p.buf = p.k & 1u;  // iteration k reads x_k/outdeg (control set iter = k+1)
+            p.t0 = globaltimer();
+            p.tb0 = F.pl_tb[pass];
+            p.ntiles = F.pl_tb[pass + 1] - p.tb0 - 1;
+        }
+        s_pro = p;
+    }
+    __syncthreads();
+    if (!s_pro.go) return;
+    const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
+    const unsigned ebase = __ldg(off);
+    const unsigned long long items = (unsigned long long)Vf + (__ldg(off + Vf) - ebase);
+    const double* cx = c.cxw[s_pro.owner] + (size_t)s_pro.buf * c.num_vertices;
+    const unsigned* pcol = F.pl_col + ebase;
+    double* acc = F.acc;
+    const unsigned long long tb0 = s_pro.tb0, ntiles = s_pro.ntiles;
+    unsigned long long edges = 0;
+    // tile-table entries of the next tile are loaded one tile ahead (threads 0 and 1)
+    unsigned nx_tx = 0;
+    if (threadIdx.x < 2 && blockIdx.x < ntiles) nx_tx = __ldg(F.pl_tx + tb0 + blockIdx.x + threadIdx.x);
+    for (unsigned long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        if (threadIdx.x < 2) {
+            s_tx[threadIdx.x] = nx_tx;
+            const unsigned long long tn = t + gridDim.x;
+            if (tn < ntiles) nx_tx = __ldg(F.pl_tx + tb0 + tn + threadIdx.x);
+        }
+        __syncthreads();
+        const unsigned x0 = s_tx[0], x1 = s_tx[1];
+        const unsigned long long d0 = t * kPullTile;
+        const unsigned long long d1 = d0 + kPullTile < items ? d0 + kPullTile : items;
+        const unsigned y0 = (unsigned)(d0 - x0), y1 = (unsigned)(d1 - x1);
+        const unsigned ne_t = y1 - y0;
+        // stage: edge values (coalesced col ids, all gathers of a thread issued back to back), row ends and
+        // the accumulators of rows x0 .. min(x1, Vf-1), row x0's start
+        {
+            unsigned cu[kPullIPT];
+#pragma unroll
+            for (int j = 0; j < kPullIPT; j++) {
+                const unsigned e = threadIdx.x + j * kThreads;
+                cu[j] = e < ne_t ? __ldcs(pcol + y0 + e) : 0u;
+            }
+#pragma unroll
+            for (int j = 0; j < kPullIPT; j++) {
+                const unsigned e = threadIdx.x + j * kThreads;
+                if (e < ne_t) s_val[e] = __ldg(cx + cu[j]);
+            }
+        }
+        const unsigned nr = (x1 < Vf ? x1 : Vf - 1u) - x0 + 1u;
+        for (unsigned i = threadIdx.x; i < nr; i += kThreads) {
+            s_re[i] = __ldg(off + x0 + i + 1) - ebase;
+            s_acc[i] = __ldcg(acc + x0 + i);
+        }
+        if (threadIdx.x == kThreads - 1) s_tx[2] = __ldg(off + x0) - ebase;
+        __syncthreads();
+        edges += ne_t;  // (the same tile total in every thread; thread 0's is flushed)
+        // this thread's merge-path coordinate inside the tile
+        const unsigned tl = (unsigned)(d1 - d0);
+        const unsigned dl = threadIdx.x * kPullIPT < tl ? threadIdx.x * kPullIPT : tl;
+        const unsigned ni = tl - dl < (unsigned)kPullIPT ? tl - dl : (unsigned)kPullIPT;
+        unsigned lo = dl > ne_t ? dl - ne_t : 0u, hi = dl < x1 - x0 ? dl : x1 - x0;
+        while (lo < hi) {
+            const unsigned mid = (lo + hi) >> 1;
+            if (s_re[mid] <= y0 + (dl - mid) - 1u) lo = mid + 1u;
+            else hi = mid;
+        }
+        const unsigned xs = x0 + lo, ys = y0 + dl - lo;
+        // walk: a row that ends in this thread after its first row is complete here -> one store
+        double sum = 0.0, first_sum = 0.0;
+        bool has_first = false;
+        unsigned xi = xs, yi = ys;
+#pragma unroll
+        for (int k = 0; k < kPullIPT; k++) {
+            if ((unsigned)k < ni) {
+                if (yi < s_re[xi - x0]) {
+                    sum += s_val[yi - y0];
+                    yi++;
+                } else {
+                    if (!has_first) {
+                        has_first = true;
+                        first_sum = sum;
+                    } else if (sum != 0.0) {
+                        acc[xi] = s_acc[xi - x0] + sum;
+                    }
+                    sum = 0.0;
+                    xi++;
+                }
+            }
+        }
+        // block-wide inclusive segmented scan of the carry-outs (key = row in progress; keys are monotone)
+        unsigned key = xi;
+        double val = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const double v2 = __shfl_up_sync(0xffffffffu, val, o);
+            const unsigned k2 = __shfl_up_sync(0xffffffffu, key, o);
+            if (lane >= (unsigned)o && k2 == key) val += v2;
+        }
+        if (lane == 31) {
+            s_wkey[wid] = key;
+            s_wval[wid] = val;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned ck = 0xFFFFFFFFu;
+            double cv = 0.0;
+            for (int w = 0; w < kThreads / 32; w++) {
+                s_ckey[w] = ck;
+                s_cval[w] = cv;
+                if (s_wkey[w] == ck) {
+                    cv += s_wval[w];
+                } else {
+                    ck = s_wkey[w];
+                    cv = s_wval[w];
+                }
+            }
+        }
+        __syncthreads();
+        if (key == s_ckey[wid]) val += s_cval[wid];
+        s_key[threadIdx.x] = key;
+        s_inc[threadIdx.x] = val;
+        __syncthreads();
+        if (has_first) {
+            // this thread's first row: add what earlier threads of the tile carried into it; a row that
+            // began in an earlier tile gets the rest from that tile's atomic, so it is added atomically too
+            double tot = first_sum;
+            if (threadIdx.x > 0 && s_key[threadIdx.x - 1] == xs) tot += s_inc[threadIdx.x - 1];
+            if (xs == x0 && s_tx[2] < y0) {
+                if (tot != 0.0) atomicAdd(acc + xs, tot);
+            } else if (tot != 0.0) {
+                acc[xs] = s_acc[xs - x0] + tot;
+            }
+        }
+        if (threadIdx.x == kThreads - 1 && key < Vf && val != 0.0) atomicAdd(acc + key, val);  // continues in t+1
+    }
+    if (threadIdx.x == 0 && edges) {
+        atomicAdd(&F.ctl->edges_done, edges);
+        gum_iter_trace* tr = c.trace[w0];
+        const unsigned k = s_pro.k, o = s_pro.owner;
+        if (tr && k < (unsigned)kTraceMax) {  // per-worker busy window and edges (trace)
+            atomicAdd((unsigned long long*)&tr[k].edges_own[o], edges);
+            atomicMin((unsigned long long*)&tr[k].t_start[o], s_pro.t0);
+            atomicMax((unsigned long long*)&tr[k].t_end[o], globaltimer());
+        }
+    }
+}
+
+cudaError_t pr_pull_occupancy(int* blocks_per_sm) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_pr_pull, kThreads, 0);
+}
+
 // ------------------------------------------------------------------------------------------ PR finalize
 __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant__ DevCtx c, int w0, int nw) {
     RunCtl* rc = c.rctl[w0];
     const int f = blockIdx.y;
     __shared__ unsigned s_go;  // prologue by one thread per CTA (hot run-control addresses)
     __shared__ double s_D;
+    __shared__ unsigned s_nbuf;
     if (threadIdx.x == 0) {
         const unsigned o = vload(&rc->owner[f]);
         s_go = !vload(&rc->done) && (int)o >= w0 && (int)o < w0 + nw;
         s_D = vload(&rc->pr_D);
+        s_nbuf = vload(&rc->iter) & 1u;
     }
     __syncthreads();
     if (!s_go) return;
@@ -2432,6 +2636,7 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
         for (int q = 0; q < kMaxW; q++) F.ctl->pclaim[q] = 0;
     }
     const double N = (double)c.num_vertices, d = c.pr_d, D = s_D;
+    const unsigned nbuf = s_nbuf;  // PR pull replicas: x_{k+1}/outdeg goes to buffer (k+1)&1
     double dang = 0.0, res = 0.0;
     const bool mir = c.mirrors && c.P > 1;
     for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < F.V; i += gridDim.x * blockDim.x) {
@@ -2452,8 +2657,10 @@ __global__ void __launch_bounds__(kThreads) k_pr_finalize(const __grid_constant_
         const unsigned long long od = __ldg(F.row_ptr + i + 1) - __ldg(F.row_ptr + i);
         if (od == 0) dang += nx;
         F.x[i] = nx;
-        F.cx[i] = od ? nx / (double)od : 0.0;  // next iteration's push value x'/outdeg
+        const double cxv = od ? nx / (double)od : 0.0;  // next iteration's push / pull value x'/outdeg
+        F.cx[i] = cxv;
         F.acc[i] = 0.0;
+        for (int r = 0; r < c.n_rep; r++) c.cxrep[r][(size_t)nbuf * c.num_vertices + F.base + i] = cxv;
     }
 #pragma unroll
     for (int s = 16; s > 0; s >>= 1) {
@@ -2512,7 +2719,13 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
             break;
         case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
         case KER_ADVANCE:
-            if (ALG == ALG_PR && c.P == 1 && c.f[0].pr2_q_v)
+            if (ALG == ALG_PR && c.pl_B) {
+                for (unsigned b = 0; b < c.pl_B; b++) {
+                    k_pr_pull<<<dim3(L.pull_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw, (int)b);
+                    cudaError_t e = cudaGetLastError();
+                    if (e != cudaSuccess) return e;
+                }
+            } else if (ALG == ALG_PR && c.P == 1 && c.f[0].pr2_q_v)
                 k_pr_push<<<L.adv_grid_pr, kThreads, 0, s>>>(c, L.w0, L.nw);
             else if (c.P > 1)
                 if (c.mirrors || c.hub_on)

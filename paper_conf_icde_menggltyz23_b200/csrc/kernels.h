@@ -17,6 +17,7 @@ struct LaunchCfg {
     int init_grid;
     int tail_grid;    // tail engine CTAs (cooperative; 0 = engine disabled)
     int adv_grid_pr;  // PR warp-task push (single fragment): occupancy-sized grid
+    int pull_grid;    // PR pull: CTAs per fragment
 };
 
 enum { KER_FILTER = 0, KER_CONTROL = 1, KER_ADVANCE = 2, KER_FINALIZE = 3, KER_INIT = 4, KER_TAIL = 5, KER_APPLY = 6, KER_PULL = 7, KER_COUNT = 8 };
@@ -34,6 +35,7 @@ cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
 cudaError_t filter_occupancy(int* blocks_per_sm);
 cudaError_t pr_push_occupancy(int* blocks_per_sm);
+cudaError_t pr_pull_occupancy(int* blocks_per_sm);
 // PR single fragment: cut the destination-blocked queue's entries into pieces of <= piece edges
 // (q2_off gets n2 + 1 entries; *n2 = pieces). tmp sized by setup_scan_tmp_bytes(n).
 cudaError_t setup_pr_pieces_count(const unsigned long long* q_off, unsigned long long n, unsigned piece,
@@ -41,6 +43,13 @@ cudaError_t setup_pr_pieces_count(const unsigned long long* q_off, unsigned long
 cudaError_t setup_pr_pieces_emit(const unsigned* q_v, const unsigned long long* q_off, unsigned long long n,
                                  unsigned piece, const unsigned long long* pos, unsigned* q2_v,
                                  unsigned long long* q2_off, cudaStream_t s);
+// PR pull: fragment in-CSR (rows = the fragment's vertices, cols = global source ids, rebased row_ptr) ->
+// source-block-major layout with u32 offsets (pl_off[B*Vf+1]) and the per-pass merge-path tile table.
+// h_tb receives the B+1 tile-table bases (host); pl_tx must hold h_tb[B] entries (call with pl_tx = null
+// first to size it). tmp sized by setup_pr_tmp_bytes(Vf, B).
+cudaError_t setup_pr_pull(const unsigned long long* in_rp, const unsigned* in_col, unsigned Vf, unsigned long long Ein,
+                          unsigned S, int B, unsigned tile, unsigned* pl_off, unsigned* pl_col, unsigned* pl_tx,
+                          unsigned long long* h_tb, void* tmp, size_t tmp_bytes, cudaStream_t s);
 // BFS propagation blocking: static per-block capacities (in-degree histogram of the blocks) -> pb_off
 cudaError_t setup_pb_offsets(const unsigned* col, unsigned long long E, unsigned shift, unsigned nb,
                              unsigned long long* pb_off, void* tmp, size_t tmp_bytes, cudaStream_t s);

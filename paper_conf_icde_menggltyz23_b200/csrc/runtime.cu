@@ -82,6 +82,11 @@ struct FragBufs {
     unsigned* pb_buf = nullptr;
     // NEXT-1 outer-vertex mirror of this worker (V entries of 8 B; PR acc / BFS bits / SSSP-WCC min alias it)
     void* mbuf = nullptr;
+    // PR pull (gum_prepare(PR) without pr_push): source-block-major in-edges + merge-path tile table
+    unsigned* pl_off = nullptr;
+    unsigned* pl_col = nullptr;
+    unsigned* pl_tx = nullptr;
+    unsigned long long* pl_tb = nullptr;
 };
 
 // NEXT-1 hub cache: worker w's copy of fragment f's hub lists
@@ -107,6 +112,7 @@ struct gum_ctx {
     int filter_occ = 2;
     int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
     int pr_push_occ = 8;
+    int pull_occ = 4;
     std::string err;
     bool poisoned = false;
     std::vector<Alloc> load_allocs, part_allocs, misc_allocs;
@@ -132,6 +138,9 @@ struct gum_ctx {
     bool pr_ready = false;
     bool pb_ready = false;
     bool in_ready = false;
+    bool pl_ready = false;  // PR pull structures built (else PR pushes)
+    unsigned pl_B = 0;      // PR pull: source-block passes per iteration
+    double* cxg[kMaxW] = {nullptr};  // PR pull: per unit, replica of x/outdeg [2][V] (global ids)
     unsigned pb_shift = 0, pb_nb = 0;
     int pr_blocks = 1;
     FragBufs fr[kMaxW];
@@ -273,6 +282,9 @@ void drop_partition(gum_ctx* c) {
     c->pr_ready = false;
     c->pb_ready = false;
     c->in_ready = false;
+    c->pl_ready = false;
+    c->pl_B = 0;
+    for (auto& p : c->cxg) p = nullptr;
     c->pb_shift = c->pb_nb = 0;
     c->has_result = false;
     c->inv = nullptr;
@@ -307,7 +319,8 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     grid = (grid / L.nw) * L.nw;
     if (grid < L.nw) grid = L.nw;
     L.adv_grid = grid;
-    static const int filter_per_sm = getenv("GUM_FILTER_CTAS_PER_SM") ? std::max(1, atoi(getenv("GUM_FILTER_CTAS_PER_SM"))) : 0;
+    // clamped to 8: lb_parts (one look-back slot per filter CTA) is sized for nsm * 8 CTAs
+    static const int filter_per_sm = getenv("GUM_FILTER_CTAS_PER_SM") ? std::min(8, std::max(1, atoi(getenv("GUM_FILTER_CTAS_PER_SM")))) : 0;
     L.filter_grid = std::max(1, (c->nsm * (filter_per_sm ? filter_per_sm : c->filter_occ)) /
                                     (c->single_device ? std::min(c->P, 4) : 1));
     if (c->split && c->single_device) L.adv_grid = std::max(1, L.adv_grid / c->P);
@@ -315,6 +328,7 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.tail_grid = (c->n_units == 1 && c->cfg.tail_vertices && alg != GUM_PR) ? c->nsm * c->tail_occ : 0;
     L.adv_grid_pr = c->nsm * c->pr_push_occ;
+    L.pull_grid = std::max(1, (c->nsm * c->pull_occ) / L.nw);
     return L;
 }
 
@@ -377,12 +391,25 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.ctl = F.ctl;
         p.V = F.V;
         p.base = F.base;
+        if (alg == GUM_PR && c->pl_ready) {
+            p.pl_off = F.pl_off;
+            p.pl_col = F.pl_col;
+            p.pl_tx = F.pl_tx;
+            p.pl_tb = F.pl_tb;
+        }
         p.macc = (double*)F.mbuf;
         p.msent = (unsigned*)F.mbuf;
         p.mmin = (unsigned*)F.mbuf;
         d.lb[f] = c->lb[f];
     }
     d.mirrors = (c->cfg.mirrors && c->P > 1 && c->fr[0].mbuf) ? 1 : 0;
+    if (alg == GUM_PR && c->pl_ready) {
+        // one replica of x/outdeg per launch unit; worker w pulls from its unit's
+        d.pl_B = c->pl_B;
+        d.n_rep = c->n_units;
+        for (int u = 0; u < c->n_units; u++) d.cxrep[u] = c->cxg[unit_w0(c, u)];
+        for (int w = 0; w < c->P; w++) d.cxw[w] = c->cxg[unit_w0(c, c->split ? w : 0)];
+    }
     const int hk = alg == GUM_WCC ? 2 : (alg == GUM_PR ? -1 : 1);
     d.hub_on = (c->hub_kind == hk) ? 1 : 0;
     for (int w = 0; w < c->P && d.hub_on; w++)
@@ -466,7 +493,7 @@ gum_status unit_barrier(gum_ctx* c) {
 
 // Multi-process: the device buffers of fragment f that peers map (everything a kernel may touch after
 // OSteal hands the fragment to another worker), plus the unit's run control, trace and signal pad.
-constexpr int kMpFields = 40;
+constexpr int kMpFields = 48;
 int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     FragBufs& F = c->fr[f];
     int n = 0;
@@ -477,7 +504,7 @@ int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     GUM_FLD(F.ctl); GUM_FLD(F.pr_col); GUM_FLD(F.pr_q_v); GUM_FLD(F.pr_q_off); GUM_FLD(F.pr_tile);
     GUM_FLD(F.sq_col); GUM_FLD(F.sq_q_v); GUM_FLD(F.sq_q_off); GUM_FLD(F.sq_tile); GUM_FLD(F.in_row_ptr);
     GUM_FLD(F.in_col); GUM_FLD(c->lb[f]); GUM_FLD(c->rctl[f]); GUM_FLD(c->trace[f]); GUM_FLD(c->pad[f]);
-    GUM_FLD(F.mbuf);
+    GUM_FLD(F.mbuf); GUM_FLD(F.pl_off); GUM_FLD(F.pl_col); GUM_FLD(F.pl_tx); GUM_FLD(F.pl_tb); GUM_FLD(c->cxg[f]);
 #undef GUM_FLD
     return n;
 }
@@ -793,8 +820,122 @@ gum_status run_phase(gum_ctx* c, int alg, int phase, const DevCtx& d, const Laun
 
 // PR's frontier is every vertex with out-degree > 0 in every iteration: build it once, regrouped by
 // destination block so that consecutive chunks push into one L2-resident slice of acc.
+// PR pull (default): every fragment's in-edges regrouped by source block (an x/outdeg slice
+// sized to stay L2-resident while a pass gathers from it), plus one replica of x/outdeg per launch unit.
+gum_status build_pr_pull(gum_ctx* c) {
+    const unsigned long long block_bytes = getenv("GUM_PR_PULL_BLOCK_BYTES")
+                                               ? strtoull(getenv("GUM_PR_PULL_BLOCK_BYTES"), 0, 10)
+                                               : (48ull << 20);
+    unsigned long long S = std::max<unsigned long long>(1024, block_bytes / 8);
+    int B = (int)((c->V + S - 1) / S);
+    if (B > 64) {
+        B = 64;
+        S = (c->V + 63) / 64;
+    }
+    if (B < 1) B = 1;
+    const int d0 = c->dev[0];
+    CK(cudaSetDevice(d0));
+    cudaStream_t s = c->stream[0];
+    std::vector<Alloc> tmp;
+    unsigned long long* trp = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, tmp);
+    unsigned* tcol = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(c->E, 1) * 4, tmp);
+    unsigned long long* cursor = (unsigned long long*)dalloc(c, d0, (c->V + 1ull) * 8, tmp);
+    const size_t tb = setup_scan_tmp_bytes(c->V);
+    void* t = dalloc(c, d0, tb, tmp);
+    if (!trp || !tcol || !cursor || !t) {
+        free_list(c, tmp);
+        return fail(c, GUM_ENOMEM, "PR pull: transpose alloc failed");
+    }
+    cudaError_t e = setup_transpose(c->p_row_ptr, c->p_col, c->V, c->E, trp, tcol, cursor, t, tb, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) {
+        free_list(c, tmp);
+        return fail(c, GUM_ECUDA, "PR pull transpose: %s", cudaGetErrorString(e));
+    }
+    std::vector<unsigned long long> hb(c->P + 1);
+    for (int f = 0; f <= c->P; f++) CK(cudaMemcpy(&hb[f], trp + c->bounds[f], 8, cudaMemcpyDeviceToHost));
+    for (int f = 0; f < c->P; f++) {
+        FragBufs& F = c->fr[f];
+        F.pr_qlen = F.V;  // every vertex pulls (stats / byte model: one queue entry per vertex)
+        F.pr_qedges = F.E;
+        if (!frag_local(c, f)) continue;
+        const unsigned long long Ein = hb[f + 1] - hb[f];
+        if (Ein >= (1ull << 32)) {
+            free_list(c, tmp);
+            return fail(c, GUM_EUNSUP, "PR pull: fragment %d has >= 2^32 in-edges: use more workers", f);
+        }
+        std::vector<Alloc> t2;
+        unsigned long long* irp = (unsigned long long*)dalloc(c, d0, (F.V + 1ull) * 8, t2);
+        const size_t tb2 = setup_pr_tmp_bytes(F.V, B);
+        void* tt = dalloc(c, d0, tb2, t2);
+        if (!irp || !tt) {
+            free_list(c, t2);
+            free_list(c, tmp);
+            return fail(c, GUM_ENOMEM, "PR pull: fragment %d temp alloc failed", f);
+        }
+        CK(setup_rebase_rows(trp, c->bounds[f], c->bounds[f + 1], irp, s));
+        std::vector<unsigned long long> htb(B + 1);
+        CK(setup_pr_pull(irp, tcol + hb[f], F.V, Ein, (unsigned)S, B, kPullTile, nullptr, nullptr, nullptr, htb.data(),
+                         tt, tb2, s));
+        const unsigned long long n_off = (unsigned long long)B * F.V + 1;
+        // built on worker 0's device; copied to the fragment's device when it differs
+        const bool here = F.dev == d0;
+        std::vector<Alloc>& dst_list = here ? c->part_allocs : t2;
+        unsigned* off = (unsigned*)dalloc(c, d0, n_off * 4, dst_list);
+        unsigned* pcol = (unsigned*)dalloc(c, d0, std::max<unsigned long long>(Ein, 1) * 4, dst_list);
+        unsigned* tx = (unsigned*)dalloc(c, d0, htb[B] * 4, dst_list);
+        unsigned long long* tbd = (unsigned long long*)dalloc(c, d0, (B + 1) * 8, dst_list);
+        if (!off || !pcol || !tx || !tbd) {
+            free_list(c, t2);
+            free_list(c, tmp);
+            return fail(c, GUM_ENOMEM, "PR pull: fragment %d alloc failed (%llu in-edges)", f, Ein);
+        }
+        CK(setup_pr_pull(irp, tcol + hb[f], F.V, Ein, (unsigned)S, B, kPullTile, off, pcol, tx, htb.data(), tt, tb2,
+                         s));
+        CK(cudaMemcpyAsync(tbd, htb.data(), (B + 1) * 8, cudaMemcpyHostToDevice, s));
+        CK(cudaStreamSynchronize(s));
+        if (here) {
+            F.pl_off = off;
+            F.pl_col = pcol;
+            F.pl_tx = tx;
+            F.pl_tb = tbd;
+        } else {
+            F.pl_off = (unsigned*)dalloc(c, F.dev, n_off * 4, c->part_allocs);
+            F.pl_col = (unsigned*)dalloc(c, F.dev, std::max<unsigned long long>(Ein, 1) * 4, c->part_allocs);
+            F.pl_tx = (unsigned*)dalloc(c, F.dev, htb[B] * 4, c->part_allocs);
+            F.pl_tb = (unsigned long long*)dalloc(c, F.dev, (B + 1) * 8, c->part_allocs);
+            if (!F.pl_off || !F.pl_col || !F.pl_tx || !F.pl_tb) {
+                free_list(c, t2);
+                free_list(c, tmp);
+                return fail(c, GUM_ENOMEM, "PR pull: fragment %d device copy alloc failed", f);
+            }
+            CK(cudaMemcpyPeerAsync(F.pl_off, F.dev, off, d0, n_off * 4, s));
+            if (Ein) CK(cudaMemcpyPeerAsync(F.pl_col, F.dev, pcol, d0, Ein * 4, s));
+            CK(cudaMemcpyPeerAsync(F.pl_tx, F.dev, tx, d0, htb[B] * 4, s));
+            CK(cudaMemcpyPeerAsync(F.pl_tb, F.dev, tbd, d0, (B + 1) * 8, s));
+            CK(cudaStreamSynchronize(s));
+        }
+        free_list(c, t2);
+    }
+    free_list(c, tmp);
+    for (int u = 0; u < c->n_units; u++) {
+        if (!unit_local(c, u)) continue;
+        const int w0 = unit_w0(c, u);
+        c->cxg[w0] = (double*)dalloc(c, unit_dev(c, u), 2ull * c->V * 8, c->part_allocs);
+        if (!c->cxg[w0]) return fail(c, GUM_ENOMEM, "PR pull: x/outdeg replica alloc failed");
+    }
+    CK(cudaSetDevice(d0));
+    c->pl_B = (unsigned)B;
+    c->pl_ready = true;
+    c->pr_ready = true;
+    drop_graphs(c);
+    return GUM_OK;
+}
+
 gum_status build_pr(gum_ctx* c) {
     if (c->pr_ready) return GUM_OK;
+    // pull unless the caller asked for the push, or NEXT-1 mirrors (which aggregate pushes) are on
+    if (!c->cfg.pr_push && !(c->cfg.mirrors && c->P > 1)) return build_pr_pull(c);
     const unsigned long long block_bytes = getenv("GUM_PR_BLOCK_BYTES") ? strtoull(getenv("GUM_PR_BLOCK_BYTES"), 0, 10)
                                                                        : (48ull << 20);
     unsigned long long S = std::max<unsigned long long>(1024, block_bytes / 8);
@@ -1102,6 +1243,9 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
         if (filter_occupancy(&occ) == cudaSuccess && occ > 0) c->filter_occ = std::min(occ, 4);
         occ = 0;
         if (pr_push_occupancy(&occ) == cudaSuccess && occ > 0) c->pr_push_occ = occ;
+        occ = 0;
+        if (pr_pull_occupancy(&occ) == cudaSuccess && occ > 0) c->pull_occ = occ;
+        if (const char* e = getenv("GUM_PULL_CTAS_PER_SM")) c->pull_occ = std::max(1, atoi(e));
         if (const char* e = getenv("GUM_PR_PUSH_CTAS_PER_SM")) c->pr_push_occ = std::max(1, atoi(e));
         cudaGetLastError();
     }
@@ -1123,7 +1267,7 @@ static unsigned long long config_hash(const gum_config* cfg) {
     GUM_HC(osteal_active_threshold); GUM_HC(osteal_edges_per_worker); GUM_HC(chunk_edges); GUM_HC(pr_iterations);
     GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
     GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt); GUM_HC(osteal_sync_edges);
-    GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree);
+    GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree); GUM_HC(pr_push);
 #undef GUM_HC
     return h;
 }

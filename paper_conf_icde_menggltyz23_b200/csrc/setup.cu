@@ -3,6 +3,9 @@
 #include <cub/cub.cuh>
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <vector>
+
 #include "kernels.h"
 
 namespace gum {
@@ -441,6 +444,75 @@ cudaError_t setup_pr_blocked(const unsigned long long* rp, const unsigned* col, 
     if (e != cudaSuccess) return e;
     e = cudaStreamSynchronize(s);  // Ef is a by-value host local
     (void)e;
+    return cudaGetLastError();
+}
+
+// ---- PR pull (gum_prepare(PR)): the fragment's in-edges regrouped source-block-major ---------------
+// Same counting as the destination-blocked push queue (k_pr_count / k_pr_scatter), applied to the
+// fragment's in-CSR: block b holds the in-edges whose SOURCE is in [b*S, (b+1)*S), rows ascending, so a
+// pull pass over block b gathers x/outdeg from one L2-sized slice. Offsets narrowed to u32 (the caller
+// checks Ein < 2^32); merge-path tile starts precomputed per pass (one binary search per tile, untimed).
+__global__ void k_pl_narrow(const unsigned long long* off, unsigned long long n, unsigned* out) {
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i <= n;
+         i += (unsigned long long)gridDim.x * blockDim.x)
+        out[i] = (unsigned)off[i];
+}
+
+// tile t of a pass starts at merge-path diagonal t*tile over (row ends, edges): the first row whose end
+// has not been consumed (Merrill & Garland's MergePathSearch)
+__global__ void k_pl_tiles(const unsigned* off /* pass rows: [Vf+1] */, unsigned Vf, unsigned long long tile,
+                           unsigned long long ntiles, unsigned* tx) {
+    const unsigned long long base = off[0], nE = off[Vf] - base, items = (unsigned long long)Vf + nE;
+    for (unsigned long long t = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; t <= ntiles;
+         t += (unsigned long long)gridDim.x * blockDim.x) {
+        const unsigned long long d = t * tile < items ? t * tile : items;
+        unsigned long long lo = d > nE ? d - nE : 0, hi = d < Vf ? d : Vf;
+        while (lo < hi) {
+            const unsigned long long pivot = (lo + hi) >> 1;
+            if ((unsigned long long)(off[pivot + 1] - base) <= d - pivot - 1) lo = pivot + 1;
+            else hi = pivot;
+        }
+        tx[t] = (unsigned)lo;
+    }
+}
+
+cudaError_t setup_pr_pull(const unsigned long long* in_rp, const unsigned* in_col, unsigned Vf, unsigned long long Ein,
+                          unsigned S, int B, unsigned tile, unsigned* pl_off, unsigned* pl_col, unsigned* pl_tx,
+                          unsigned long long* h_tb, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+    (void)Ein;
+    const unsigned long long n = (unsigned long long)B * Vf;
+    char* t = (char*)tmp;
+    unsigned long long* off = (unsigned long long*)t;
+    t += ((n + 1) * 8 + 255) / 256 * 256;
+    void* cub_tmp = t;
+    size_t cub_bytes = tmp_bytes - (size_t)(t - (char*)tmp);
+    const int warps_per_cta = 8;
+    k_pr_count<<<1184, 32 * warps_per_cta, warps_per_cta * B * sizeof(unsigned), s>>>(in_rp, in_col, Vf, S, B, off);
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, off, off, (size_t)n + 1, s);
+    if (e != cudaSuccess) return e;
+    std::vector<unsigned long long> hb(B + 1);
+    for (int b = 0; b <= B; b++) {
+        e = cudaMemcpyAsync(&hb[b], off + (unsigned long long)b * Vf, 8, cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) return e;
+    }
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return e;
+    unsigned long long acc = 0;
+    for (int b = 0; b < B; b++) {
+        const unsigned long long items = (unsigned long long)Vf + (hb[b + 1] - hb[b]);
+        h_tb[b] = acc;
+        acc += (items + tile - 1) / tile + 1;
+    }
+    h_tb[B] = acc;
+    if (!pl_off || !pl_col || !pl_tx) return cudaGetLastError();
+    k_pr_scatter<<<1184, 32 * warps_per_cta, warps_per_cta * B * sizeof(unsigned long long), s>>>(in_rp, in_col, Vf, S,
+                                                                                                  B, off, pl_col);
+    k_pl_narrow<<<1184, 256, 0, s>>>(off, n, pl_off);
+    for (int b = 0; b < B; b++) {
+        const unsigned long long nt = h_tb[b + 1] - h_tb[b] - 1;
+        k_pl_tiles<<<(unsigned)std::min<unsigned long long>((nt + 256) / 256, 4096), 256, 0, s>>>(
+            pl_off + (unsigned long long)b * Vf, Vf, tile, nt, pl_tx + h_tb[b]);
+    }
     return cudaGetLastError();
 }
 

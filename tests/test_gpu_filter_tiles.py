@@ -34,3 +34,26 @@ def test_filter_multi_tile_per_cta():
                        capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert r.stdout.count("ok ") == 12, r.stdout
+
+
+def test_filter_stride_coprime_6159_tiles():
+    """with 6159 = 3 * 2053 filter tiles the old stride search (2053 -> 2055) shared the factor 3
+    with n_tiles, so a third of the tiles were filtered three times and the rest never. V = 6159 * 2048
+    gives 6159 sparse-list tiles (WCC iteration 0, 8 entries per thread) and 6159 dense bitmap tiles (BFS
+    forced dense); both must equal the oracle."""
+    import numpy as np
+
+    import inputs
+    from tests.gpu_helpers import check, csr_of
+
+    V = 6159 * 2048
+    rng = np.random.default_rng(6159)
+    E = 1 << 20
+    src = rng.integers(0, V, E, dtype=np.int64).astype(np.uint32)
+    dst = rng.integers(0, V, E, dtype=np.int64).astype(np.uint32)
+    g = inputs.EdgeList(V, src, dst, None, "stride6159")
+    csr = csr_of(g)
+    check(g, "wcc", 0, csr=csr)
+    s = int(src[0])
+    check(g, "bfs", s, csr=csr, force_mode="dense", tail_vertices=0)
+    check(g, "bfs", s, csr=csr, force_mode="sparse", tail_vertices=0)

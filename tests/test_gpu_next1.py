@@ -32,7 +32,9 @@ def test_mirrors_parity(alg, P, part):
     s = inputs.pick_source(g, 41)
     ref = oracle.run(alg, g, s)
     csr = csr_of(g)
-    _, plain, _ = check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P, tail_vertices=0)
+    # (PR: the plain path compared here is the push, whose per-edge remote atomics the mirrors aggregate)
+    _, plain, _ = check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P, tail_vertices=0,
+                        pr_push=(alg == "pr"))
     _, st, _ = check(g, alg, s, csr=csr, ref=ref, num_gpus=P, part=part, seed=P, tail_vertices=0, mirrors=True)
     assert st.remote_filtered > 0
     if alg == "pr":

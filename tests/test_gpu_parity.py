@@ -199,11 +199,11 @@ def test_split_units_multi_device_path(alg, monkeypatch):
 
 @pytest.mark.parametrize("P", [1, 3])
 def test_pr_destination_blocked_queue(monkeypatch, P):
-    """Force the PR destination blocking (8 KiB acc blocks -> many blocks) and check parity."""
+    """PR push (pr_push=1): force the destination blocking (8 KiB acc blocks -> many blocks), check parity."""
     monkeypatch.setenv("GUM_PR_BLOCK_BYTES", "8192")
     g = inputs.rmat(13, 16, seed=31, weighted=False)
     ref = oracle.run("pr", g)
-    out, st, _ = check(g, "pr", 0, ref=ref, num_gpus=P, part="random" if P > 1 else "seg", seed=3)
+    out, st, _ = check(g, "pr", 0, ref=ref, num_gpus=P, part="random" if P > 1 else "seg", seed=3, pr_push=True)
     assert st.vertices_frontier > 20 * np.count_nonzero(np.bincount(g.src, minlength=g.num_vertices))
 
 
