@@ -198,6 +198,14 @@ typedef struct {
     uint64_t tail_edges;
     uint64_t tail_vertices;
     uint64_t tail_activations;
+    /* multi-unit runs in the device-resident loop (one CUDA graph per device / process): per launch
+     * unit, the number of device barriers it arrived at and the iteration of its last arrival. A unit
+     * evicted by OSteal stops arriving: its last arrival is the barrier right after the eviction. */
+    uint32_t unit_barriers[GUM_MAX_WORKERS];
+    uint32_t unit_last_iter[GUM_MAX_WORKERS];
+    /* host-side launches of this process in the run (kernels + graph launches): in the device-resident
+     * loops this does not depend on the number of iterations */
+    uint64_t host_launches;
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

@@ -83,7 +83,8 @@ class gum_run_stats(ctypes.Structure):
                 ("remote_filtered", ctypes.c_uint64), ("hub_cached_edges", ctypes.c_uint64),
                 ("mirror_flush_bytes", ctypes.c_uint64), ("blocked_iterations", ctypes.c_uint32),
                 ("pad0", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
-                ("tail_activations", ctypes.c_uint64)]
+                ("tail_activations", ctypes.c_uint64), ("unit_barriers", ctypes.c_uint32 * MAX_WORKERS),
+                ("unit_last_iter", ctypes.c_uint32 * MAX_WORKERS), ("host_launches", ctypes.c_uint64)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -198,6 +199,9 @@ class RunStats:
     tail_edges: int = 0
     tail_vertices: int = 0
     tail_activations: int = 0
+    unit_barriers: list = None
+    unit_last_iter: list = None
+    host_launches: int = 0
 
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
@@ -357,7 +361,10 @@ class Context:
         s = gum_run_stats()
         self._check(load_library().gum_run(self._ctx, ALGS[alg], int(source), ctypes.byref(s)))
         self._last_alg = alg
-        return RunStats(**{k: getattr(s, k) for k, _ in gum_run_stats._fields_})
+        vals = {k: getattr(s, k) for k, _ in gum_run_stats._fields_}
+        for k in ("unit_barriers", "unit_last_iter"):
+            vals[k] = list(vals[k])[: self.num_gpus]
+        return RunStats(**vals)
 
     def result(self, out=None):
         dt = np.float64 if self._last_alg == "pr" else np.uint32

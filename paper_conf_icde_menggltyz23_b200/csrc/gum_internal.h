@@ -101,6 +101,13 @@ struct alignas(128) RunCtl {
     double pr_resid;
     unsigned int ticket[kMaxW];   // filter partition tickets per fragment (reset by control)
     unsigned int filt_done[kMaxW];
+    // device-resident multi-unit loop: barrier members {0..mb-1}; mb_next takes effect at the
+    // next phase-A barrier (units >= mb_next leave it and park until woken); wakes[u] counts unit u's
+    // wake-ups (computed identically by every member; the signal pad holds the same count); bar_ep is the
+    // epoch of this unit's last device barrier (monotone across runs, equal on all members)
+    unsigned int mb, mb_next;
+    unsigned int wakes[kMaxW];
+    unsigned long long bar_ep;
 };
 
 // Decoupled look-back slot of the filter scan (one per partition per fragment, unit-local).
@@ -180,9 +187,17 @@ struct HubPtrs {
     const unsigned int* w;          // cached weights (SSSP) or null
 };
 
-// Multi-process signal pads (a10): pad[u][s] = last barrier epoch unit s signalled to unit u;
-// pad[u][kMaxW] = timeout flag (a peer never arrived).
-constexpr int kPadWords = 16;
+// Signal pads of the multi-unit barriers (a10), one per launch unit in its device memory (peer / IPC
+// mapped): words [0, kMaxW) = host-loop barrier epochs by sender; kPadTimeout = a peer never arrived;
+// kPadWake = wake count written by unit 0 (OSteal give-back / end of run); kPadArr / kPadLastIt = this
+// unit's device-barrier arrivals in the current run and the iteration of the last one (stats);
+// [kPadGraph, kPadGraph + kMaxW) = device-loop barrier epochs by sender.
+constexpr int kPadWords = 32;
+constexpr int kPadTimeout = kMaxW;
+constexpr int kPadWake = kMaxW + 1;
+constexpr int kPadArr = kMaxW + 2;
+constexpr int kPadLastIt = kMaxW + 3;
+constexpr int kPadGraph = 16;
 struct MpPads {
     unsigned long long* pad[kMaxW];
 };
@@ -228,6 +243,11 @@ struct DevCtx {
     int n_rep;
     double* cxrep[kMaxW];
     const double* cxw[kMaxW];
+    // device-resident multi-unit loop: one CUDA graph per launch unit, device barriers over the member
+    // units through these pads (unit u's pad in unit u's memory); 0 = single unit or host-driven loop
+    int units_dev;
+    int n_units;
+    unsigned long long* pad[kMaxW];
     int hub_on;                 // NEXT-1 hub cache built for this algorithm
     HubPtrs hub[kMaxW][kMaxW];  // [worker][fragment] (fragment != worker)
 };

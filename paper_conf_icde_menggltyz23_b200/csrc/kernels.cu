@@ -181,6 +181,13 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     rc->pb = 0;
     rc->pull = 0;
     rc->nf_T = c.nf_delta ? (unsigned long long)c.nf_delta : 0xFFFFFFFFull;
+    // device-resident multi-unit loop: every unit is a member at the start (bar_ep and wakes[] stay
+    // monotone across runs: the pads keep their last values)
+    rc->mb = rc->mb_next = (unsigned)c.n_units;
+    if (c.pad[w0]) {
+        c.pad[w0][kPadArr] = 0;
+        c.pad[w0][kPadLastIt] = 0;
+    }
 }
 
 // ------------------------------------------------------------------------------------------ filter
@@ -831,6 +838,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         done = err != 0 || (active == 0 && !nf_bump) || k >= c.max_iter;
     }
     unsigned m = rc->m;
+    unsigned grow_to = 0;  // device-resident multi-unit loop: members to wake for the next iteration
     if (!done) {
         // a6 OSteal: the active owner set is re-decided every iteration from the global
         // counts. Below the active-vertex threshold the survivors are {0..m'-1} (uniform-fabric
@@ -849,6 +857,13 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
                     const unsigned long long want = (total_edges + c.os_epw - 1) / c.os_epw;
                     mp = want < 1 ? 1u : (want > (unsigned long long)c.P ? (unsigned)c.P : (unsigned)want);
                 }
+            }
+            if (c.units_dev && mp > rc->mb) {
+                // give-back to parked units (device-resident multi-unit loop): they are woken now, rejoin
+                // the barriers at the next phase-A barrier and own their fragments from the next control on;
+                // this iteration's owners stay within the current members
+                grow_to = mp;
+                mp = rc->mb;
             }
             if (mp != m) {
                 for (int f = 0; f < c.P; f++) rc->owner[f] = (unsigned)f < mp ? (unsigned)f : (unsigned)f % mp;
@@ -940,8 +955,13 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             total_edges <= 8ull * c.tail_enter) {
             rc->tail = 1;
             for (int f = 0; f < c.P; f++) {
-                c.f[f].ctl->tcnt[1] = 0;
-                c.f[f].ctl->tedges[1] = 0;
+                // the engine's first next-list counters live in the fragments' (shared) control blocks: only
+                // the unit that runs the engine resets them -- another unit's late control would otherwise
+                // clear appends the engine already made
+                if (w0 == 0) {
+                    c.f[f].ctl->tcnt[1] = 0;
+                    c.f[f].ctl->tedges[1] = 0;
+                }
                 rc->owner[f] = 0;
             }
             if (m != 1) rc->osteal_iter = k;
@@ -985,7 +1005,44 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         rc->done = 1;
         rc->err = err;
     }
+    // device-resident multi-unit loop (a6 across devices, "GPU1 will not participate in
+    // synchronization anymore"): the members of the next phase-A barrier are the owners of this iteration
+    // (units >= m leave that barrier and park: no launches, no arrivals), plus units being given ownership
+    // back; parked units are woken for a give-back or for the end of the run. Every member computes the
+    // same membership and wake counts; unit 0 alone copies its run control into each woken unit and then
+    // releases the unit's wake word.
+    unsigned wk_lo = 0, wk_hi = 0;
+    if (c.units_dev) {
+        const unsigned mb = rc->mb;
+        unsigned nm = mb;
+        if (!done) {
+            nm = m;
+            if (grow_to > nm) nm = grow_to;
+        }
+        rc->mb_next = nm;
+        if (done) {
+            wk_lo = mb;
+            wk_hi = (unsigned)c.n_units;
+        } else if (nm > mb) {
+            wk_lo = mb;
+            wk_hi = nm;
+        }
+        for (unsigned u = wk_lo; u < wk_hi; u++) rc->wakes[u] = rc->wakes[u] + 1;
+    }
     __threadfence();
+    if (c.units_dev && w0 == 0 && wk_hi > wk_lo) {
+        constexpr int kWords = (int)(sizeof(RunCtl) / 8);
+        const unsigned long long* src = reinterpret_cast<const unsigned long long*>(rc);
+        for (unsigned u = wk_lo; u < wk_hi; u++) {
+            unsigned long long* dst = reinterpret_cast<unsigned long long*>(c.rctl[u]);
+            for (int i = 0; i < kWords; i++) dst[i] = src[i];
+        }
+        asm volatile("fence.sc.sys;" ::: "memory");
+        for (unsigned u = wk_lo; u < wk_hi; u++)
+            asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(c.pad[u] + kPadWake),
+                         "l"((unsigned long long)rc->wakes[u])
+                         : "memory");
+    }
     if (use_h) cudaGraphSetConditional(h, done ? 0u : 1u);
 }
 
@@ -1902,7 +1959,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
     RunCtl* rc = c.rctl[w0];
     __shared__ unsigned s_hdr[4];  // gen, k0, nfT, fslot
     if (threadIdx.x == 0) {
-        s_go = vload(&rc->tail) && !vload(&rc->done);
+        s_go = vload(&rc->tail) && !vload(&rc->done) && w0 == 0;  // OSteal's m'=1: unit 0 runs every fragment
         s_hdr[0] = vload(&rc->tbar_gen);
         s_hdr[1] = vload(&rc->iter) - 1;  // control already counted the first tail iteration
         const unsigned long long T = vload(&rc->nf_T);
@@ -2845,6 +2902,81 @@ __global__ void k_mp_barrier(const MpPads p, int P, int me, unsigned long long e
         }
         __nanosleep(200);
     }
+}
+
+// Device-resident multi-unit loop: the a10 barrier of one unit's CUDA graph, one thread.
+// Members are the units {0..mb-1} of the unit's run control (the same on every member). Arrival =
+// fence.sc.sys, then st.release.sys of the next epoch into every other member's pad, then an acquire spin
+// on this unit's pad until every member has signalled it. At the phase-A barrier (before the filter) the
+// membership decided by the previous control takes effect: a unit that is no longer a member (OSteal
+// eviction) leaves after this last barrier and parks here -- it launches nothing and arrives
+// at no further barrier -- until unit 0 wakes it (give-back, or end of run) after copying its run
+// control into it; it then re-evaluates its membership with that state. 60 s without progress sets the
+// timeout flag and ends the run (GUM_ENCCL) instead of hanging.
+__global__ void k_unit_bar(const __grid_constant__ DevCtx c, int u, int phase) {
+    if (threadIdx.x != 0) return;
+    RunCtl* rc = c.rctl[u];
+    unsigned long long* me = c.pad[u];
+    unsigned long long t0 = globaltimer();
+    for (;;) {
+        if (vload(&rc->done)) return;
+        const unsigned mb = vload(&rc->mb);
+        unsigned nm = mb, target = 0;
+        if (phase == 0) {
+            nm = vload(&rc->mb_next);
+            target = vload(&rc->wakes[u]) + 1u;  // read before arriving: unit 0 may wake us right after
+        }
+        // this barrier: the old members (leavers included, so their last writes precede any wake-up) and
+        // the joiners woken by the previous control
+        const unsigned mem = nm > mb ? nm : mb;
+        if ((unsigned)u < mem) {
+            const unsigned long long ep = rc->bar_ep + 1;
+            rc->bar_ep = ep;
+            if (nm != mb) rc->mb = nm;  // later barriers use the new member set
+            me[kPadArr] = me[kPadArr] + 1;
+            me[kPadLastIt] = rc->iter;
+            asm volatile("fence.sc.sys;" ::: "memory");
+            for (unsigned t = 0; t < mem; t++)
+                if (t != (unsigned)u)
+                    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(c.pad[t] + kPadGraph + u), "l"(ep) : "memory");
+            for (unsigned t = 0; t < mem; t++) {
+                if (t == (unsigned)u) continue;
+                for (;;) {
+                    unsigned long long v;
+                    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(me + kPadGraph + t) : "memory");
+                    if (v >= ep) break;
+                    if (globaltimer() - t0 > 60ull * 1000000000ull) {
+                        atomicExch(me + kPadTimeout, 1ull);
+                        rc->err = 2;
+                        rc->done = 1;
+                        return;
+                    }
+                    __nanosleep(64);
+                }
+            }
+            if ((unsigned)u < nm) return;
+        }
+        // parked: wait for unit 0's wake (it wrote our run control first), then re-evaluate
+        t0 = globaltimer();
+        for (;;) {
+            unsigned long long v;
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(me + kPadWake) : "memory");
+            if (v >= target) break;
+            if (globaltimer() - t0 > 600ull * 1000000000ull) {  // parked units may wait a whole long tail
+                atomicExch(me + kPadTimeout, 1ull);
+                rc->err = 2;
+                rc->done = 1;
+                return;
+            }
+            __nanosleep(256);
+        }
+        t0 = globaltimer();
+    }
+}
+
+cudaError_t launch_unit_bar(const DevCtx& c, int u, int phase, cudaStream_t s) {
+    k_unit_bar<<<1, 32, 0, s>>>(c, u, phase);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_mp_barrier(const MpPads& p, int P, int me, unsigned long long epoch, cudaStream_t s) {

@@ -31,6 +31,9 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
 cudaError_t launch_gather(const DevCtx& c, int f, void* out, int is_pr, cudaStream_t s, int grid);
 // multi-process barrier: every rank signals epoch into every peer's pad, then waits for all peers
 cudaError_t launch_mp_barrier(const MpPads& p, int P, int me, unsigned long long epoch, cudaStream_t s);
+// device-resident multi-unit loop: unit u's barrier (phase 0 = before the filter, with OSteal membership
+// changes and parking; phase 1 = before control)
+cudaError_t launch_unit_bar(const DevCtx& c, int u, int phase, cudaStream_t s);
 cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm);
 cudaError_t tail_occupancy(int* blocks_per_sm);
 cudaError_t filter_occupancy(int* blocks_per_sm);

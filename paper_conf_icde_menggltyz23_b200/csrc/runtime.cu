@@ -159,6 +159,7 @@ struct gum_ctx {
     RunCtl* h_rctl = nullptr;  // pinned
     void* d_res = nullptr;
     cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaGraphExec_t gexec_u[4][kMaxW] = {};  // device-resident multi-unit loop: one graph per unit
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     std::vector<cudaEvent_t> bar_ev;
     std::vector<cudaEvent_t> prof_ev;  // pairs (start, end)
@@ -176,6 +177,7 @@ struct gum_ctx {
     unsigned long long* pad[kMaxW] = {nullptr};  // per unit: signal pad (epochs by unit + timeout flag)
     unsigned long long mp_epoch = 0;
     unsigned long long launches = 0;  // kernel launches of the current run (gum_run_stats.kernel_launches)
+    unsigned long long hlaunch = 0;   // host-side launches (kernels + graphs) of the current run
     std::map<std::pair<int, unsigned long long>, void*> ipc_map;  // (peer, peer pointer) -> mapped pointer
 };
 
@@ -253,6 +255,11 @@ void drop_graphs(gum_ctx* c) {
         if (g) cudaGraphExecDestroy(g);
         g = nullptr;
     }
+    for (auto& row : c->gexec_u)
+        for (auto& g : row) {
+            if (g) cudaGraphExecDestroy(g);
+            g = nullptr;
+        }
 }
 
 void drop_partition(gum_ctx* c) {
@@ -326,7 +333,15 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     if (c->split && c->single_device) L.adv_grid = std::max(1, L.adv_grid / c->P);
     L.fin_grid = std::max(1, (c->nsm * 4) / L.nw);
     L.init_grid = std::max(1, (c->nsm * 4) / L.nw);
-    L.tail_grid = (c->n_units == 1 && c->cfg.tail_vertices && alg != GUM_PR) ? c->nsm * c->tail_occ : 0;
+    // the tail engine (OSteal's m'=1 mode) runs on unit 0 over every fragment; with several units on one
+    // device one CTA slot per SM is left for the parked units' barrier kernels (co-residency of the
+    // cooperative grid)
+    // (the host-driven multi-unit loop has no run-control hand-over between units, so it keeps the tail engine
+    // off: the other units' iteration counters would not follow the engine's iterations)
+    const bool tail_ok = c->n_units == 1 || !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
+    L.tail_grid = (u == 0 && tail_ok && c->cfg.tail_vertices && alg != GUM_PR)
+                      ? c->nsm * ((c->split && c->single_device && c->tail_occ > 1) ? c->tail_occ - 1 : c->tail_occ)
+                      : 0;
     L.adv_grid_pr = c->nsm * c->pr_push_occ;
     L.pull_grid = std::max(1, (c->nsm * c->pull_occ) / L.nw);
     return L;
@@ -425,6 +440,9 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         d.tsplit[w] = c->tsplit[unit_w0(c, u)];
     }
     d.lb_parts = c->lb_parts;
+    d.n_units = c->n_units;
+    for (int u = 0; u < c->n_units; u++) d.pad[u] = c->pad[unit_w0(c, u)];
+    d.units_dev = (c->n_units > 1 && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))) ? 1 : 0;
     for (int i = 0; i <= c->P; i++) d.bounds[i] = c->bounds[i];
     d.P = c->P;
     d.chunk = c->cfg.chunk_edges;
@@ -443,7 +461,9 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.force_mode = (c->cfg.flags & GUM_CFG_FORCE_DENSE) ? 2u : ((c->cfg.flags & GUM_CFG_FORCE_SPARSE) ? 1u : 0u);
     d.dense_div = 32;
     d.nf_delta = alg == GUM_SSSP ? c->cfg.sssp_delta : 0u;
-    d.tail_enter = (c->n_units == 1 && alg != GUM_PR) ? c->cfg.tail_vertices : 0u;
+    d.tail_enter = (alg != GUM_PR && (c->n_units == 1 || !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))))
+                       ? c->cfg.tail_vertices
+                       : 0u;
     d.tail_exit = 4u * c->cfg.tail_vertices;
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
     d.pb_nb = c->pb_nb;
@@ -1126,6 +1146,46 @@ gum_status capture_graph(gum_ctx* c, int alg, const DevCtx& d, const LaunchCfg& 
     return GUM_OK;
 }
 
+// Device-resident multi-unit loop: unit u's graph = a conditional WHILE node whose body is
+// unit barrier (phase A: OSteal membership, parking) -> phase-0 kernels -> unit barrier -> phase-1 kernels.
+// Every unit decides convergence and OSteal redundantly in its control kernel and sets its own condition;
+// a parked unit sits in its phase-A barrier until woken. No host round trip per iteration.
+gum_status capture_unit_graph(gum_ctx* c, int alg, int u, const DevCtx& d, const LaunchCfg& L) {
+    if (c->gexec_u[alg][u]) return GUM_OK;
+    CK(cudaSetDevice(unit_dev(c, u)));
+    cudaStream_t s = c->stream[L.w0];
+    cudaGraph_t g;
+    CK(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle h;
+    CK(cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault));
+    alignas(cudaGraphNodeParams) unsigned char pbuf[sizeof(cudaGraphNodeParams)];
+    memset(pbuf, 0, sizeof(pbuf));
+    cudaGraphNodeParams& p = *reinterpret_cast<cudaGraphNodeParams*>(pbuf);
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = cudaGraphCondTypeWhile;
+    p.conditional.size = 1;
+    cudaGraphNode_t node;
+    CK(cudaGraphAddNode(&node, g, nullptr, 0, &p));
+    cudaGraph_t body = p.conditional.phGraph_out[0];
+    CK(cudaStreamBeginCaptureToGraph(s, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+    cudaError_t e = launch_unit_bar(d, u, 0, s);
+    if (e == cudaSuccess) e = launch_phase(alg, 0, d, L, s, h, 1);
+    if (e == cudaSuccess) e = launch_unit_bar(d, u, 1, s);
+    if (e == cudaSuccess) e = launch_phase(alg, 1, d, L, s, h, 1);
+    cudaGraph_t captured;
+    cudaError_t e2 = cudaStreamEndCapture(s, &captured);
+    if (e != cudaSuccess || e2 != cudaSuccess) {
+        cudaGraphDestroy(g);
+        return fail(c, GUM_ECUDA, "unit %d graph capture: %s / %s", u, cudaGetErrorString(e), cudaGetErrorString(e2));
+    }
+    cudaGraphExec_t ex;
+    CK(cudaGraphInstantiate(&ex, g, 0));
+    cudaGraphDestroy(g);
+    c->gexec_u[alg][u] = ex;
+    return GUM_OK;
+}
+
 }  // namespace
 
 // ================================================================================ C ABI
@@ -1604,7 +1664,7 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
     for (int u = 0; u < c->n_units; u++) {
         if (!unit_local(c, u)) continue;
         int w0 = unit_w0(c, u), d = unit_dev(c, u);
-        if (c->mp) {
+        if (c->n_units > 1) {
             c->pad[w0] = (unsigned long long*)dalloc(c, d, kPadWords * 8, c->part_allocs);
             if (!c->pad[w0]) return fail(c, GUM_ENOMEM, "signal pad alloc failed");
             CK(cudaSetDevice(d));
@@ -1694,20 +1754,27 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     const double D0 = (double)c->n_dangling / (double)c->V;
     const bool profile = (c->cfg.flags & GUM_CFG_PROFILE) != 0;
     if (profile && c->n_units > 1) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single launch unit");
-    const bool graph_mode = c->n_units == 1 && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
+    const bool graph_mode = !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
     for (auto e : c->prof_ev) cudaEventDestroy(e);
     c->prof_ev.clear();
     c->prof_kind.clear();
     memset(&c->prof, 0, sizeof(c->prof));
     cudaEvent_t init_a = nullptr, init_b = nullptr;
-    if (graph_mode) {
+    if (graph_mode && c->n_units == 1) {
         CK(cudaSetDevice(c->dev[0]));
         st = capture_graph(c, alg, d, make_launch(c, 0, alg));
         if (st != GUM_OK) return st;
+    } else if (graph_mode) {
+        for (int u = 0; u < c->n_units; u++) {
+            if (!unit_local(c, u)) continue;
+            st = capture_unit_graph(c, alg, u, d, make_launch(c, u, alg));
+            if (st != GUM_OK) return st;
+        }
     }
     CK(cudaSetDevice(c->dev[0]));
     CK(cudaEventRecord(c->ev0, c->stream[0]));
     c->launches = 0;
+    c->hlaunch = 0;
     if (c->n_units > 1) {
         st = unit_barrier(c);
         if (st != GUM_OK) return st;
@@ -1725,8 +1792,20 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         c->launches += 2 + ((src_frag >= L.w0 && src_frag < L.w0 + L.nw) ? 1 : 0);
     }
     if (profile) CK(cudaEventRecord(init_b, c->stream[0]));
-    if (graph_mode) {
+    if (graph_mode && c->n_units > 1) {
+        for (int u = 0; u < c->n_units; u++) {
+            if (!unit_local(c, u)) continue;
+            CK(cudaSetDevice(unit_dev(c, u)));
+            CK(cudaGraphLaunch(c->gexec_u[alg][u], c->stream[unit_w0(c, u)]));
+            c->hlaunch++;
+        }
+        if (c->mp) {  // peers read this rank's fragment until they finish: leave together (device barrier)
+            st = unit_barrier(c);
+            if (st != GUM_OK) return st;
+        }
+    } else if (graph_mode) {
         CK(cudaGraphLaunch(c->gexec[alg], c->stream[0]));
+        c->hlaunch++;
         if (getenv("GUM_DEBUG")) {  // watchdog: sample the run control block from a side stream
             cudaStream_t side;
             cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking);
@@ -1819,6 +1898,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
 #endif
     c->last_alg = alg;
     c->last_iters = R.iter;
+    if (R.err == 2) return fail(c, GUM_ENCCL, "device barrier timeout: a unit never arrived");
     if (R.err) return fail(c, GUM_ERANGE, "SSSP distance reached 2^32-1");
     if (stats) {
         memset(stats, 0, sizeof(*stats));
@@ -1831,9 +1911,30 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         stats->blocked_iterations = R.blocked_iters;
         stats->bodies = R.bodies;
         stats->kernel_launches = c->launches;
-        if (graph_mode) {
+        stats->host_launches = c->launches + c->hlaunch;
+        if (graph_mode && c->n_units == 1) {
             const LaunchCfg L0 = make_launch(c, 0, alg);
             stats->kernel_launches += (unsigned long long)(R.iter + 1) * (count_phase(alg, 0, d, L0) + count_phase(alg, 1, d, L0));
+        } else if (graph_mode) {
+            // per local unit: its executed bodies (control launches that did work, + the exiting one)
+            for (int u = 0; u < c->n_units; u++) {
+                if (!unit_local(c, u)) continue;
+                RunCtl ru;
+                CK(cudaSetDevice(unit_dev(c, u)));
+                CK(cudaMemcpy(&ru, c->rctl[unit_w0(c, u)], sizeof(RunCtl), cudaMemcpyDeviceToHost));
+                const LaunchCfg Lu = make_launch(c, u, alg);
+                stats->kernel_launches += (unsigned long long)(ru.bodies + 1) * (count_phase(alg, 0, d, Lu) + count_phase(alg, 1, d, Lu) + 2);
+            }
+        }
+        // device barrier arrivals per unit (multi-unit runs): an evicted unit stops arriving
+        for (int u = 0; u < c->n_units && c->n_units > 1; u++) {
+            unsigned long long pw[2] = {0, 0};
+            const unsigned long long* pu = c->pad[unit_w0(c, u)];
+            if (!pu) continue;
+            CK(cudaSetDevice(unit_dev(c, u)));
+            CK(cudaMemcpy(pw, pu + kPadArr, 16, cudaMemcpyDeviceToHost));
+            stats->unit_barriers[u] = (uint32_t)pw[0];
+            stats->unit_last_iter[u] = (uint32_t)pw[1];
         }
         unsigned long long qedges_total = 0;
         for (int f = 0; f < c->P; f++) {
