@@ -42,6 +42,9 @@ def _load():
     lib.oracle_pagerank.restype = ctypes.c_int
     lib.oracle_pagerank.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_int, ctypes.c_double,
                                     pd, pd]
+    lib.oracle_delta_pagerank.restype = ctypes.c_int
+    lib.oracle_delta_pagerank.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_double, ctypes.c_double,
+                                          pd, pd, ctypes.POINTER(ctypes.c_uint32)]
     lib.oracle_pagerank_pull.restype = ctypes.c_int
     lib.oracle_pagerank_pull.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_int, ctypes.c_double,
                                          ctypes.c_int, pd, pd, ctypes.POINTER(ctypes.c_int)]
@@ -144,6 +147,30 @@ def pagerank_pull(V, src, dst, iterations=20, damping=0.85, threads=0, return_re
     return x, used.value
 
 
+def dpr_epsilon(V, tolerance=1e-6, damping=0.85):
+    """Residual threshold of delta-PageRank for a target L1 tolerance (reading #27):
+    eps = tolerance * (1 - d) / V, so that sum(x* - x) <= V * eps / (1 - d) = tolerance."""
+    return tolerance * (1.0 - damping) / float(V)
+
+
+def delta_pagerank(V, src, dst, damping=0.85, eps=None, tolerance=1e-6, return_state=False):
+    """NEXT-4 delta-PageRank (residual push in BSP rounds). Returns x, or (x, r, rounds)."""
+    src, dst = _u32(src), _u32(dst)
+    if eps is None:
+        eps = dpr_epsilon(V, tolerance, damping)
+    x = np.empty(int(V), dtype=np.float64)
+    r = np.empty(int(V), dtype=np.float64)
+    rounds = ctypes.c_uint32(0)
+    rc = _load().oracle_delta_pagerank(int(V), int(src.shape[0]), _p(src, ctypes.c_uint32), _p(dst, ctypes.c_uint32),
+                                       float(damping), float(eps), _p(x, ctypes.c_double), _p(r, ctypes.c_double),
+                                       ctypes.byref(rounds))
+    if rc != 0:
+        raise ValueError(f"oracle_delta_pagerank rc={rc}")
+    if return_state:
+        return x, r, rounds.value
+    return x
+
+
 def run(alg: str, g, source: int = 0, pr_iterations: int = 20, pr_damping: float = 0.85):
     """Convenience: run one algorithm on an inputs.EdgeList."""
     if alg == "bfs":
@@ -154,4 +181,6 @@ def run(alg: str, g, source: int = 0, pr_iterations: int = 20, pr_damping: float
         return wcc(g.num_vertices, g.src, g.dst)
     if alg == "pr":
         return pagerank(g.num_vertices, g.src, g.dst, pr_iterations, pr_damping)
+    if alg == "dpr":
+        return delta_pagerank(g.num_vertices, g.src, g.dst, pr_damping)
     raise ValueError(alg)

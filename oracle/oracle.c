@@ -277,3 +277,58 @@ int oracle_pagerank_pull(uint32_t V, uint64_t E, const uint32_t* src, const uint
     free(outdeg); free(in_ptr); free(in_src); free(x); free(cx); free(y);
     return 0;
 }
+
+/* ---- NEXT-4 delta-PageRank (§I: "delta-PageRank, SSSP, and BFS" suffer the long tail) ----
+ * DESIGN.md reading #27. The paper names the algorithm without defining it; the reading is the
+ * residual-push ("delta") formulation of PageRank run as frontier-driven BSP rounds:
+ *   target  x* = the unique solution of x = (1-d)/V + d * sum_{(u,v) in E} x_u / outdeg(u)
+ *           (a dangling vertex's mass is not redistributed -- the delta-based variant of the literature);
+ *   state   x = 0, residual r = (1-d)/V for every vertex;
+ *   round   F = { u : r_u > eps } in vertex order. Every u in F first hands its residual over
+ *           (x_u += r_u, push_u = d*r_u/outdeg(u) or 0 if dangling, r_u = 0); then for each u in F and each
+ *           out-edge (u, v) in edge order, r_v += push_u.
+ *   stop    F empty. rounds_out = number of rounds with a non-empty F.
+ * The identity x + (I - d P^T)^{-1} r = x* holds after every round, so 0 <= x* - x componentwise and
+ * sum(x* - x) <= sum(r) / (1 - d) <= V * eps / (1 - d) at the end (pinned in tests/test_oracle.py).        */
+int oracle_delta_pagerank(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, double d, double eps,
+                          double* x, double* r, uint32_t* rounds_out) {
+    if (V == 0) return 0;
+    uint64_t* row_ptr = (uint64_t*)calloc((size_t)V + 1, sizeof(uint64_t));
+    uint32_t* adj = (uint32_t*)malloc(sizeof(uint32_t) * (size_t)(E ? E : 1));
+    double* push = (double*)malloc(sizeof(double) * V);
+    uint32_t* F = (uint32_t*)malloc(sizeof(uint32_t) * V);
+    if (!row_ptr || !adj || !push || !F) {
+        free(row_ptr); free(adj); free(push); free(F);
+        return -2;
+    }
+    if (oracle_build_adj(V, E, src, dst, NULL, row_ptr, adj, NULL) != 0) {
+        free(row_ptr); free(adj); free(push); free(F);
+        return -1;
+    }
+    for (uint32_t v = 0; v < V; v++) {
+        x[v] = 0.0;
+        r[v] = (1.0 - d) / (double)V;
+    }
+    uint32_t rounds = 0;
+    for (;;) {
+        size_t nf = 0;
+        for (uint32_t v = 0; v < V; v++)
+            if (r[v] > eps) F[nf++] = v;
+        if (nf == 0) break;
+        rounds++;
+        for (size_t i = 0; i < nf; i++) {
+            uint32_t u = F[i];
+            uint64_t od = row_ptr[u + 1] - row_ptr[u];
+            x[u] += r[u];
+            push[u] = od ? d * r[u] / (double)od : 0.0;
+            r[u] = 0.0;
+        }
+        for (size_t i = 0; i < nf; i++) {
+            uint32_t u = F[i];
+            for (uint64_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) r[adj[e]] += push[u];
+        }
+    }
+    if (rounds_out) *rounds_out = rounds;
+    free(row_ptr); free(adj); free(push); free(F);
+    return 0;
+}

@@ -387,3 +387,82 @@ def test_pr_pull_torus_uniform():
     x, _ = oracle.pagerank_pull(g.num_vertices, g.src, g.dst, 20, 0.85, threads=3)
     assert np.allclose(x, 1.0 / g.num_vertices, rtol=1e-13, atol=0)
     assert abs(x.sum() - 1.0) < 1e-12
+
+
+# ---- NEXT-4 delta-PageRank (reading #27): pinned to the target fixpoint x* (a linear solve, not the
+# push), closed forms and networkx
+def dpr_fixpoint(g, d=0.85):
+    """x* = (I - d P^T)^{-1} (1-d)/V with P = D^{-1} A (multiplicity counted; dangling rows zero)."""
+    V = g.num_vertices
+    A = sp.coo_matrix((np.ones(g.num_edges), (g.src.astype(np.int64), g.dst.astype(np.int64))), shape=(V, V)).tocsr()
+    out = np.asarray(A.sum(axis=1)).ravel()
+    inv = np.divide(1.0, out, out=np.zeros_like(out), where=out > 0)
+    P = sp.diags(inv) @ A
+    M = sp.identity(V, format="csc") - d * P.T.tocsc()
+    import scipy.sparse.linalg as spla
+    return spla.spsolve(M, np.full(V, (1 - d) / V)), M
+
+
+def check_dpr_bounds(g, x, r, eps, d=0.85):
+    xs, M = dpr_fixpoint(g, d)
+    import scipy.sparse.linalg as spla
+    V = g.num_vertices
+    assert np.all(r <= eps)  # converged: no residual above the threshold
+    assert np.all(x <= xs * (1 + 1e-12) + 1e-300)  # x approaches x* from below
+    gap = float((xs - x).sum())
+    assert -1e-12 <= gap <= V * eps / (1 - d) + 1e-12
+    # bookkeeping identity x + (I - d P^T)^{-1} r = x*
+    assert np.allclose(x + spla.spsolve(M, r), xs, rtol=1e-10, atol=1e-15)
+
+
+def test_dpr_directed_cycle_closed_form():
+    n, d = 50, 0.85
+    g = inputs.from_pairs(n, [(i, (i + 1) % n) for i in range(n)])
+    eps = oracle.dpr_epsilon(n, 1e-6)
+    x, r, K = oracle.delta_pagerank(n, g.src, g.dst, d, eps=eps, return_state=True)
+    # every vertex holds (1-d) d^k / V in round k; it is active while that exceeds eps
+    K_ref = 0
+    while (1 - d) * d ** K_ref / n > eps:
+        K_ref += 1
+    assert K == K_ref
+    assert np.allclose(x, (1 - d ** K_ref) / n, rtol=1e-12, atol=0)
+
+
+def test_dpr_in_star_exact():
+    n, d = 20, 0.85  # leaves 1..n -> centre 0 (the centre is dangling)
+    V = n + 1
+    g = inputs.from_pairs(V, [(i, 0) for i in range(1, V)])
+    x, r, K = oracle.delta_pagerank(V, g.src, g.dst, d, tolerance=1e-9, return_state=True)
+    t = (1 - d) / V
+    assert K == 2
+    assert np.allclose(x[1:], t, rtol=1e-15) and abs(x[0] - (t + d * n * t)) < 1e-16
+    assert np.all(r == 0)
+
+
+@settings(max_examples=30, deadline=None)
+@given(st.integers(1, 60), st.integers(0, 300), st.integers(0, 2**32 - 1), st.sampled_from([1e-3, 1e-6, 1e-9]))
+def test_dpr_bounds_random(V, E, seed, tol):
+    rng = np.random.default_rng(seed)
+    g = random_graph(rng, V, E)
+    eps = oracle.dpr_epsilon(V, tol)
+    x, r, _ = oracle.delta_pagerank(V, g.src, g.dst, 0.85, eps=eps, return_state=True)
+    check_dpr_bounds(g, x, r, eps)
+
+
+def test_dpr_rmat_bounds_and_networkx():
+    g = inputs.rmat(11, 8, seed=21, weighted=False)
+    eps = oracle.dpr_epsilon(g.num_vertices, 1e-7)
+    x, r, K = oracle.delta_pagerank(g.num_vertices, g.src, g.dst, 0.85, eps=eps, return_state=True)
+    check_dpr_bounds(g, x, r, eps)
+    assert K > 20  # the frontier-driven rounds have a long tail (P:31)
+    # no dangling vertex (a self-loop on every vertex): x* is the normalised PageRank networkx computes
+    V = 512
+    pairs = [(v, v) for v in range(V)] + list(zip(*np.random.default_rng(3).integers(0, V, (2, 3000)).tolist()))
+    h = inputs.from_pairs(V, pairs)
+    xh = oracle.delta_pagerank(V, h.src, h.dst, 0.85, tolerance=1e-9)
+    G = nx.MultiDiGraph()
+    G.add_nodes_from(range(V))
+    G.add_edges_from(zip(h.src.tolist(), h.dst.tolist()))
+    ref = nx.pagerank(G, alpha=0.85, tol=1e-15, max_iter=1000)
+    ref = np.array([ref[i] for i in range(V)])
+    assert float(np.abs(xh - ref).sum()) <= 1e-9 + 1e-12
