@@ -43,7 +43,11 @@ typedef enum {
 /* Algorithms. Outputs (reading #1): BFS hop depth, SSSP distance (uint32 weights,
  * uint64 arithmetic), WCC = minimum ORIGINAL vertex id of the weakly connected component,
  * PR = x_K of the fixed-K power iteration with uniform dangling redistribution (fp64). */
-typedef enum { GUM_BFS = 0, GUM_SSSP = 1, GUM_WCC = 2, GUM_PR = 3 } gum_alg;
+/* GUM_DPR (NEXT-4, "delta-PageRank"): residual-push PageRank in frontier-driven rounds (DESIGN.md
+ * reading #27): x -> x* = (I - d P^T)^{-1} (1-d)/V (dangling mass not redistributed), every vertex whose
+ * residual exceeds eps = dpr_tolerance * (1-d)/V is active; output x as double[V], with
+ * 0 <= x* - x and sum(x* - x) <= dpr_tolerance. */
+typedef enum { GUM_BFS = 0, GUM_SSSP = 1, GUM_WCC = 2, GUM_PR = 3, GUM_DPR = 4 } gum_alg;
 
 /* Partitioners (P:315, P:382 Exp-6): SEG = contiguous id ranges with ~equal out-edges; RANDOM =
  * keyed Feistel relabel of ids, then SEG (reading #17). metis is out of scope.
@@ -161,6 +165,9 @@ typedef struct {
      * out-edge into the destination's accumulator (the GAS scatter of P:53; also used whenever mirrors = 1,
      * whose aggregation is a push). Results agree within the PR tolerance either way. */
     int pr_push;
+    /* delta-PageRank (GUM_DPR): target L1 tolerance; the residual threshold is dpr_tolerance * (1-d)/V
+     * (0 => 1e-6). Damping is pr_damping. */
+    double dpr_tolerance;
 } gum_config;
 
 /* Fills *cfg with the defaults: 1 worker, fsteal=1, osteal=1, t1=t2=0, osteal threshold 0 (off until

@@ -23,7 +23,7 @@ LIB_PATH = os.environ.get("GUM_LIB") or os.path.join(_HERE, "libgum.so")  # GUM_
 GUM_OK, GUM_EINVAL, GUM_ENOMEM, GUM_ESTATE, GUM_ERANGE, GUM_ECUDA, GUM_ENCCL, GUM_EUNSUP = 0, -1, -2, -3, -4, -5, -6, -7
 STATUS_NAMES = {0: "GUM_OK", -1: "GUM_EINVAL", -2: "GUM_ENOMEM", -3: "GUM_ESTATE", -4: "GUM_ERANGE",
                 -5: "GUM_ECUDA", -6: "GUM_ENCCL", -7: "GUM_EUNSUP"}
-ALGS = {"bfs": 0, "sssp": 1, "wcc": 2, "pr": 3}
+ALGS = {"bfs": 0, "sssp": 1, "wcc": 2, "pr": 3, "dpr": 4}
 PARTS = {"seg": 0, "random": 1, "degree": 2}
 INF = 0xFFFFFFFF
 MAX_WORKERS = 8
@@ -61,7 +61,7 @@ class gum_config(ctypes.Structure):
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p)),
                 ("mirrors", ctypes.c_int), ("hub_cache", ctypes.c_int), ("hub_degree", ctypes.c_uint32),
-                ("pr_push", ctypes.c_int)]
+                ("pr_push", ctypes.c_int), ("dpr_tolerance", ctypes.c_double)]
 
 
 EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p)
@@ -209,7 +209,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=16384,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
                 use_torch_allocator=False, streams=None, osteal_sync_edges=0.0, mirrors=False, hub_cache=False,
-                hub_degree=0, pr_push=False):
+                hub_degree=0, pr_push=False, dpr_tolerance=1e-6):
     """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
     config points to and must live as long as the context."""
     lib = load_library()
@@ -241,6 +241,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
     cfg.hub_cache = int(bool(hub_cache))      # NEXT-1 hub adjacency caching
     cfg.hub_degree = int(hub_degree)          # t4
     cfg.pr_push = int(bool(pr_push))          # PR advance: pull over source blocks (default) or push
+    cfg.dpr_tolerance = float(dpr_tolerance)  # delta-PageRank: L1 tolerance (eps = tol * (1-d) / V)
     flags = 0
     if trace:
         flags |= CFG_TRACE
@@ -367,7 +368,7 @@ class Context:
         return RunStats(**vals)
 
     def result(self, out=None):
-        dt = np.float64 if self._last_alg == "pr" else np.uint32
+        dt = np.float64 if self._last_alg in ("pr", "dpr") else np.uint32
         if out is None:
             out = np.empty(self.num_vertices, dtype=dt)
         nbytes = out.nbytes if hasattr(out, "nbytes") else out.numel() * out.element_size()

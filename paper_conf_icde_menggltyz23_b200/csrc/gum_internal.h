@@ -220,6 +220,7 @@ struct DevCtx {
     unsigned int max_iter;
     int pr_iters;
     double pr_d;
+    double dpr_eps;             // delta-PageRank residual threshold (absolute)
     unsigned int force_mode;    // 0 auto, 1 sparse, 2 dense
     unsigned int dense_div;     // dense filter iff app_cnt > V_f / dense_div
     unsigned int nf_delta;      // SSSP near-far split increment (0 = plain BSP frontier, the paper's)

@@ -77,7 +77,12 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         if (i < F.V) {
             if (ALG == ALG_BFS || ALG == ALG_SSSP) F.state[i] = GUM_INF;
             if (ALG == ALG_WCC) F.state[i] = F.orig ? F.orig[i] : F.base + i;
-            if (ALG == ALG_WCC || ALG == ALG_PR) F.app[i] = i;  // all-active frontier as a list too
+            if (ALG == ALG_WCC || ALG == ALG_PR || ALG == ALG_DPR) F.app[i] = i;  // all-active frontier as a list too
+            if (ALG == ALG_DPR) {  // delta-PR: x = 0, residual (in acc) = (1-d)/V, every vertex active
+                F.x[i] = 0.0;
+                F.acc[i] = (1.0 - c.pr_d) / (double)c.num_vertices;
+                F.cx[i] = 0.0;
+            }
             if (ALG == ALG_PR) {
                 const double x0 = 1.0 / (double)c.num_vertices;
                 const unsigned long long od = F.row_ptr[i + 1] - F.row_ptr[i];
@@ -89,7 +94,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         }
         if (i < nwords) {
             unsigned wv = 0;
-            if (ALG == ALG_PR || (ALG == ALG_WCC && !F.sq_col)) {
+            if (ALG == ALG_PR || ALG == ALG_DPR || (ALG == ALG_WCC && !F.sq_col)) {
                 unsigned rem = F.V - i * 32;
                 wv = rem >= 32 ? 0xFFFFFFFFu : ((1u << rem) - 1u);
             }
@@ -118,7 +123,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->ntiles = (ALG == ALG_PR) ? (F.pr_qedges + c.chunk - 1) / c.chunk : (sq ? (F.sq_edges + c.chunk - 1) / c.chunk : 0);
         ct->qlen = (ALG == ALG_PR) ? F.pr_qlen : (sq ? F.sq_len : 0);
         ct->qedges = (ALG == ALG_PR) ? F.pr_qedges : (sq ? F.sq_edges : 0);
-        ct->app_cnt = (ALG == ALG_WCC && !sq) ? F.V : 0;
+        ct->app_cnt = ((ALG == ALG_WCC && !sq) || ALG == ALG_DPR) ? F.V : 0;
         ct->err = 0;
         ct->dense = 0;
         ct->pr_dang[0] = ct->pr_dang[1] = 0.0;
@@ -388,10 +393,19 @@ __device__ __forceinline__ void nf_flush(FragCtl* ct, unsigned fslot, const NfAc
     }
 }
 
-template <int MODE>
+// delta-PR (reading #27): an activated vertex hands its residual over when the filter takes it into the next
+// frontier: x += r, push value cx = d*r/outdeg (0 for a dangling vertex), r = 0 (BSP: no advance runs now)
+__device__ __forceinline__ void dpr_take(const FragPtrs& F, unsigned v, unsigned long long od, double dd) {
+    const double dl = F.acc[v];
+    F.x[v] += dl;
+    F.acc[v] = 0.0;
+    F.cx[v] = od ? dd * dl / (double)od : 0.0;
+}
+
+template <int MODE, bool DPR = false>
 __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool keep_fbm, unsigned depth, unsigned tile, bool dense, bool sweep,
                                             bool nf, unsigned nfT, unsigned nwords, unsigned app_cnt, unsigned ipt,
-                                            unsigned chunk, unsigned long long pos, unsigned long long off) {
+                                            unsigned chunk, unsigned long long pos, unsigned long long off, double dd = 0.0) {
     const unsigned lane = lane_id();
     Pair mine{0, 0};
     if (dense) {
@@ -450,6 +464,11 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
 #pragma unroll
                 for (int q = 0; q <= kDenseVertsPerThread; q++) rpv[q] = (vb + q <= F.V) ? __ldg(rp + q) : 0ull;
             }
+            if (DPR && MODE == FT_EMIT) {
+#pragma unroll
+                for (int q = 0; q < kDenseVertsPerThread; q++)
+                    if ((bits >> q) & 1u) dpr_take(F, vb + q, rpv[q + 1] - rpv[q], dd);
+            }
             static_assert(kDenseVertsPerThread == 8, "filter_accept8 takes 8 candidates");
             unsigned vs[8], cand = 0;
 #pragma unroll
@@ -489,6 +508,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
                 if (MODE == FT_EMIT && depth != GUM_INF) F.state[v] = depth;  // BFS (see the dense path)
                 rp0[j] = __ldg(F.row_ptr + v);
                 d[j] = __ldg(F.row_ptr + v + 1) - rp0[j];
+                if (DPR && MODE == FT_EMIT) dpr_take(F, v, d[j], dd);
             }
         }
         static_assert(kFilterAppPerThread == 8, "filter_accept8 takes 8 candidates");
@@ -513,9 +533,10 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
 // block scan for the per-thread offsets and the emit in one walk of the tile (FT_COUNT + FT_EMIT read the
 // bitmap word and the row_ptr run twice). Only the 8-bit accepted mask stays live across the scan; the
 // row_ptr run is re-read after it from L1 (the same thread's lines). Returns the tile's totals.
+template <bool DPR = false>
 __device__ __forceinline__ Pair filter_tile_dense_fused(const FragPtrs& F, bool keep_fbm, unsigned depth, unsigned tile,
                                                         unsigned nwords, unsigned chunk, unsigned long long pos,
-                                                        unsigned long long off, Pair* s_warp) {
+                                                        unsigned long long off, Pair* s_warp, double dd = 0.0) {
     const unsigned lane = lane_id();
     const unsigned wbase = tile * kDenseWordsPerPart + (threadIdx.x >> 5) * kDenseWordsPerWarp;
     const unsigned vb = wbase * 32u + lane * kDenseVertsPerThread;
@@ -566,6 +587,11 @@ __device__ __forceinline__ Pair filter_tile_dense_fused(const FragPtrs& F, bool 
 #pragma unroll
             for (int q = 0; q <= kDenseVertsPerThread; q++) rpv[q] = (vb + q <= F.V) ? __ldg(rp + q) : 0ull;
         }
+        if (DPR) {
+#pragma unroll
+            for (int q = 0; q < kDenseVertsPerThread; q++)
+                if ((bits >> q) & 1u) dpr_take(F, vb + q, rpv[q + 1] - rpv[q], dd);
+        }
 #pragma unroll
         for (int q = 0; q < kDenseVertsPerThread; q++) {
             if (((bits >> q) & 1u) && rpv[q + 1] != rpv[q]) {
@@ -607,7 +633,7 @@ __device__ unsigned g_fcall;
 #endif
 // NF: SSSP near-far parking compiled in (its batched state loads and far-bit atomics cost registers the
 // other algorithms' filters do not need)
-template <bool NF>
+template <bool NF, bool DPR = false>
 __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
     FT_MARK(0);
     // Prologue by thread 0 only, broadcast through shared memory: the run-control fields are a handful of
@@ -655,6 +681,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     const unsigned app_cnt = s_pro.app_cnt;
     const bool keep_fbm = c.wcc_blocked != 0 && !nf;
     const unsigned depth = s_pro.depth;
+    const double dd = DPR ? c.pr_d : 0.0;
     const unsigned nwords = (F.V + 31) / 32;
     const unsigned long long n_items = dense ? nwords : app_cnt;
     // sparse lists: items per thread so that the tiles cover the grid (1..8)
@@ -689,7 +716,7 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     Pair mine{0, 0};
     NfAcc nfa;
     for (unsigned t = t_lo; t < t_hi; t++) {
-        const Pair q = filter_tile<FT_CLASSIFY>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+        const Pair q = filter_tile<FT_CLASSIFY, DPR>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0, dd);
         mine.cnt += q.cnt;
         mine.deg += q.deg;
     }
@@ -730,28 +757,28 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     unsigned long long run_cnt = excl.cnt, run_deg = excl.deg;
     if (t_hi - t_lo == 1) {
         // one tile: pass 1's per-thread counts are this tile's (same acceptance), no re-count
-        filter_tile<FT_EMIT>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t_lo * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
-                             run_deg + tex1.deg);
+        filter_tile<FT_EMIT, DPR>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t_lo * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex1.cnt,
+                                  run_deg + tex1.deg, dd);
         filter_flush_long(F);
     } else {
         for (unsigned t = t_lo; t < t_hi; t++) {
             const unsigned pt = (unsigned)((unsigned long long)t * stride % n_tiles);
             if (dense && !nf) {
-                const Pair tot = filter_tile_dense_fused(F, keep_fbm, depth, pt, nwords, chunk, run_cnt, run_deg, s_warp);
+                const Pair tot = filter_tile_dense_fused<DPR>(F, keep_fbm, depth, pt, nwords, chunk, run_cnt, run_deg, s_warp, dd);
                 filter_flush_long(F);
                 run_cnt += tot.cnt;
                 run_deg += tot.deg;
                 continue;
             }
-            const Pair q = filter_tile<FT_COUNT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0);
+            const Pair q = filter_tile<FT_COUNT, DPR>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0, dd);
             Pair tot;
 #ifdef GUM_PACK2
             const Pair tex = block_excl_scan_tile(q, s_warp, tot);  // A/B variant "pack2" (filter 0.390 ms/run on C2)
 #else
             const Pair tex = block_excl_scan(q, s_warp, tot);  // "pack": packed scan in the fused dense tile only (0.384)
 #endif
-            filter_tile<FT_EMIT>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
-                                 run_deg + tex.deg);
+            filter_tile<FT_EMIT, DPR>(F, nfa, keep_fbm, depth, pt, dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, run_cnt + tex.cnt,
+                                      run_deg + tex.deg, dd);
             filter_flush_long(F);
             run_cnt += tot.cnt;
             run_deg += tot.deg;
@@ -1055,6 +1082,10 @@ template <>
 struct ValT<ALG_PR> {
     typedef double T;
 };
+template <>
+struct ValT<ALG_DPR> {
+    typedef double T;
+};
 
 // Warp-aggregated append of this thread's activations (bit j of need: slot j) to the owner
 // fragments' activation lists: one reservation atomic per warp and target fragment.
@@ -1258,7 +1289,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     auto chunk_ref = [&](int f, unsigned long long t, int stolen) {
         ChunkRef r{f, t, stolen, 0u, 0u, 0u, false};
         if (f < 0) return r;
-        r.hc = MULTI && NX && ALG != ALG_PR && c.hub_on && f != w;
+        r.hc = MULTI && NX && ALG != ALG_PR && ALG != ALG_DPR && c.hub_on && f != w;
         const FragPtrs& F = c.f[f];
         const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned* const tilep = sq ? F.sq_tile : F.tile;
@@ -1293,7 +1324,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         }
     };
     auto value_of = [&](const ChunkRef& r, unsigned u) -> VT {
-        if (ALG == ALG_PR) return (VT)__ldcg(c.f[r.f].cx + u);
+        if (ALG == ALG_PR || ALG == ALG_DPR) return (VT)__ldcg(c.f[r.f].cx + u);
         // masked blocked pass: a source outside the frontier (its bit clear in the filter's copy) gets the
         // value INF, and its edges are skipped in the expansion
         if (ALG == ALG_WCC && blk == 2 && !((__ldcg(c.f[r.f].far + (u >> 5)) >> (u & 31)) & 1u)) return (VT)GUM_INF;
@@ -1441,7 +1472,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                 if (MULTI && NX) hub_e += hv ? 1 : 0;
                 vv[j] = __ldcs((hv ? c.hub[w][f].col : colp) + ci);
                 if (ALG == ALG_BFS) cv[j] = (VT)(k + 1);  // every frontier vertex has depth k
-                if (ALG == ALG_WCC || ALG == ALG_PR) cv[j] = s_val[kk];
+                if (ALG == ALG_WCC || ALG == ALG_PR || ALG == ALG_DPR) cv[j] = s_val[kk];
                 if (ALG == ALG_SSSP) {
                     const unsigned long long nd = (unsigned long long)s_val[kk] + __ldcs((hv ? c.hub[w][f].w : F.w) + ci);
                     if (nd >= (unsigned long long)GUM_INF) {
@@ -1474,6 +1505,41 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                     }
                     atomicAdd(c.f[tf].acc + lv, (double)cv[j]);
                 }
+            }
+        } else if (ALG == ALG_DPR) {
+            // delta-PR apply (reading #27): add d*delta_u/outdeg(u) to the destination's residual with a
+            // returning atom.add.f64; the add that lifts the residual above eps activates v (residuals only
+            // grow during an advance, so exactly one add per vertex and round crosses)
+            unsigned lvv[kEdgesPerThread];
+            unsigned char tfv[kEdgesPerThread];
+            double old[kEdgesPerThread];
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++) {
+                tfv[j] = 0;
+                lvv[j] = vv[j];
+                old[j] = 0.0;
+                if (vv[j] != GUM_INF) {
+                    if (MULTI) {
+                        const int tf = frag_of(c, vv[j]);
+                        tfv[j] = (unsigned char)tf;
+                        lvv[j] = vv[j] - c.bounds[tf];
+                        remote += (s_owner[tf] != (unsigned)w) ? 1 : 0;
+                    }
+                    old[j] = atomicAdd(c.f[tfv[j]].acc + lvv[j], (double)cv[j]);
+                }
+            }
+            const double eps = c.dpr_eps;
+            unsigned upd = 0;
+#pragma unroll
+            for (int j = 0; j < kEdgesPerThread; j++)
+                if (vv[j] != GUM_INF && old[j] <= eps && old[j] + (double)cv[j] > eps) upd |= 1u << j;
+            if (next_dense) {
+#pragma unroll
+                for (int j = 0; j < kEdgesPerThread; j++)
+                    if (upd & (1u << j)) atomicOr(c.f[tfv[j]].bm + (lvv[j] >> 5), 1u << (lvv[j] & 31));  // RED.OR
+                acts += __popc(upd);
+            } else {
+                acts += append_activations<MULTI>(c, upd, tfv, lvv);  // (one crossing per vertex: no dedupe)
             }
         } else if (ALG == ALG_BFS && pb) {
             // Propagation blocking (dense BFS iteration): instead of one random visited-bit probe per
@@ -2250,7 +2316,10 @@ cudaError_t tail_occupancy(int* blocks_per_sm) {
 
 template <int ALG>
 static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t s) {
-    if (ALG == ALG_PR || L.tail_grid <= 0) return cudaSuccess;
+    if constexpr (ALG == ALG_PR || ALG == ALG_DPR) {
+        return cudaSuccess;  // (no tail engine for the PageRank variants)
+    } else {
+    if (L.tail_grid <= 0) return cudaSuccess;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(L.tail_grid);
     cfg.blockDim = dim3(kTailThreads);
@@ -2262,6 +2331,7 @@ static cudaError_t launch_tail(const DevCtx& c, const LaunchCfg& L, cudaStream_t
     cfg.numAttrs = 1;
     if (c.P > 1) return cudaLaunchKernelEx(&cfg, k_tail<ALG, true>, c, L.w0);
     return cudaLaunchKernelEx(&cfg, k_tail<ALG, false>, c, L.w0);
+    }
 }
 
 // ------------------------------------------------------------------------------------------ bottom-up
@@ -2771,6 +2841,8 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
         case KER_FILTER:
             if (c.nf_delta)
                 k_filter<true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+            else if (ALG == ALG_DPR)
+                k_filter<false, true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
             else
                 k_filter<false><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
             break;
@@ -2818,6 +2890,7 @@ cudaError_t launch_kernel(int alg, int kind, const DevCtx& c, const LaunchCfg& L
         case ALG_BFS: return launch_kernel_t<ALG_BFS>(kind, c, L, s, h, use_h);
         case ALG_SSSP: return launch_kernel_t<ALG_SSSP>(kind, c, L, s, h, use_h);
         case ALG_WCC: return launch_kernel_t<ALG_WCC>(kind, c, L, s, h, use_h);
+        case ALG_DPR: return launch_kernel_t<ALG_DPR>(kind, c, L, s, h, use_h);
         default: return launch_kernel_t<ALG_PR>(kind, c, L, s, h, use_h);
     }
 }
@@ -2871,10 +2944,11 @@ cudaError_t launch_init(int alg, const DevCtx& c, const LaunchCfg& L, cudaStream
         case ALG_BFS: k_init<ALG_BFS><<<g, kThreads, 0, s>>>(c, f0); break;
         case ALG_SSSP: k_init<ALG_SSSP><<<g, kThreads, 0, s>>>(c, f0); break;
         case ALG_WCC: k_init<ALG_WCC><<<g, kThreads, 0, s>>>(c, f0); break;
+        case ALG_DPR: k_init<ALG_DPR><<<g, kThreads, 0, s>>>(c, f0); break;
         default: k_init<ALG_PR><<<g, kThreads, 0, s>>>(c, f0); break;
     }
     // the initial frontier: {source} as a list (BFS/SSSP) or every vertex as a full bitmap (WCC/PR)
-    const unsigned nd0 = c.force_mode == 1 ? 0u : ((alg == ALG_WCC || alg == ALG_PR) ? 1u : 0u);
+    const unsigned nd0 = c.force_mode == 1 ? 0u : ((alg == ALG_WCC || alg == ALG_PR || alg == ALG_DPR) ? 1u : 0u);
     k_init_run<<<1, 1, 0, s>>>(c, L.w0, D0, nd0, (alg == ALG_WCC && c.f[0].sq_col) ? 1u : 0u);
     if (src_frag >= f0 && src_frag < f0 + nf) k_init_source<<<1, 1, 0, s>>>(c, src_frag, src_local);
     return cudaGetLastError();
@@ -3038,6 +3112,8 @@ cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm) {
         carveout<ALG_WCC, true>();
         carveout<ALG_PR, false>();
         carveout<ALG_PR, true>();
+        carveout<ALG_DPR, false>();
+        carveout<ALG_DPR, true>();
     }
     switch (alg * 2 + (multi ? 1 : 0)) {
         case 0: return occ_of<ALG_BFS, false>(blocks_per_sm);
@@ -3047,7 +3123,9 @@ cudaError_t advance_occupancy(int alg, int multi, int* blocks_per_sm) {
         case 4: return occ_of<ALG_WCC, false>(blocks_per_sm);
         case 5: return occ_of<ALG_WCC, true>(blocks_per_sm);
         case 6: return occ_of<ALG_PR, false>(blocks_per_sm);
-        default: return occ_of<ALG_PR, true>(blocks_per_sm);
+        case 7: return occ_of<ALG_PR, true>(blocks_per_sm);
+        case 8: return occ_of<ALG_DPR, false>(blocks_per_sm);
+        default: return occ_of<ALG_DPR, true>(blocks_per_sm);
     }
 }
 

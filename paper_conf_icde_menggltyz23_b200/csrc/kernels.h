@@ -6,7 +6,8 @@
 
 namespace gum {
 
-enum { ALG_BFS = GUM_BFS, ALG_SSSP = GUM_SSSP, ALG_WCC = GUM_WCC, ALG_PR = GUM_PR };
+enum { ALG_BFS = GUM_BFS, ALG_SSSP = GUM_SSSP, ALG_WCC = GUM_WCC, ALG_PR = GUM_PR, ALG_DPR = GUM_DPR };
+constexpr int kNumAlgs = 5;
 
 // One launch unit = the workers [w0, w0+nw) that live on one device.
 struct LaunchCfg {

@@ -110,7 +110,7 @@ struct gum_ctx {
     int nsm = 148;
     int tail_occ = 1;
     int filter_occ = 2;
-    int adv_occ[4][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
+    int adv_occ[kNumAlgs][2] = {{4, 4}, {4, 4}, {4, 4}, {4, 4}, {4, 4}};  // advance CTAs per SM by [alg][multi]
     int pr_push_occ = 8;
     int pull_occ = 4;
     std::string err;
@@ -158,8 +158,8 @@ struct gum_ctx {
     TailSplit* tsplit[kMaxW] = {nullptr};
     RunCtl* h_rctl = nullptr;  // pinned
     void* d_res = nullptr;
-    cudaGraphExec_t gexec[4] = {nullptr, nullptr, nullptr, nullptr};
-    cudaGraphExec_t gexec_u[4][kMaxW] = {};  // device-resident multi-unit loop: one graph per unit
+    cudaGraphExec_t gexec[kNumAlgs] = {};
+    cudaGraphExec_t gexec_u[kNumAlgs][kMaxW] = {};  // device-resident multi-unit loop: one graph per unit
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     std::vector<cudaEvent_t> bar_ev;
     std::vector<cudaEvent_t> prof_ev;  // pairs (start, end)
@@ -339,7 +339,7 @@ LaunchCfg make_launch(const gum_ctx* c, int u, int alg) {
     // (the host-driven multi-unit loop has no run-control hand-over between units, so it keeps the tail engine
     // off: the other units' iteration counters would not follow the engine's iterations)
     const bool tail_ok = c->n_units == 1 || !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
-    L.tail_grid = (u == 0 && tail_ok && c->cfg.tail_vertices && alg != GUM_PR)
+    L.tail_grid = (u == 0 && tail_ok && c->cfg.tail_vertices && alg != GUM_PR && alg != GUM_DPR)
                       ? c->nsm * ((c->split && c->single_device && c->tail_occ > 1) ? c->tail_occ - 1 : c->tail_occ)
                       : 0;
     L.adv_grid_pr = c->nsm * c->pr_push_occ;
@@ -417,7 +417,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.mmin = (unsigned*)F.mbuf;
         d.lb[f] = c->lb[f];
     }
-    d.mirrors = (c->cfg.mirrors && c->P > 1 && c->fr[0].mbuf) ? 1 : 0;
+    d.mirrors = (c->cfg.mirrors && c->P > 1 && c->fr[0].mbuf && alg != GUM_DPR) ? 1 : 0;
     if (alg == GUM_PR && c->pl_ready) {
         // one replica of x/outdeg per launch unit; worker w pulls from its unit's
         d.pl_B = c->pl_B;
@@ -425,7 +425,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         for (int u = 0; u < c->n_units; u++) d.cxrep[u] = c->cxg[unit_w0(c, u)];
         for (int w = 0; w < c->P; w++) d.cxw[w] = c->cxg[unit_w0(c, c->split ? w : 0)];
     }
-    const int hk = alg == GUM_WCC ? 2 : (alg == GUM_PR ? -1 : 1);
+    const int hk = alg == GUM_WCC ? 2 : ((alg == GUM_PR || alg == GUM_DPR) ? -1 : 1);
     d.hub_on = (c->hub_kind == hk) ? 1 : 0;
     for (int w = 0; w < c->P && d.hub_on; w++)
         for (int f = 0; f < c->P; f++) {
@@ -458,10 +458,11 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.max_iter = c->cfg.max_iterations ? c->cfg.max_iterations : 0x7FFFFFFFu;
     d.pr_iters = c->cfg.pr_iterations;
     d.pr_d = c->cfg.pr_damping;
+    d.dpr_eps = (c->cfg.dpr_tolerance > 0.0 ? c->cfg.dpr_tolerance : 1e-6) * (1.0 - c->cfg.pr_damping) / (double)c->V;
     d.force_mode = (c->cfg.flags & GUM_CFG_FORCE_DENSE) ? 2u : ((c->cfg.flags & GUM_CFG_FORCE_SPARSE) ? 1u : 0u);
     d.dense_div = 32;
     d.nf_delta = alg == GUM_SSSP ? c->cfg.sssp_delta : 0u;
-    d.tail_enter = (alg != GUM_PR && (c->n_units == 1 || !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))))
+    d.tail_enter = (alg != GUM_PR && alg != GUM_DPR && (c->n_units == 1 || !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))))
                        ? c->cfg.tail_vertices
                        : 0u;
     d.tail_exit = 4u * c->cfg.tail_vertices;
@@ -1287,7 +1288,7 @@ gum_status gum_create(const gum_config* cfg, gum_ctx** out) {
     }
     cudaSetDevice(c->dev[0]);
     cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->dev[0]);
-    for (int a = 0; a < 4; a++)
+    for (int a = 0; a < kNumAlgs; a++)
         for (int m = 0; m < 2; m++) {
             int occ = 0;
             if (advance_occupancy(a, m, &occ) == cudaSuccess && occ > 0) c->adv_occ[a][m] = occ;
@@ -1327,7 +1328,7 @@ static unsigned long long config_hash(const gum_config* cfg) {
     GUM_HC(osteal_active_threshold); GUM_HC(osteal_edges_per_worker); GUM_HC(chunk_edges); GUM_HC(pr_iterations);
     GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
     GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt); GUM_HC(osteal_sync_edges);
-    GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree); GUM_HC(pr_push);
+    GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree); GUM_HC(pr_push); GUM_HC(dpr_tolerance);
 #undef GUM_HC
     return h;
 }
@@ -1707,7 +1708,7 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
     if (!c) return GUM_EINVAL;
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_prepare before gum_partition");
-    if (alg < 0 || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
+    if (alg < 0 || alg > GUM_DPR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
     gum_status st = GUM_OK;
     bool built = false;  // multi-process: new buffers must be published (all ranks agree: same state)
     if (alg == GUM_WCC) {
@@ -1730,7 +1731,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     if (!c) return GUM_EINVAL;
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->partitioned) return fail(c, GUM_ESTATE, "gum_run before gum_partition");
-    if (alg < GUM_BFS || alg > GUM_PR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
+    if (alg < GUM_BFS || alg > GUM_DPR) return fail(c, GUM_EINVAL, "bad algorithm %d", (int)alg);
     if (alg == GUM_SSSP && !c->has_w) return fail(c, GUM_EINVAL, "SSSP needs edge weights");
     if ((alg == GUM_BFS || alg == GUM_SSSP) && source >= c->V) return fail(c, GUM_ERANGE, "source %u >= V", source);
     gum_status st = gum_prepare(c, alg);
@@ -1973,7 +1974,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
 }
 
 static gum_status gather_result(gum_ctx* c, void* dst_dev) {
-    const bool pr = c->last_alg == GUM_PR;
+    const bool pr = c->last_alg == GUM_PR || c->last_alg == GUM_DPR;  // double results
     const DevCtx d = make_devctx(c, c->last_alg);
     for (int f = 0; f < c->P; f++) {
         CK(cudaSetDevice(c->fr[f].dev));
@@ -1987,7 +1988,7 @@ gum_status gum_result(gum_ctx* c, void* out, uint64_t out_bytes) {
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->has_result) return fail(c, GUM_ESTATE, "gum_result before a successful gum_run");
     if (!out) return fail(c, GUM_EINVAL, "null output buffer");
-    const size_t es = c->last_alg == GUM_PR ? 8 : 4;
+    const size_t es = (c->last_alg == GUM_PR || c->last_alg == GUM_DPR) ? 8 : 4;
     if (out_bytes < (uint64_t)c->V * es) return fail(c, GUM_EINVAL, "output buffer too small");
     gum_status st = gather_result(c, c->d_res);
     if (st != GUM_OK) return st;
@@ -2002,7 +2003,7 @@ gum_status gum_result_device(gum_ctx* c, void* out, uint64_t out_bytes) {
     if (c->poisoned) return fail(c, GUM_ESTATE, "context poisoned");
     if (!c->has_result) return fail(c, GUM_ESTATE, "gum_result_device before a successful gum_run");
     if (!out) return fail(c, GUM_EINVAL, "null output buffer");
-    const size_t es = c->last_alg == GUM_PR ? 8 : 4;
+    const size_t es = (c->last_alg == GUM_PR || c->last_alg == GUM_DPR) ? 8 : 4;
     if (out_bytes < (uint64_t)c->V * es) return fail(c, GUM_EINVAL, "output buffer too small");
     return gather_result(c, out);
 }
