@@ -92,11 +92,11 @@ typedef struct {
      * osteal_edges_per_worker), 1, num_gpus) (0 => m' = 1); above it ownership is given back.
      * Fragment f is owned by worker f if f < m', else by f mod m'.
      * osteal = 0: off; 1: this active-vertex threshold trigger (the north_star's rule, the default);
-     * 2: the paper's cost model (NEXT-3, Alg. 2 P:201-211 with Eq. (4)): every iteration,
+     * 2: the paper's cost model (NEXT-3, Alg. 2 P:188-211 with Eq. (4)): every iteration,
      * for m = 1..num_gpus, E(m) = z(m) + p*m with z(m) the Eq. (1) makespan when only workers {0..m-1}
      * process (evicted fragments' edges at the remote cost, see gum_osteal_plan) and p =
-     * osteal_sync_edges; the first m with the lowest E(m) becomes the active owner set (shrinking or
-     * giving ownership back). */
+     * osteal_sync_edges (or its online estimate); the first m with the lowest E(m) becomes the active
+     * owner set (shrinking or giving ownership back). */
     int osteal;
     uint64_t osteal_active_threshold;
     uint64_t osteal_edges_per_worker;
@@ -130,8 +130,10 @@ typedef struct {
      * depth among its in-edges). Same depths; 0 = push only (the paper's GUM, the default). */
     int bfs_direction_opt;
     /* OSteal cost model (osteal = 2): p of Eq. (4), the per-worker synchronisation cost of one
-     * iteration expressed in edge-processing time units (edges); 0 => 500000 (B200: ~3.5 us of
-     * per-unit launch + barrier cost at ~7 ps per expanded edge). */
+     * iteration expressed in edge-processing time units (edges). > 0: this constant. 0 (default):
+     * estimated during the run from previous iterations: p = S / (m * tau) with S the measured
+     * non-advance time of an iteration and tau the advance time per edge and worker, averaged over
+     * iterations (reading #23); 500000 until the first measurement. */
     double osteal_sync_edges;
     /* Optional device allocator (e.g. the PyTorch caching allocator) and per-worker streams. */
     void* (*alloc)(uint64_t bytes, int device, void* user);
@@ -213,6 +215,11 @@ typedef struct {
     /* host-side launches of this process in the run (kernels + graph launches): in the device-resident
      * loops this does not depend on the number of iterations */
     uint64_t host_launches;
+    /* OSteal cost model (osteal = 2): p of Eq. (4) used at the end of the run (edges) and the number of
+     * iterations it was estimated from (0 = the configured / initial value) */
+    double osteal_p;
+    uint32_t osteal_p_samples;
+    uint32_t pad1;
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

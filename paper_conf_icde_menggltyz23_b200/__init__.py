@@ -84,7 +84,8 @@ class gum_run_stats(ctypes.Structure):
                 ("mirror_flush_bytes", ctypes.c_uint64), ("blocked_iterations", ctypes.c_uint32),
                 ("pad0", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
                 ("tail_activations", ctypes.c_uint64), ("unit_barriers", ctypes.c_uint32 * MAX_WORKERS),
-                ("unit_last_iter", ctypes.c_uint32 * MAX_WORKERS), ("host_launches", ctypes.c_uint64)]
+                ("unit_last_iter", ctypes.c_uint32 * MAX_WORKERS), ("host_launches", ctypes.c_uint64),
+                ("osteal_p", ctypes.c_double), ("osteal_p_samples", ctypes.c_uint32), ("pad1", ctypes.c_uint32)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -202,6 +203,9 @@ class RunStats:
     unit_barriers: list = None
     unit_last_iter: list = None
     host_launches: int = 0
+    osteal_p: float = 0.0
+    osteal_p_samples: int = 0
+    pad1: int = 0
 
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,

@@ -108,6 +108,13 @@ struct alignas(128) RunCtl {
     unsigned int mb, mb_next;
     unsigned int wakes[kMaxW];
     unsigned long long bar_ep;
+    // NEXT-3 online estimate of p (Eq. 4; "p ... can be estimated during previous iterations"): unit
+    // 0's history by iteration & 3 (control start time, advance window, frontier edges, owners, tail flag);
+    // every unit reads unit 0's history and updates its own estimate identically
+    unsigned long long h_tctl[4], h_adv0[4], h_adv1[4], h_edges[4];
+    unsigned int h_m[4], h_tail[4];
+    double os_p;
+    unsigned int os_p_n, pad_p;
 };
 
 // Decoupled look-back slot of the filter scan (one per partition per fragment, unit-local).
@@ -215,7 +222,8 @@ struct DevCtx {
     unsigned int num_vertices;  // |V|
     int fsteal, osteal;         // fsteal: 0 off, 1 steal queue, 2 planned (Eq. 1 / Alg. 1)
     double remote_cost;         // planned FSteal: cost of a remote edge relative to a local one
-    double os_p;                // OSteal cost model (osteal = 2): p of Eq. (4) in edges
+    double os_p;                // OSteal cost model (osteal = 2): p of Eq. (4) in edges (initial value when online)
+    int os_p_online;            // estimate p online from unit 0's iteration history (osteal_sync_edges == 0)
     unsigned long long t1, t2, os_thresh, os_epw;
     unsigned int max_iter;
     int pr_iters;

@@ -189,6 +189,14 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     // device-resident multi-unit loop: every unit is a member at the start (bar_ep and wakes[] stay
     // monotone across runs: the pads keep their last values)
     rc->mb = rc->mb_next = (unsigned)c.n_units;
+    rc->os_p = 0.0;
+    rc->os_p_n = 0;
+    for (int i = 0; i < 4; i++) {
+        rc->h_tctl[i] = rc->h_adv1[i] = rc->h_edges[i] = 0;
+        rc->h_adv0[i] = ~0ull;
+        rc->h_m[i] = 1;
+        rc->h_tail[i] = 1;  // no measurement from iterations that did not run
+    }
     if (c.pad[w0]) {
         c.pad[w0][kPadArr] = 0;
         c.pad[w0][kPadLastIt] = 0;
@@ -803,6 +811,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         if (use_h) cudaGraphSetConditional(h, 0);
         return;
     }
+    const unsigned long long t_ctl = globaltimer();
     const unsigned k = rc->iter;
     unsigned long long active = 0, total_edges = 0, l[kMaxW];
     unsigned err = 0;
@@ -877,7 +886,32 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
                 // NEXT-3: Alg. 2 with Eq. (4) on this iteration's per-fragment active edges
                 unsigned long long lf[kMaxW];
                 for (int f = 0; f < c.P; f++) lf[f] = vload(&c.f[f].ctl->qedges);
-                mp = (unsigned)osteal_choose(lf, c.P, c.remote_cost, c.os_p, nullptr);
+                double p = c.os_p;
+                if (c.os_p_online) {
+                    // p from unit 0's iteration k-2 (complete, and on one clock): its period (control to next
+                    // control) minus its advance window is the per-iteration synchronisation time S; the
+                    // advance processed e edges over m workers in A, i.e. tau = A*m/e per edge; Eq. 4's
+                    // T_hat = p*m gives p = S/(m*tau) edges. Halved-weight running average; iterations
+                    // touching the tail engine are skipped (their period holds many engine iterations).
+                    const RunCtl* r0 = c.rctl[0];
+                    if (k >= 2) {
+                        const unsigned a = (k - 2) & 3u, b2 = (k - 1) & 3u;
+                        const unsigned long long ta = vload(&r0->h_tctl[a]), tb = vload(&r0->h_tctl[b2]);
+                        const unsigned long long a0 = vload(&r0->h_adv0[a]), a1 = vload(&r0->h_adv1[a]);
+                        const unsigned long long e = vload(&r0->h_edges[a]);
+                        const unsigned m2 = vload(&r0->h_m[a]);
+                        const bool clean = !vload(&r0->h_tail[a]) && !vload(&r0->h_tail[b2]);
+                        if (clean && a1 > a0 && a1 - a0 > 2000ull && tb > ta && tb - ta > a1 - a0 && m2 >= 1 &&
+                            e >= 64ull * m2) {
+                            const double A = (double)(a1 - a0), S = (double)(tb - ta) - A;
+                            const double pk = S * (double)e / (A * (double)m2 * (double)m2);
+                            rc->os_p = rc->os_p_n ? 0.5 * rc->os_p + 0.5 * pk : pk;
+                            rc->os_p_n = rc->os_p_n + 1;
+                        }
+                    }
+                    if (rc->os_p_n) p = rc->os_p;
+                }
+                mp = (unsigned)osteal_choose(lf, c.P, c.remote_cost, p, nullptr);
             } else if (active < c.os_thresh) {
                 mp = 1;
                 if (c.os_epw) {
@@ -1023,6 +1057,15 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             rc->blocked_iters = rc->blocked_iters + 1;
             rc->tail = 0;
         }
+    }
+    if (c.osteal == 2 && c.os_p_online && !done) {
+        const unsigned hs = k & 3u;
+        rc->h_tctl[hs] = t_ctl;
+        rc->h_edges[hs] = total_edges;
+        rc->h_m[hs] = m;
+        rc->h_tail[hs] = rc->tail;
+        rc->h_adv0[hs] = ~0ull;
+        rc->h_adv1[hs] = 0;
     }
     rc->bodies = rc->bodies + 1;
     rc->skip_filter = 0;
@@ -1801,6 +1844,10 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         // (thread 0 holds the per-chunk counts; in a masked WCC pass every warp's lane 0 holds a share)
         if (e_own) atomicAdd((unsigned long long*)&r->edges_own[w], e_own);
         if (e_stolen) atomicAdd((unsigned long long*)&r->edges_stolen[w], e_stolen);
+    }
+    if (c.os_p_online && c.osteal == 2 && threadIdx.x == 0) {  // NEXT-3 online p: this unit's advance window
+        atomicMin(&rc->h_adv0[k & 3u], t0);
+        atomicMax(&rc->h_adv1[k & 3u], globaltimer());
     }
 }
 

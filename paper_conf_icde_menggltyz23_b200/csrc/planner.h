@@ -57,7 +57,7 @@ GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double
     return z;
 }
 
-// OSteal cost model (§IV-A/B, Eq. (4), Alg. 2).
+// OSteal cost model (§IV-A/B, Eq. (4), p estimated online P:172, Alg. 2).
 // For a cluster size m the reduction tree on a uniform fabric keeps workers R(m) = {0..m-1} (DESIGN.md
 // reading #13); the revised Eq. (1) lets only R(m) process (x_ij = 0 for j outside R(m)): an evicted
 // fragment's edges are all processed remotely at cost b, a survivor keeps its own at cost 1 and trades

@@ -451,6 +451,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.remote_cost = c->cfg.fsteal_remote_cost > 0.0 ? c->cfg.fsteal_remote_cost : 1.0;
     d.osteal = c->cfg.osteal;
     d.os_p = c->cfg.osteal_sync_edges > 0.0 ? c->cfg.osteal_sync_edges : 500000.0;
+    d.os_p_online = c->cfg.osteal_sync_edges > 0.0 ? 0 : 1;  // 0 => estimated online (initial 500K)
     d.t1 = c->cfg.t1_min_max_edges;
     d.t2 = c->cfg.t2_min_spread_edges;
     d.os_thresh = c->cfg.osteal_active_threshold;
@@ -1908,6 +1909,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
         stats->final_owners = R.m;
         stats->osteal_iteration = R.osteal_iter;
         stats->pr_last_residual = R.pr_resid;
+        stats->osteal_p = R.os_p_n ? R.os_p : d.os_p;
+        stats->osteal_p_samples = R.os_p_n;
         stats->tail_iterations = R.tail_iters;
         stats->blocked_iterations = R.blocked_iters;
         stats->bodies = R.bodies;

@@ -319,8 +319,8 @@ def test_wcc_blocked_first_iteration(monkeypatch, P):
 @pytest.mark.parametrize("p", [1e-9, 2e4, 1e12])
 def test_osteal_cost_model(alg, p):
     """NEXT-3: OSteal by Alg. 2 / Eq. (4) (osteal='cost'): outputs unchanged for any p; p -> inf keeps one
-    owner, p -> 0 keeps all of them (z(m) is non-increasing in m). (p = 0 itself selects the default
-    500000, include/gum.h osteal_sync_edges.)"""
+    owner, p -> 0 keeps all of them (z(m) is non-increasing in m). (p = 0 itself selects the online estimate,
+    tests/test_gpu_units.py test_osteal_online_p.)"""
     g = inputs.rmat(13, 16, seed=33)
     s = inputs.pick_source(g, 33)
     _, st, _ = check(g, alg, s, num_gpus=4, part="random", seed=3, osteal="cost", osteal_sync_edges=p,

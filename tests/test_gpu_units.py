@@ -115,3 +115,17 @@ def test_units_repeated_runs_race_check(alg):
               osteal_edges_per_worker=30000)
         check(g, alg, s, csr=csr, ref=ref, num_gpus=5, split_units=True, tail_vertices=0, chunk_edges=64)
         check(gb, alg, 0, csr=csr_gb, ref=ref_gb, num_gpus=4, split_units=True, tail_vertices=32)
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
+@pytest.mark.parametrize("kw", [dict(num_gpus=4, split_units=True), dict(num_gpus=4), dict(num_gpus=3, split_units=True,
+                                                                                          part="random", seed=3)])
+def test_osteal_online_p(alg, kw):
+    """NEXT-3: p of Eq. (4) estimated during the run from previous iterations: osteal='cost' with
+    osteal_sync_edges=0 measures each iteration's synchronisation time against its advance time per edge;
+    outputs stay exact whatever owner sets it picks."""
+    g = inputs.grid(128, seed=9)
+    ref = oracle.run(alg, g, 0)
+    _, st, _ = check(g, alg, 0, ref=ref, osteal="cost", osteal_sync_edges=0.0, tail_vertices=0, **kw)
+    assert st.osteal_p_samples > 0
+    assert 0.0 < st.osteal_p < 1e12
