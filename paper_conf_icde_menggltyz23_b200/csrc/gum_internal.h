@@ -234,6 +234,7 @@ struct DevCtx {
     unsigned int nf_delta;      // SSSP near-far split increment (0 = plain BSP frontier, the paper's)
     unsigned int tail_enter;    // tail engine: enter when the frontier has <= tail_enter vertices (0 = off)
     unsigned int tail_exit;     // tail engine: hand back when the next frontier exceeds tail_exit vertices
+    unsigned int tail_local;    // tail engine: local relaxation rounds per CTA before each grid barrier
     unsigned int pb_shift;      // BFS propagation blocking: log2(block size); 0 = off
     unsigned int pb_nb;         // bins of fragment 0 (single-fragment only)
     unsigned int bfs_pull;      // direction-optimising BFS enabled (in-CSR built)

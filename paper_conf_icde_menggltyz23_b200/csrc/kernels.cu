@@ -1861,6 +1861,21 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
 // released (acq) before its value is read, so an improvement after the read re-activates it.
 constexpr int kTailThreads = 256;
 
+// Dedupe bit of a next list, set with release semantics (orders the preceding red.min on the state before
+// the bit) and released by a local relaxation round with acquire semantics (orders the state read after it):
+// if an improvement's OR finds the bit still set, the local round's AND comes later in the bit's coherence
+// order and its state read sees that improvement; if the OR comes later, it finds the bit clear and appends.
+__device__ __forceinline__ unsigned atom_or_release(unsigned* p, unsigned v) {
+    unsigned old;
+    asm volatile("atom.release.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ unsigned atom_and_acquire(unsigned* p, unsigned v) {
+    unsigned old;
+    asm volatile("atom.acquire.gpu.global.and.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
 __device__ __forceinline__ void tail_barrier(RunCtl* rc, unsigned nblocks, unsigned& gen) {
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -1922,7 +1937,9 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
                 if (ok && cand < vload(T.state + lu)) {
                     atomicMin(T.state + lu, cand);
                     // the next list of iteration `it` dedupes on bm (it even) / bm2 (it odd)
-                    const unsigned ob = atomicOr(((it & 1) ? T.bm2 : T.bm) + (lu >> 5), bit);
+                    unsigned* const dw = ((it & 1) ? T.bm2 : T.bm) + (lu >> 5);
+                    // (release ordering is only needed when local rounds take entries out of the list)
+                    const unsigned ob = c.tail_local ? atom_or_release(dw, bit) : atomicOr(dw, bit);
                     need = !(ob & bit);
                 }
             }
@@ -2018,7 +2035,9 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
                 }
                 if (ok && cand < vload(T.state + lu)) {
                     atomicMin(T.state + lu, cand);
-                    const unsigned ob = atomicOr(((it & 1) ? T.bm2 : T.bm) + (lu >> 5), bit);
+                    unsigned* const dw = ((it & 1) ? T.bm2 : T.bm) + (lu >> 5);
+                    // (release ordering is only needed when local rounds take entries out of the list)
+                    const unsigned ob = c.tail_local ? atom_or_release(dw, bit) : atomicOr(dw, bit);
                     need = !(ob & bit);
                 }
             }
@@ -2068,7 +2087,12 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         s_app_lim[threadIdx.x] = app_cap;
         s_app_e[threadIdx.x] = 0;
     }
-    __shared__ unsigned long long s_tn[kMaxW], s_te[kMaxW];
+    __shared__ unsigned long long s_tn[kMaxW], s_te[kMaxW], s_rep_e;
+    __shared__ unsigned s_app_lo;  // local relaxation rounds: buffered entries [0, s_app_lo) are already expanded
+    if (threadIdx.x == 0) {
+        s_rep_e = 0;
+        s_app_lo = 0;
+    }
     RunCtl* rc = c.rctl[w0];
     __shared__ unsigned s_hdr[4];  // gen, k0, nfT, fslot
     if (threadIdx.x == 0) {
@@ -2110,14 +2134,12 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         // go to the split list
         constexpr unsigned kTailG = TailGroup<MULTI>::G, kTailVPW = TailGroup<MULTI>::VPW;
         const unsigned sub = lane / kTailG, gl = lane % kTailG, src = sub * kTailG;
-        for (int f = 0; f < nfrag; f++) {
+        // one pass over list entries [lo, n) of `cur`, vertices spread over `nw` warps from warp `gwi`.
+        // local = entries of this CTA's own append buffer (a local relaxation round, see below): their
+        // next-list dedupe bits stay set (they are flushed to the next list as well)
+        auto pass = [&](int f, const unsigned* cur, unsigned lo, unsigned n, unsigned gwi, unsigned nw, bool local) {
             const FragPtrs& F = c.f[f];
-            const unsigned* cur = (it & 1) ? F.app : F.q_v;
-            const unsigned n = s_n[f];
-            n_all += n;
-            if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
-            if (gw == 0 && lane == 0) tail_v += n;
-            for (unsigned i0 = gw * kTailVPW; i0 < n; i0 += nwarps * kTailVPW) {  // warp-uniform trip count
+            for (unsigned i0 = lo + gwi * kTailVPW; i0 < n; i0 += nw * kTailVPW) {  // warp-uniform trip count
                 const unsigned i = i0 + sub;
                 const bool have = i < n;
                 const unsigned v = have ? cur[i] : 0u;
@@ -2127,10 +2149,14 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 unsigned slot = 0xFFFFFFFFu;
                 bool park = !have;
                 if (have && gl == 0) {
+                    if (local) atomicAdd(&s_rep_e, s1 - s0);  // (its edges leave the next list's count)
                     if (ALG != ALG_BFS) {
                         // release the cur list's dedupe bit (reused two iterations later); any
                         // improvement of v from now on appends it to the NEXT list (other parity)
-                        if (it > 0) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
+                        if (it > 0 && !local) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
+                        // a local round takes v out of the NEXT list: release its bit there first (acquire),
+                        // so an improvement after the state read below appends v again
+                        if (local) atom_and_acquire(((it & 1) ? F.bm2 : F.bm) + (v >> 5), ~(1u << (v & 31)));
                         sval = vload(F.state + v);
                         // v's far bit is only changed by v's own processing: read it with the state (one
                         // round trip) instead of after the near/far decision
@@ -2151,8 +2177,8 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                     if (!park) {
                         it_edges += s1 - s0;
                         e_done[f] += s1 - s0;
-                        if (it > 0) e_front[f] += s1 - s0;
-                        if (s1 - s0 > kTailSplit) {
+                        if (it > 0 || local) e_front[f] += s1 - s0;
+                        if (s1 - s0 > kTailSplit && !local) {
                             slot = atomicAdd(&rc->tsplit_cnt[it & 1], 1u);
                             if (slot < kTailSplitCap) split[slot] = TailSplit{(unsigned)f, v, sval, 0u, s0, s1};
                         }
@@ -2175,6 +2201,41 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                     a_sum += tail_expand<ALG, MULTI>(c, F, wv, w0s, w1s, k, it, ns);
                 }
             }
+        };
+        for (int f = 0; f < nfrag; f++) {
+            const FragPtrs& F = c.f[f];
+            const unsigned* cur = (it & 1) ? F.app : F.q_v;
+            const unsigned n = s_n[f];
+            n_all += n;
+            if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
+            if (gw == 0 && lane == 0) tail_v += n;
+            pass(f, cur, 0, n, gw, nwarps, false);
+        }
+        // local relaxation rounds (single fragment, min-algorithms): before the grid barrier the CTA expands
+        // the vertices it has just activated (its append buffer), up to c.tail_local rounds -- the frontier
+        // advances several hops per engine iteration. The entries stay in the buffer and reach the next list
+        // anyway (their dedupe bits stay set, so an improvement by another CTA after the local expansion is
+        // still expanded next iteration): same min-fixpoint, fewer grid barriers.
+        if (!MULTI && ALG != ALG_BFS && c.tail_local) {
+            unsigned done_lo = 0;
+            for (unsigned lr = 0; lr < c.tail_local; lr++) {
+                __syncthreads();
+                const unsigned nb = s_app_n[0] < s_app_lim[0] ? s_app_n[0] : s_app_lim[0];
+                if (nb <= done_lo) break;  // CTA-uniform (read after the barrier)
+                if (threadIdx.x == 0) {
+                    tail_v += nb - done_lo;
+                    v_front[0] += nb - done_lo;
+                }
+                pass(0, s_app, done_lo, nb, threadIdx.x >> 5, kTailThreads / 32, true);
+                done_lo = nb;
+            }
+            __syncthreads();
+            // the expanded entries leave the buffer: only what the last round activated reaches the next list
+            if (threadIdx.x == 0) {
+                s_app_lo = done_lo;
+                s_app_e[0] -= s_rep_e;
+                s_rep_e = 0;
+            }
         }
         {
             // the CTA's buffered appends: one reservation per target fragment's next list, then a copy
@@ -2185,18 +2246,20 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         {
             if (threadIdx.x < (unsigned)nfrag) {
                 const unsigned f = threadIdx.x;
-                const unsigned na = s_app_n[f] < s_app_lim[f] ? s_app_n[f] : s_app_lim[f];
+                const unsigned lo = f == 0 ? s_app_lo : 0u;  // entries a local round already expanded
+                const unsigned nv = s_app_n[f] < s_app_lim[f] ? s_app_n[f] : s_app_lim[f];
+                const unsigned na = nv > lo ? nv - lo : 0u;
                 if (na) {
                     s_app_base[f] = atomicAdd(&c.f[f].ctl->tcnt[ns], na);
                     atomicAdd(&c.f[f].ctl->tedges[ns], s_app_e[f]);
                 }
-                s_app_na[f] = na;  // (the valid prefix to copy; s_app_n stays as read by every thread above)
+                s_app_na[f] = na;  // (the valid range to copy; s_app_n stays as read by every thread above)
             }
             __syncthreads();
             for (int f = 0; f < nfrag; f++) {
-                const unsigned na = s_app_na[f];
+                const unsigned na = s_app_na[f], lo = f == 0 ? s_app_lo : 0u;
                 unsigned* nxt = (it & 1) ? c.f[f].q_v : c.f[f].app;
-                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base[f] + i] = s_app[f * app_cap + i];
+                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base[f] + i] = s_app[f * app_cap + lo + i];
             }
             __syncthreads();
             if (threadIdx.x < (unsigned)kMaxW) {
@@ -2205,6 +2268,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                 s_app_e[threadIdx.x] = 0;
             }
         }
+            if (threadIdx.x == 0) s_app_lo = 0;
         }
         if (tr && k < (unsigned)kTraceMax) {
             it_edges = warp_sum_u64(it_edges);  // (group leaders hold the counts)
@@ -2295,7 +2359,8 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
             atomicAdd(&c.f[0].ctl->tail_edges, e_done[f]);
             if (e_front[f]) atomicAdd(&c.f[f].ctl->frontier_edges, e_front[f]);
         }
-        if (gw == 0 && lane == 0 && v_front[f]) atomicAdd(&c.f[f].ctl->frontier_vertices, v_front[f]);
+        // (thread 0 of warp 0 holds the list counts; thread 0 of every CTA its local rounds' entries)
+        if (threadIdx.x == 0 && v_front[f]) atomicAdd(&c.f[f].ctl->frontier_vertices, v_front[f]);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) a_sum += __shfl_xor_sync(0xffffffffu, a_sum, o);

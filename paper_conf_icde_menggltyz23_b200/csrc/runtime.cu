@@ -467,6 +467,11 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
                        ? c->cfg.tail_vertices
                        : 0u;
     d.tail_exit = 4u * c->cfg.tail_vertices;
+    // local relaxation rounds per CTA before each grid barrier of the tail engine (SSSP/WCC, one fragment):
+    // C3 8192^2 grid 252 -> 241 ms at 6 rounds; the tail is bound by the per-hop chain of dependent loads,
+    // not by the barriers (4096^2: 10186 -> 1281 engine iterations at 8 rounds, 103 -> 91 ms)
+    static const int env_tl = getenv("GUM_TAIL_LOCAL") ? atoi(getenv("GUM_TAIL_LOCAL")) : 8;
+    d.tail_local = (unsigned)std::max(0, env_tl);
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
     d.pb_nb = c->pb_nb;
     d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
