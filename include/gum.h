@@ -286,7 +286,8 @@ gum_status gum_result_device(gum_ctx* ctx, void* out_device, uint64_t out_bytes)
 gum_status gum_trace(const gum_ctx* ctx, gum_iter_trace* out, uint32_t max_records, uint32_t* n_records);
 
 /* Per-kernel device time of the last run, from CUDA events recorded on the launching stream around
- * every launch (only with GUM_CFG_PROFILE; single-device). */
+ * every launch (only with GUM_CFG_PROFILE; one launch unit per process: single device, or this rank's
+ * unit in multi-process mode). */
 typedef struct {
     double filter_ms, control_ms, advance_ms, finalize_ms, init_ms, tail_ms;
     uint32_t filter_launches, control_launches, advance_launches, finalize_launches, init_launches, tail_launches;
@@ -336,7 +337,7 @@ gum_status gum_mp_handshake(const gum_config* cfg, const gum_mp_config* mp);
  * gum_partition (each rank builds and keeps only its own fragment, then the fragments are
  * IPC-exchanged), gum_prepare, gum_run (each rank drives its own unit; stats->ms is this rank's device
  * time -- take the max over ranks), gum_result (every rank gathers the full result through the peer
- * mappings), gum_destroy. GUM_CFG_PROFILE is not supported (EUNSUP). */
+ * mappings), gum_destroy. GUM_CFG_PROFILE runs the host-driven loop and times this rank's kernels. */
 gum_status gum_create_mp(const gum_config* cfg, const gum_mp_config* mp, gum_ctx** out);
 
 /* Host helper of the OSteal cost model (NEXT-3): Alg. 2 over m = 1..n for per-fragment loads l[0..n)

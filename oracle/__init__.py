@@ -44,7 +44,7 @@ def _load():
                                     pd, pd]
     lib.oracle_delta_pagerank.restype = ctypes.c_int
     lib.oracle_delta_pagerank.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_double, ctypes.c_double,
-                                          pd, pd, ctypes.POINTER(ctypes.c_uint32)]
+                                          pd, pd, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint64)]
     lib.oracle_pagerank_pull.restype = ctypes.c_int
     lib.oracle_pagerank_pull.argtypes = [ctypes.c_uint32, ctypes.c_uint64, p32, p32, ctypes.c_int, ctypes.c_double,
                                          ctypes.c_int, pd, pd, ctypes.POINTER(ctypes.c_int)]
@@ -153,22 +153,24 @@ def dpr_epsilon(V, tolerance=1e-6, damping=0.85):
     return tolerance * (1.0 - damping) / float(V)
 
 
-def delta_pagerank(V, src, dst, damping=0.85, eps=None, tolerance=1e-6, return_state=False):
-    """NEXT-4 delta-PageRank (residual push in BSP rounds). Returns x, or (x, r, rounds)."""
+def delta_pagerank(V, src, dst, damping=0.85, eps=None, tolerance=1e-6, return_state=False, return_work=False):
+    """NEXT-4 delta-PageRank (residual push in BSP rounds). Returns x, or (x, r, rounds); return_work adds the
+    number of edges pushed along."""
     src, dst = _u32(src), _u32(dst)
     if eps is None:
         eps = dpr_epsilon(V, tolerance, damping)
     x = np.empty(int(V), dtype=np.float64)
     r = np.empty(int(V), dtype=np.float64)
     rounds = ctypes.c_uint32(0)
+    work = ctypes.c_uint64(0)
     rc = _load().oracle_delta_pagerank(int(V), int(src.shape[0]), _p(src, ctypes.c_uint32), _p(dst, ctypes.c_uint32),
                                        float(damping), float(eps), _p(x, ctypes.c_double), _p(r, ctypes.c_double),
-                                       ctypes.byref(rounds))
+                                       ctypes.byref(rounds), ctypes.byref(work))
     if rc != 0:
         raise ValueError(f"oracle_delta_pagerank rc={rc}")
     if return_state:
-        return x, r, rounds.value
-    return x
+        return (x, r, rounds.value, work.value) if return_work else (x, r, rounds.value)
+    return (x, work.value) if return_work else x
 
 
 def run(alg: str, g, source: int = 0, pr_iterations: int = 20, pr_damping: float = 0.85):

@@ -291,7 +291,7 @@ int oracle_pagerank_pull(uint32_t V, uint64_t E, const uint32_t* src, const uint
  * The identity x + (I - d P^T)^{-1} r = x* holds after every round, so 0 <= x* - x componentwise and
  * sum(x* - x) <= sum(r) / (1 - d) <= V * eps / (1 - d) at the end (pinned in tests/test_oracle.py).        */
 int oracle_delta_pagerank(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, double d, double eps,
-                          double* x, double* r, uint32_t* rounds_out) {
+                          double* x, double* r, uint32_t* rounds_out, uint64_t* work_out) {
     if (V == 0) return 0;
     uint64_t* row_ptr = (uint64_t*)calloc((size_t)V + 1, sizeof(uint64_t));
     uint32_t* adj = (uint32_t*)malloc(sizeof(uint32_t) * (size_t)(E ? E : 1));
@@ -310,6 +310,7 @@ int oracle_delta_pagerank(uint32_t V, uint64_t E, const uint32_t* src, const uin
         r[v] = (1.0 - d) / (double)V;
     }
     uint32_t rounds = 0;
+    uint64_t work = 0; /* edges pushed along (the work rate's numerator) */
     for (;;) {
         size_t nf = 0;
         for (uint32_t v = 0; v < V; v++)
@@ -326,9 +327,11 @@ int oracle_delta_pagerank(uint32_t V, uint64_t E, const uint32_t* src, const uin
         for (size_t i = 0; i < nf; i++) {
             uint32_t u = F[i];
             for (uint64_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) r[adj[e]] += push[u];
+            work += row_ptr[u + 1] - row_ptr[u];
         }
     }
     if (rounds_out) *rounds_out = rounds;
+    if (work_out) *work_out = work;
     free(row_ptr); free(adj); free(push); free(F);
     return 0;
 }

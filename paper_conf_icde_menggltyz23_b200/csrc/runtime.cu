@@ -1384,8 +1384,7 @@ gum_status gum_create_mp(const gum_config* cfg, const gum_mp_config* mp, gum_ctx
         for (int i = 0; i < kMaxW; i++) devs[i] = mp->device;
         c1.device_ids = devs;
         c1.flags &= ~GUM_CFG_SPLIT_UNITS;
-        if (cfg->flags & GUM_CFG_PROFILE) local = GUM_EUNSUP;
-        else local = gum_create(&c1, &c);
+        local = gum_create(&c1, &c);
     }
     // agree: every rank creates its context or none keeps one
     long long mine = local, all[kMaxW];
@@ -1760,7 +1759,8 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
     }
     const double D0 = (double)c->n_dangling / (double)c->V;
     const bool profile = (c->cfg.flags & GUM_CFG_PROFILE) != 0;
-    if (profile && c->n_units > 1) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single launch unit");
+    // (one process per GPU: each rank profiles its own unit's launches)
+    if (profile && c->n_units > 1 && !c->mp) return fail(c, GUM_EUNSUP, "GUM_CFG_PROFILE needs a single launch unit per process");
     const bool graph_mode = !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE));
     for (auto e : c->prof_ev) cudaEventDestroy(e);
     c->prof_ev.clear();

@@ -1,3 +1,4 @@
 O=gpurun_out/dbg1; mkdir -p $O
-timeout 1200 python -m pytest tests -m gpu -q -x -k "tail or near_far or units or grid or sssp" > $O/tail.log 2>&1; echo "tests rc=$?"; tail -2 $O/tail.log; grep -E "^E  " $O/tail.log | head
-for L in 0 8 16; do GUM_TAIL_LOCAL=$L timeout 900 python tools/kbench.py --config C3 --alg sssp --runs 3 --kw '{"sssp_delta": 4096}' > $O/c3_local$L.txt 2>&1; echo "local=$L"; cat $O/c3_local$L.txt | cut -c1-300; done
+timeout 900 python bench.py > $O/b_c2.log 2>&1; echo "c2 rc=$?"; tail -1 $O/b_c2.log | cut -c1-1500
+GUM_BENCH_DEVICE=0 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29511 bench.py --gpus 2 --config C1 --steps 3 --warmup 3 > $O/b_mp.log 2>&1; echo "mp rc=$?"; grep metric $O/b_mp.log | tail -1 | cut -c1-2500
+timeout 900 python bench.py --config C1 --alg dpr --steps 5 --warmup 3 > $O/b_dpr.log 2>&1; echo "dpr rc=$?"; tail -1 $O/b_dpr.log | cut -c1-1200
