@@ -12,7 +12,12 @@ NVFLAGS  := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC,-fopenmp,-O3 -Xptx
 GUM_SRCS := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 GUM_HDRS := $(wildcard $(PKG)/csrc/*.h) $(wildcard $(PKG)/csrc/*.cuh) include/gum.h
 
-all: inputs oracle gum
+all: inputs oracle gum linkbench
+
+linkbench: tools/linkbench/liblinkbench.so
+
+tools/linkbench/liblinkbench.so: tools/linkbench/linkbench.cu
+	$(NVCC) -O3 -std=c++17 $(ARCH) -Xcompiler -fPIC -shared -o $@ $<
 
 inputs: inputs/libgen.so
 oracle: oracle/liboracle.so
@@ -31,6 +36,6 @@ $(PKG)/libgum.so: $(GUM_SRCS) $(GUM_HDRS)
 $(shell mkdir -p build)
 
 clean:
-	rm -f inputs/libgen.so oracle/liboracle.so $(PKG)/libgum.so
+	rm -f inputs/libgen.so oracle/liboracle.so $(PKG)/libgum.so tools/linkbench/liblinkbench.so
 
-.PHONY: all inputs oracle gum clean
+.PHONY: all inputs oracle gum linkbench clean

@@ -170,6 +170,13 @@ typedef struct {
     /* delta-PageRank (GUM_DPR): target L1 tolerance; the residual threshold is dpr_tolerance * (1-d)/V
      * (0 => 1e-6). Damping is pr_damping. */
     double dpr_tolerance;
+    /* NEXT-3 copy-migration of evicted fragments' frontiers (P:238 Ex. 4 step 2: "the generated frontier
+     * queue will directly be on another GPU"; "migrating the residual frontiers from victims").
+     * 0 (default): an evicted fragment's queue, CSR and state stay in its GPU's memory and the new owner reads
+     * them remotely ("extended memory"). 1: the owner's filter generates the evicted fragment's queue in a
+     * foster buffer in the owner's own memory and the owner's advance reads it locally (state, bitmaps and
+     * CSR stay remote; the CSR can be replicated with hub_cache = 1, hub_degree = 0). BFS/SSSP/WCC/DPR. */
+    int osteal_migrate;
 } gum_config;
 
 /* Fills *cfg with the defaults: 1 worker, fsteal=1, osteal=1, t1=t2=0, osteal threshold 0 (off until
@@ -220,6 +227,8 @@ typedef struct {
     double osteal_p;
     uint32_t osteal_p_samples;
     uint32_t pad1;
+    /* NEXT-3 copy-migration: frontier-queue entries generated in a foster queue on an evicted fragment's owner */
+    uint64_t migrated_queue_entries;
 } gum_run_stats;
 
 /* Per-iteration trace record (GUM_CFG_TRACE). Times are %globaltimer ns of the advance phase:

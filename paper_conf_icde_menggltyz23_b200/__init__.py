@@ -61,7 +61,7 @@ class gum_config(ctypes.Structure):
                 ("alloc", ALLOC_FN),
                 ("free_fn", FREE_FN), ("alloc_user", ctypes.c_void_p), ("streams", ctypes.POINTER(ctypes.c_void_p)),
                 ("mirrors", ctypes.c_int), ("hub_cache", ctypes.c_int), ("hub_degree", ctypes.c_uint32),
-                ("pr_push", ctypes.c_int), ("dpr_tolerance", ctypes.c_double)]
+                ("pr_push", ctypes.c_int), ("dpr_tolerance", ctypes.c_double), ("osteal_migrate", ctypes.c_int)]
 
 
 EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p)
@@ -85,7 +85,8 @@ class gum_run_stats(ctypes.Structure):
                 ("pad0", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
                 ("tail_activations", ctypes.c_uint64), ("unit_barriers", ctypes.c_uint32 * MAX_WORKERS),
                 ("unit_last_iter", ctypes.c_uint32 * MAX_WORKERS), ("host_launches", ctypes.c_uint64),
-                ("osteal_p", ctypes.c_double), ("osteal_p_samples", ctypes.c_uint32), ("pad1", ctypes.c_uint32)]
+                ("osteal_p", ctypes.c_double), ("osteal_p_samples", ctypes.c_uint32), ("pad1", ctypes.c_uint32),
+                ("migrated_queue_entries", ctypes.c_uint64)]
 
 
 class gum_kernel_times(ctypes.Structure):
@@ -206,6 +207,7 @@ class RunStats:
     osteal_p: float = 0.0
     osteal_p_samples: int = 0
     pad1: int = 0
+    migrated_queue_entries: int = 0
 
 
 def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=0, osteal_threshold=0,
@@ -213,7 +215,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
                 trace=False, host_loop=False, profile=False, split_units=False, sssp_delta=0, tail_vertices=16384,
                 pb_block_log2=0, fsteal_remote_cost=1.0, bfs_direction_opt=False, force_mode=None,
                 use_torch_allocator=False, streams=None, osteal_sync_edges=0.0, mirrors=False, hub_cache=False,
-                hub_degree=0, pr_push=False, dpr_tolerance=1e-6):
+                hub_degree=0, pr_push=False, dpr_tolerance=1e-6, osteal_migrate=False):
     """Builds a gum_config (host only). Returns (cfg, keepalive): keepalive holds the ctypes objects the
     config points to and must live as long as the context."""
     lib = load_library()
@@ -246,6 +248,7 @@ def make_config(num_gpus=1, device_ids=None, fsteal=True, osteal=True, t1=0, t2=
     cfg.hub_degree = int(hub_degree)          # t4
     cfg.pr_push = int(bool(pr_push))          # PR advance: pull over source blocks (default) or push
     cfg.dpr_tolerance = float(dpr_tolerance)  # delta-PageRank: L1 tolerance (eps = tol * (1-d) / V)
+    cfg.osteal_migrate = int(bool(osteal_migrate))  # NEXT-3: evicted fragments' queues generated on the owner
     flags = 0
     if trace:
         flags |= CFG_TRACE

@@ -65,6 +65,10 @@ struct alignas(128) FragCtl {
     unsigned long long remote_filtered;  // NEXT-1 mirrors: cross-fragment updates absorbed locally
     unsigned long long hub_edges;        // NEXT-1 hub cache: non-local edges expanded from a local copy
     unsigned long long tail_edges, tail_vertices, tail_acts;  // work done inside the tail engine (stats)
+    unsigned long long migrated_q;       // NEXT-3 copy-migration: queue entries generated in a foster queue
+    unsigned int qown, pad_q;            // NEXT-3 copy-migration: the worker whose memory holds the current queue
+                                         // (set by the filter that generated it; the advance may run after an
+                                         // owner change, so it follows this, not the current owner)
 };
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
@@ -105,6 +109,7 @@ struct alignas(128) RunCtl {
     // next phase-A barrier (units >= mb_next leave it and park until woken); wakes[u] counts unit u's
     // wake-ups (computed identically by every member; the signal pad holds the same count); bar_ep is the
     // epoch of this unit's last device barrier (monotone across runs, equal on all members)
+    unsigned int fctl_cnt;    // fused control: filter CTAs that arrived in this iteration
     unsigned int mb, mb_next;
     unsigned int wakes[kMaxW];
     unsigned long long bar_ep;
@@ -187,6 +192,16 @@ struct FragPtrs {
     unsigned int* mmin;                 // SSSP/WCC: [V] upper bound of the owner's value (min sent/seen)
 };
 
+// A fragment's frontier queue (the filter's output, the advance's input): in the fragment's own memory, or --
+// NEXT-3 copy-migration (osteal_migrate) -- in a "foster" queue in the memory of the worker that owns the
+// fragment after OSteal evicted its GPU ("the generated frontier queue will directly be on another GPU").
+struct QPtrs {
+    unsigned* q_v;
+    unsigned long long* q_off;
+    long long* q_base;
+    unsigned* tile;
+};
+
 // NEXT-1 hub cache: worker w's local copy of fragment f's hub adjacency lists.
 struct HubPtrs {
     const unsigned long long* off;  // [V_f] col index of local vertex u's list in the copy, ~0 = not cached
@@ -257,7 +272,11 @@ struct DevCtx {
     // units through these pads (unit u's pad in unit u's memory); 0 = single unit or host-driven loop
     int units_dev;
     int n_units;
+    int alg;                    // the running algorithm (control_body)
+    int fuse_ctl;               // single unit, graph mode: the filter's last CTA runs the control decision
     unsigned long long* pad[kMaxW];
+    int migrate;                // NEXT-3 copy-migration: evicted fragments' queues live with their owner
+    QPtrs fq[kMaxW][kMaxW];     // [owner][fragment] foster queues (fragment > owner), in the owner's memory
     int hub_on;                 // NEXT-1 hub cache built for this algorithm
     HubPtrs hub[kMaxW][kMaxW];  // [worker][fragment] (fragment != worker)
 };

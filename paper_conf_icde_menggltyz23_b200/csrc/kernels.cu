@@ -58,6 +58,14 @@ __host__ __device__ __forceinline__ unsigned gcd_u32(unsigned a, unsigned b) {
     return a;
 }
 
+// The frontier queue of fragment f when worker o owns it: a foster queue in o's memory under NEXT-3
+// copy-migration, else the fragment's own.
+__device__ __forceinline__ QPtrs queue_of(const DevCtx& c, int f, unsigned o) {
+    if (c.migrate && o != (unsigned)f && c.fq[o][f].q_v) return c.fq[o][f];
+    const FragPtrs& F = c.f[f];
+    return QPtrs{F.q_v, F.q_off, F.q_base, F.tile};
+}
+
 // owner fragment of a global (relabelled) vertex id: <= 7 compares ("global to local id").
 __device__ __forceinline__ int frag_of(const DevCtx& c, unsigned v) {
     int f = 0;
@@ -137,6 +145,8 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->remote_filtered = 0;
         ct->hub_edges = 0;
         ct->tail_edges = ct->tail_vertices = ct->tail_acts = 0;
+        ct->qown = (unsigned)f;
+        ct->migrated_q = 0;
         if (sq) {
             ct->frontier_edges = F.sq_edges;
             ct->frontier_vertices = F.sq_len;
@@ -183,6 +193,7 @@ __global__ void k_init_run(const __grid_constant__ DevCtx c, int w0, double D0, 
     rc->bodies = 0;
     rc->tsplit_cnt[0] = rc->tsplit_cnt[1] = 0;
     rc->fbar_cnt = 0;
+    rc->fctl_cnt = 0;
     rc->pb = 0;
     rc->pull = 0;
     rc->nf_T = c.nf_delta ? (unsigned long long)c.nf_delta : 0xFFFFFFFFull;
@@ -275,12 +286,14 @@ constexpr int kLongCap = 512;
 constexpr unsigned kLongInline = 2;
 __shared__ unsigned s_long_n;
 __shared__ unsigned s_long_pos[kLongCap], s_long_t0[kLongCap], s_long_t1[kLongCap];
+__shared__ QPtrs s_qo;  // the filter CTA's output queue (queue_of the fragment under its current owner)
 
 __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, unsigned v, unsigned long long rp,
                                             unsigned long long deg, unsigned long long pos, unsigned long long off) {
-    F.q_v[pos] = v;
-    F.q_off[pos] = off;
-    F.q_base[pos] = (long long)rp - (long long)off;
+    (void)F;
+    s_qo.q_v[pos] = v;
+    s_qo.q_off[pos] = off;
+    s_qo.q_base[pos] = (long long)rp - (long long)off;
     // chunk table: every chunk whose first edge lies in [off, off+deg) starts at queue entry pos
     unsigned long long t = (off + chunk - 1) / chunk;
     const unsigned long long t1 = (off + deg + chunk - 1) / chunk;
@@ -293,7 +306,7 @@ __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, u
             return;
         }
     }
-    for (; t < t1; t++) F.tile[t] = (unsigned)pos;
+    for (; t < t1; t++) s_qo.tile[t] = (unsigned)pos;
 }
 
 // all threads of the CTA: write the deferred chunk-table runs (a warp per run, lanes over its chunks)
@@ -303,7 +316,7 @@ __device__ __forceinline__ void filter_flush_long(const FragPtrs& F) {
     if (n == 0) return;  // CTA-uniform (read after the barrier; the next append follows another barrier)
     for (unsigned e = threadIdx.x >> 5; e < n; e += kThreads / 32) {
         const unsigned pos = s_long_pos[e], t1 = s_long_t1[e];
-        for (unsigned t = s_long_t0[e] + (threadIdx.x & 31); t < t1; t += 32) F.tile[t] = pos;
+        for (unsigned t = s_long_t0[e] + (threadIdx.x & 31); t < t1; t += 32) s_qo.tile[t] = pos;
     }
     __syncthreads();
     if (threadIdx.x == 0) s_long_n = 0;
@@ -641,8 +654,28 @@ __device__ unsigned g_fcall;
 #endif
 // NF: SSSP near-far parking compiled in (its batched state loads and far-bit atomics cost registers the
 // other algorithms' filters do not need)
+__device__ __noinline__ void control_body(const DevCtx& c, const int alg, int w0, int nw, cudaGraphConditionalHandle h,
+                                          int use_h);
+
+// fuse_ctl (single launch unit, graph mode): every CTA of the filter grid arrives on a counter once it is done;
+// the last one runs the iteration's control decision (control_body) -- one kernel launch less per iteration.
+__device__ __forceinline__ void filter_arrive(const DevCtx& c, int w0, int nw, cudaGraphConditionalHandle h, int use_h) {
+    __threadfence();  // every thread's queue / counter writes before the CTA's arrival
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        RunCtl* rc = c.rctl[w0];
+        const unsigned total = gridDim.x * gridDim.y;
+        if (atomicAdd(&rc->fctl_cnt, 1u) == total - 1) {
+            __threadfence();
+            rc->fctl_cnt = 0;
+            control_body(c, c.alg, w0, nw, h, use_h);
+        }
+    }
+}
+
 template <bool NF, bool DPR = false>
-__global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw) {
+__global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __grid_constant__ DevCtx c, int w0, int nw,
+                                                                      int fuse_ctl, cudaGraphConditionalHandle h, int use_h) {
     FT_MARK(0);
     // Prologue by thread 0 only, broadcast through shared memory: the run-control fields are a handful of
     // L2 lines that every CTA of every kernel reads, and per-warp loads of one address serialise in its
@@ -675,13 +708,17 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
             // BFS: activations of advance k-1 have depth k = the iteration counter before control runs
             p.depth = c.bfs_filter_depth ? vload(&rc->iter) : GUM_INF;
             p.b = atomicAdd(&rc->ticket[f], 1u);  // ticket order: predecessors are running
+            s_qo = queue_of(c, f, o);
         }
         s_pro = p;
         s_long_n = 0;
     }
     __syncthreads();
     FT_MARK(1);
-    if (!s_pro.go) return;
+    if (!s_pro.go) {
+        if (fuse_ctl) filter_arrive(c, w0, nw, h, use_h);
+        return;
+    }
     const bool sweep = s_pro.sweep != 0;
     const unsigned nfT = s_pro.nfT;
     const unsigned fslot = s_pro.fslot;
@@ -706,7 +743,10 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     // small lists: only as many CTAs as tiles take part (the others leave before the prefix exchange)
     const unsigned G = n_tiles < gridDim.x ? (n_tiles ? n_tiles : 1u) : gridDim.x;
     const unsigned b = s_pro.b;
-    if (b >= G) return;
+    if (b >= G) {
+        if (fuse_ctl) filter_arrive(c, w0, nw, h, use_h);
+        return;
+    }
     const unsigned t_lo = (unsigned)(((unsigned long long)n_tiles * b) / G);
     const unsigned t_hi = (unsigned)(((unsigned long long)n_tiles * (b + 1)) / G);
     // logical tile t (queue order) -> physical tile (t * stride) mod n_tiles, stride coprime to n_tiles:
@@ -750,8 +790,10 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     block_excl_scan(pre, s_warp, excl);  // excl = sum over all predecessors
     if (b == G - 1 && threadIdx.x == 0) {
         const unsigned long long tc = excl.cnt + agg.cnt, td = excl.deg + agg.deg;
-        F.q_off[tc] = td;
+        s_qo.q_off[tc] = td;
         ct->qlen = tc;
+        ct->qown = vload(&rc->owner[f]);
+        if (c.migrate && s_qo.q_v != F.q_v) ct->migrated_q += tc;
         ct->qedges = td;
         ct->ntiles = (td + chunk - 1) / chunk;
         ct->claim = 0;
@@ -794,15 +836,18 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     }
     if (nf) nf_flush(ct, fslot, nfa);
     FT_MARK(4);
+    if (fuse_ctl) filter_arrive(c, w0, nw, h, use_h);
 #ifdef GUM_FILTER_TIMING
     if (threadIdx.x == 0 && g_fcall == GUM_FILTER_TIMING) { g_ftime[blockIdx.x][5] = b; g_ftime[blockIdx.x][6] = G; g_ftime[blockIdx.x][7] = app_cnt; }
 #endif
 }
 
 // ------------------------------------------------------------------------------------------ control
-template <int ALG>
-__global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cudaGraphConditionalHandle h, int use_h) {
-    if (threadIdx.x != 0) return;
+// a5/a6/a7-gate: the control decision of one BSP iteration (1 thread). Runs as its own kernel (k_control),
+// or -- single launch unit in graph mode -- inside the filter's last CTA (k_filter, fuse_ctl): one launch
+// less per iteration. Not inlined: its planner arrays must not raise the filter's register count.
+__device__ __noinline__ void control_body(const DevCtx& c, const int alg, int w0, int nw, cudaGraphConditionalHandle h,
+                                          int use_h) {
     RunCtl* rc = c.rctl[w0];
 #ifdef GUM_FILTER_TIMING
     g_fcall++;
@@ -824,7 +869,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         active += q;
         total_edges += e;
         l[rc->owner[f]] += e;
-        if (ALG == ALG_PR && k > 0) {
+        if (alg == ALG_PR && k > 0) {
             D += vload(&ct->pr_dang[(k - 1) & 1]);
             R += vload(&ct->pr_resid[(k - 1) & 1]);
         }
@@ -833,7 +878,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
     // smallest parked distance + delta and sweep the far set in the next filter (this iteration's
     // advance has an empty queue).
     bool nf_bump = false;
-    if (ALG == ALG_SSSP && c.nf_delta) {
+    if (alg == ALG_SSSP && c.nf_delta) {
         unsigned long long far_total = 0;
         unsigned fmin = GUM_INF;
         const unsigned slot = rc->nf_sweeps & 1u;
@@ -856,7 +901,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         }
     }
     bool done;
-    if (ALG == ALG_PR) {
+    if (alg == ALG_PR) {
         if (k > 0) {
             rc->pr_D = D;
             rc->pr_resid = R;
@@ -994,10 +1039,10 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
             r->steal_ok = rc->steal_ok;
         }
         // BFS propagation blocking for dense iterations (single fragment)
-        rc->pb = (ALG == ALG_BFS && c.pb_shift && c.P == 1 && rc->next_dense) ? 1u : 0u;
+        rc->pb = (alg == ALG_BFS && c.pb_shift && c.P == 1 && rc->next_dense) ? 1u : 0u;
         // NEXT-4 direction-optimising BFS (Beamer's rule): go bottom-up when the frontier's out-edges m_f
         // exceed 1/14 of the edges not yet reached m_u; stay while the frontier holds >= V/24 vertices.
-        if (ALG == ALG_BFS && c.bfs_pull) {
+        if (alg == ALG_BFS && c.bfs_pull) {
             unsigned long long seen = 0;
             for (int f = 0; f < c.P; f++) seen += vload(&c.f[f].ctl->frontier_edges);
             const unsigned long long mu = c.total_edges > seen ? c.total_edges - seen : 0;
@@ -1012,7 +1057,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         // long tail: hand small frontiers to the cooperative tail engine (OSteal m'=1 engine)
         // (OSteal's m'=1 mode: worker 0 owns every fragment while the engine runs)
         rc->tail = 0;
-        if (ALG != ALG_PR && c.osteal && c.tail_enter && !nf_bump && active <= c.tail_enter &&
+        if (alg != ALG_PR && c.osteal && c.tail_enter && !nf_bump && active <= c.tail_enter &&
             total_edges <= 8ull * c.tail_enter) {
             rc->tail = 1;
             for (int f = 0; f < c.P; f++) {
@@ -1035,7 +1080,7 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
         }
         rc->iter = k + 1;
     }
-    if (ALG == ALG_WCC && !done) {
+    if (alg == ALG_WCC && !done) {
         // WCC on the blocked static queue: iteration 0 (every vertex active), and later iterations whose
         // frontier (kept as a bitmap by a dense filter) holds >= 1/2 of the graph's entries: one pass over
         // the destination-blocked queue with inactive sources masked keeps the label atomics L2-resident,
@@ -1116,6 +1161,12 @@ __global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cuda
     if (use_h) cudaGraphSetConditional(h, done ? 0u : 1u);
 }
 
+template <int ALG>
+__global__ void k_control(const __grid_constant__ DevCtx c, int w0, int nw, cudaGraphConditionalHandle h, int use_h) {
+    if (threadIdx.x != 0) return;
+    control_body(c, ALG, w0, nw, h, use_h);
+}
+
 // ------------------------------------------------------------------------------------------ advance
 template <int ALG>
 struct ValT {
@@ -1186,6 +1237,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     __shared__ unsigned char s_hub[(MULTI && NX) ? kTileMax : 1];
     __shared__ unsigned long long s_ntiles[kMaxW], s_qlen[kMaxW], s_qedges[kMaxW];
     __shared__ unsigned s_owner[kMaxW];
+    __shared__ QPtrs s_q[kMaxW];                    // per fragment: where its queue lives (NEXT-3 migration)
     __shared__ unsigned long long s_cnt[kMaxW][4];  // per fragment: edges, chunks, stolen edges, stolen chunks
 
     // Prologue: thread 0 reads the run-control header once per CTA (per-warp loads of these few shared
@@ -1218,6 +1270,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
             s_qedges[threadIdx.x] = vload(&ct->qedges);
         }
         s_owner[threadIdx.x] = vload(&rc->owner[threadIdx.x]);
+        s_q[threadIdx.x] = queue_of(c, threadIdx.x, vload(&ct->qown));  // where the filter put the queue
         s_cnt[threadIdx.x][0] = s_cnt[threadIdx.x][1] = s_cnt[threadIdx.x][2] = s_cnt[threadIdx.x][3] = 0;
     }
     __syncthreads();
@@ -1335,7 +1388,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         r.hc = MULTI && NX && ALG != ALG_PR && ALG != ALG_DPR && c.hub_on && f != w;
         const FragPtrs& F = c.f[f];
         const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
-        const unsigned* const tilep = sq ? F.sq_tile : F.tile;
+        const unsigned* const tilep = sq ? F.sq_tile : s_q[f].tile;
         const unsigned long long tb = t * CH, qe = s_qedges[f];
         r.tlen = (unsigned)((qe - tb) < CH ? (qe - tb) : CH);
         r.i0 = __ldg(tilep + t);
@@ -1350,11 +1403,11 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
         const bool sq = ALG == ALG_WCC && blk && F.sq_col != nullptr;
         const unsigned i = r.i0 + kk;
         const unsigned long long tb = r.t * CH;
-        off = __ldcs((sq ? F.sq_q_off : F.q_off) + i);
+        off = __ldcs((sq ? F.sq_q_off : s_q[r.f].q_off) + i);
         // PR's (and WCC iteration 0's) blocked queue stores edges contiguously in queue order:
         // col index == q_off + j
-        base = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(F.q_base + i)));
-        u = (ALG != ALG_BFS || r.hc) ? __ldcs((sq ? F.sq_q_v : F.q_v) + i) : 0u;
+        base = (unsigned)((long long)tb + ((ALG == ALG_PR || sq) ? 0ll : __ldcs(s_q[r.f].q_base + i)));
+        u = (ALG != ALG_BFS || r.hc) ? __ldcs((sq ? F.sq_q_v : s_q[r.f].q_v) + i) : 0u;
         hub = false;
         if (MULTI && r.hc && !sq) {
             // NEXT-1: a cached hub list is read from the local copy: col index of edge j of
@@ -2204,7 +2257,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         };
         for (int f = 0; f < nfrag; f++) {
             const FragPtrs& F = c.f[f];
-            const unsigned* cur = (it & 1) ? F.app : F.q_v;
+            const unsigned* cur = (it & 1) ? F.app : (it == 0 ? queue_of(c, f, vload(&F.ctl->qown)).q_v : F.q_v);
             const unsigned n = s_n[f];
             n_all += n;
             if (it > 0 && gw == 0 && lane == 0) v_front[f] += n;
@@ -2952,11 +3005,11 @@ static cudaError_t launch_kernel_t(int kind, const DevCtx& c, const LaunchCfg& L
     switch (kind) {
         case KER_FILTER:
             if (c.nf_delta)
-                k_filter<true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+                k_filter<true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw, c.fuse_ctl, h, use_h);
             else if (ALG == ALG_DPR)
-                k_filter<false, true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+                k_filter<false, true><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw, c.fuse_ctl, h, use_h);
             else
-                k_filter<false><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw);
+                k_filter<false><<<dim3(L.filter_grid, c.P), kThreads, 0, s>>>(c, L.w0, L.nw, c.fuse_ctl, h, use_h);
             break;
         case KER_CONTROL: k_control<ALG><<<1, 32, 0, s>>>(c, L.w0, L.nw, h, use_h); break;
         case KER_ADVANCE:
@@ -3043,6 +3096,7 @@ cudaError_t launch_phase(int alg, int phase, const DevCtx& c, const LaunchCfg& L
     for (int i = 0; i < n; i++) {
         if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
         if (kinds[i] == KER_PULL && !c.bfs_pull) continue;
+        if (kinds[i] == KER_CONTROL && c.fuse_ctl && alg != ALG_PR) continue;  // run by the filter's last CTA
         cudaError_t e = launch_kernel(alg, kinds[i], c, L, s, h, use_h);
         if (e != cudaSuccess) return e;
     }

@@ -148,6 +148,9 @@ struct gum_ctx {
     unsigned* s_col_g = nullptr;
     int hub_kind = 0;                      // hub cache built from: 0 none, 1 out-CSR (BFS/SSSP), 2 symmetric (WCC)
     HubBufs hub[kMaxW][kMaxW];             // [worker][fragment]
+    QPtrs fq[kMaxW][kMaxW] = {};           // NEXT-3 copy-migration: foster queues [owner][fragment > owner]
+    unsigned long long fq_tile_cap[kMaxW][kMaxW] = {};
+    unsigned long long fq_key = 0;         // edge counts the foster queues are sized for (same on every rank)
     std::vector<Alloc> hub_allocs;
     unsigned long long hub_entries = 0;    // cached list entries per worker copy set (stats / tests)
     unsigned long long n_dangling = 0;
@@ -281,6 +284,12 @@ void drop_partition(gum_ctx* c) {
     c->hub_entries = 0;
     for (auto& row : c->hub)
         for (auto& h : row) h = HubBufs{};
+    for (int i = 0; i < kMaxW; i++)
+        for (int j = 0; j < kMaxW; j++) {
+            c->fq[i][j] = QPtrs{};
+            c->fq_tile_cap[i][j] = 0;
+        }
+    c->fq_key = 0;
     c->s_rp_g = nullptr;
     c->s_col_g = nullptr;
     free_list(c, c->part_allocs);
@@ -418,6 +427,9 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         d.lb[f] = c->lb[f];
     }
     d.mirrors = (c->cfg.mirrors && c->P > 1 && c->fr[0].mbuf && alg != GUM_DPR) ? 1 : 0;
+    d.migrate = (c->cfg.osteal_migrate && c->P > 1 && alg != GUM_PR) ? 1 : 0;
+    for (int o = 0; o < c->P && d.migrate; o++)
+        for (int f = o + 1; f < c->P; f++) d.fq[o][f] = c->fq[o][f];
     if (alg == GUM_PR && c->pl_ready) {
         // one replica of x/outdeg per launch unit; worker w pulls from its unit's
         d.pl_B = c->pl_B;
@@ -443,6 +455,10 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.n_units = c->n_units;
     for (int u = 0; u < c->n_units; u++) d.pad[u] = c->pad[unit_w0(c, u)];
     d.units_dev = (c->n_units > 1 && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))) ? 1 : 0;
+    d.alg = alg;
+    // control fused into the filter's last CTA: measured no faster on C2 (1.589 vs 1.570 ms per run), opt-in
+    static const int env_fc = getenv("GUM_FUSE_CONTROL") ? atoi(getenv("GUM_FUSE_CONTROL")) : 0;
+    d.fuse_ctl = (env_fc && c->n_units == 1 && alg != GUM_PR && !(c->cfg.flags & (GUM_CFG_HOST_LOOP | GUM_CFG_PROFILE))) ? 1 : 0;
     for (int i = 0; i <= c->P; i++) d.bounds[i] = c->bounds[i];
     d.P = c->P;
     d.chunk = c->cfg.chunk_edges;
@@ -520,7 +536,7 @@ gum_status unit_barrier(gum_ctx* c) {
 
 // Multi-process: the device buffers of fragment f that peers map (everything a kernel may touch after
 // OSteal hands the fragment to another worker), plus the unit's run control, trace and signal pad.
-constexpr int kMpFields = 48;
+constexpr int kMpFields = 88;
 int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     FragBufs& F = c->fr[f];
     int n = 0;
@@ -532,6 +548,9 @@ int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     GUM_FLD(F.sq_col); GUM_FLD(F.sq_q_v); GUM_FLD(F.sq_q_off); GUM_FLD(F.sq_tile); GUM_FLD(F.in_row_ptr);
     GUM_FLD(F.in_col); GUM_FLD(c->lb[f]); GUM_FLD(c->rctl[f]); GUM_FLD(c->trace[f]); GUM_FLD(c->pad[f]);
     GUM_FLD(F.mbuf); GUM_FLD(F.pl_off); GUM_FLD(F.pl_col); GUM_FLD(F.pl_tx); GUM_FLD(F.pl_tb); GUM_FLD(c->cxg[f]);
+    for (int g = 0; g < kMaxW; g++) {  // worker f's foster queues (NEXT-3 copy-migration)
+        GUM_FLD(c->fq[f][g].q_v); GUM_FLD(c->fq[f][g].q_off); GUM_FLD(c->fq[f][g].q_base); GUM_FLD(c->fq[f][g].tile);
+    }
 #undef GUM_FLD
     return n;
 }
@@ -806,6 +825,44 @@ gum_status build_hub(gum_ctx* c, int alg) {
     return GUM_OK;
 }
 
+// NEXT-3 copy-migration (osteal_migrate): worker o keeps a foster queue for every fragment f > o (the only
+// fragments the survivors {0..m'-1} can inherit, owner(f) = f mod m'), in o's memory, so an evicted fragment's
+// frontier queue is generated directly on its new owner and its advance reads it locally. Sized like
+// the fragment's own queue (vertices, and chunks of the larger of the out / symmetric edge counts).
+gum_status build_foster(gum_ctx* c, bool* built) {
+    *built = false;
+    if (!c->cfg.osteal_migrate || c->P == 1) return GUM_OK;
+    // decided from global sizes only, so every rank of a multi-process run agrees (and publishes) together
+    unsigned long long key = 1;
+    for (int f = 0; f < c->P; f++) key = key * 1000003ull + std::max(c->fr[f].E, c->fr[f].sE);
+    if (key == c->fq_key) return GUM_OK;
+    c->fq_key = key;
+    *built = true;
+    for (int o = 0; o < c->P; o++) {
+        if (!frag_local(c, o)) continue;  // (multi-process: every rank builds its own, peers map them)
+        for (int f = o + 1; f < c->P; f++) {
+            const FragBufs& F = c->fr[f];
+            const unsigned long long need_t = std::max(F.E, F.sE) / c->cfg.chunk_edges + 2;
+            QPtrs& Q = c->fq[o][f];
+            const int dev = c->dev[o];
+            const size_t Vn = std::max<size_t>(F.V, 1);
+            if (!Q.q_v) {
+                Q.q_v = (unsigned*)dalloc(c, dev, Vn * 4, c->part_allocs);
+                Q.q_off = (unsigned long long*)dalloc(c, dev, (Vn + 1) * 8, c->part_allocs);
+                Q.q_base = (long long*)dalloc(c, dev, Vn * 8, c->part_allocs);
+                if (!Q.q_v || !Q.q_off || !Q.q_base) return fail(c, GUM_ENOMEM, "foster queue alloc failed (%d, %d)", o, f);
+            }
+            if (c->fq_tile_cap[o][f] < need_t) {
+                Q.tile = (unsigned*)dalloc(c, dev, need_t * 4, c->part_allocs);
+                if (!Q.tile) return fail(c, GUM_ENOMEM, "foster chunk table alloc failed (%d, %d)", o, f);
+                c->fq_tile_cap[o][f] = need_t;
+            }
+        }
+    }
+    drop_graphs(c);
+    return GUM_OK;
+}
+
 // kernels launch_phase issues for (alg, phase) under d/L (the skips of kernels.cu launch_phase)
 int count_phase(int alg, int phase, const DevCtx& d, const LaunchCfg& L) {
     int kinds[4];
@@ -815,6 +872,7 @@ int count_phase(int alg, int phase, const DevCtx& d, const LaunchCfg& L) {
         if (kinds[i] == KER_TAIL && L.tail_grid <= 0) continue;
         if (kinds[i] == KER_PULL && !d.bfs_pull) continue;
         if (kinds[i] == KER_APPLY && !d.pb_shift) continue;
+        if (kinds[i] == KER_CONTROL && d.fuse_ctl && alg != GUM_PR) continue;
         k++;
     }
     return k;
@@ -1335,6 +1393,7 @@ static unsigned long long config_hash(const gum_config* cfg) {
     GUM_HC(pr_damping); GUM_HC(max_iterations); GUM_HC(flags); GUM_HC(sssp_delta); GUM_HC(tail_vertices);
     GUM_HC(pb_block_log2); GUM_HC(fsteal_remote_cost); GUM_HC(bfs_direction_opt); GUM_HC(osteal_sync_edges);
     GUM_HC(mirrors); GUM_HC(hub_cache); GUM_HC(hub_degree); GUM_HC(pr_push); GUM_HC(dpr_tolerance);
+    GUM_HC(osteal_migrate);
 #undef GUM_HC
     return h;
 }
@@ -1728,6 +1787,11 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
         if (st == GUM_OK) st = build_in(c);
     }
     if (st == GUM_OK) st = build_hub(c, alg);  // worker-local copies: nothing to publish
+    if (st == GUM_OK && alg != GUM_PR) {
+        bool fb = false;
+        st = build_foster(c, &fb);
+        built = built || fb;
+    }
     if (c->mp && built) st = mp_publish(c, st);
     return st;
 }
@@ -1963,6 +2027,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->tail_edges += fc.tail_edges;
             stats->tail_vertices += fc.tail_vertices;
             stats->tail_activations += fc.tail_acts;
+            stats->migrated_queue_entries += fc.migrated_q;
             if (getenv("GUM_DEBUG"))
                 fprintf(stderr, "[gum] frag %d: V=%u E=%llu qlen=%llu edges_done=%llu frontier_edges=%llu frontier_vertices=%llu app_cnt=%u tcnt=%u,%u,%u\n",
                         f, c->fr[f].V, (unsigned long long)(alg == GUM_WCC ? c->fr[f].sE : c->fr[f].E), fc.qlen,

@@ -1,10 +1,10 @@
 """Process-group plumbing for the multi-process mode (include/gum.h gum_create_mp).
 
 One process per GPU (the paper's one worker per GPU): torch.distributed is used only on the host
-to all-gather small byte blobs -- the configuration handshake, the CUDA IPC handles of every rank's
-fragment buffers, and once per launch batch the ranks' convergence flags. The data
-path (remote atomics, frontier steals, the per-phase barrier) is one-sided device code in libgum.so and
-never touches the process group.
+to all-gather small byte blobs -- the configuration handshake and the CUDA IPC handles of every rank's
+fragment buffers (and, only in the host-driven loop, the ranks' convergence flags). The data path (remote
+atomics, frontier steals, the device barriers of the per-rank CUDA-graph loop, OSteal parking and wake-up)
+is one-sided device code in libgum.so and never touches the process group.
 """
 from __future__ import annotations
 

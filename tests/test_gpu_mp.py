@@ -63,6 +63,17 @@ def test_mp_parity(world, part, kw):
         assert any(r["bfs"]["remote"] > 0 for r in res)
 
 
+def test_mp_copy_migration():
+    """NEXT-3 copy-migration across processes: the owner's foster queues are IPC-mapped for thieves."""
+    kw = dict(osteal_migrate=True, tail_vertices=0, osteal_threshold=1 << 30, osteal_edges_per_worker=20000,
+              chunk_edges=64)
+    res = mp_harness.run("tests.test_gpu_mp", "case_parity", world=3, args=(12, "random", kw), timeout=600,
+                         hide_gpu=False)
+    for r in res:
+        for alg, d in r.items():
+            assert d["ok"] and d["conserved"], (alg, d)
+
+
 def test_mp_forced_stealing_and_osteal():
     """FSteal with 32-edge chunks and no gating, and OSteal shrinking to one owner from the start."""
     kw = dict(chunk_edges=32, osteal_threshold=1 << 40, osteal_edges_per_worker=0)

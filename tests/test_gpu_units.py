@@ -129,3 +129,22 @@ def test_osteal_online_p(alg, kw):
     _, st, _ = check(g, alg, 0, ref=ref, osteal="cost", osteal_sync_edges=0.0, tail_vertices=0, **kw)
     assert st.osteal_p_samples > 0
     assert 0.0 < st.osteal_p < 1e12
+
+
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "wcc"])
+@pytest.mark.parametrize("kw", [dict(num_gpus=4, split_units=True), dict(num_gpus=4), dict(num_gpus=8, part="random",
+                                                                                         seed=5, split_units=True)])
+def test_copy_migration_of_evicted_frontiers(alg, kw):
+    """NEXT-3 copy-migration (osteal_migrate=1): once OSteal evicts a GPU, its fragment's frontier
+    queue is generated in a foster buffer on the new owner and expanded from there; results stay exact and the
+    counters show the migrated queue entries (with and without the tail engine, with stealing)."""
+    g = inputs.rmat(12, 16, seed=71, scramble=False)
+    s = inputs.pick_source(g, 71)
+    ref = oracle.run(alg, g, s)
+    csr = csr_of(g)
+    for extra in (dict(tail_vertices=0, osteal_threshold=1 << 30, osteal_edges_per_worker=40000),
+                  dict(tail_vertices=0, osteal="cost", osteal_sync_edges=0.0, chunk_edges=64),
+                  dict(tail_vertices=64, osteal_threshold=1 << 30, osteal_edges_per_worker=40000)):
+        _, st, _ = check(g, alg, s, csr=csr, ref=ref, osteal_migrate=True, **extra, **kw)
+        if "osteal_threshold" in extra and st.final_owners < kw["num_gpus"]:
+            assert st.migrated_queue_entries > 0, st

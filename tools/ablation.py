@@ -16,6 +16,14 @@ the workers are GPUs), updates absorbed by the mirrors, PR mirror bytes pulled p
 from a local hub copy. Outputs must be identical (PR: within the parity tolerance).
 
   python tools/ablation.py --next1 --scale 20 --workers 8
+
+NEXT-2 / Table IV: FSteal off vs the steal queue ("peek-and-grab") vs the planned
+estimate-and-reassign FSteal (Eq. (1) + Alg. 1), and OSteal off vs the cost model (Alg. 2 / Eq. (4) with online
+p), on 8 virtual workers: run time, time saved against "off", and the overhead -- the extra time of the
+control kernel (gating, planning, owner decisions; CUDA events per launch in a profile pass) -- with the
+paper's ratio saved / overhead.
+
+  python tools/ablation.py --table4 --scale 22 --grid 2048 --workers 8
 """
 import argparse
 import json
@@ -153,6 +161,71 @@ def next1(args):
     return res
 
 
+def profile_ms(csr, alg, src, reps=3, **kw):
+    """Per-kernel device time per run (profile pass: host loop, CUDA events around every launch)."""
+    rp, col, w = csr
+    with gum.Context(profile=True, **kw) as ctx:
+        ctx.load_csr(rp, col, w if alg == "sssp" else None)
+        ctx.partition("seg")
+        ctx.run(alg, src)
+        acc = {}
+        for _ in range(reps):
+            ctx.run(alg, src)
+            for k, v in ctx.profile().items():
+                if k.endswith("_ms"):
+                    acc[k] = acc.get(k, 0.0) + v / reps
+    return acc
+
+
+def table4(args):
+    res = {}
+    g = inputs.rmat(args.scale, 16, seed=9, scramble=False, weighted=False)
+    src = inputs.pick_source(g, 9)
+    csr = gum.build_csr(g.num_vertices, g.src, g.dst)
+    modes = (("off", dict(fsteal=False)), ("queue", dict(fsteal=True)), ("planned", dict(fsteal="planned")))
+    fs, outs = {}, []
+    for name, kw in modes:
+        st, tr, out = run(csr, "bfs", src, num_gpus=args.workers, chunk_edges=args.chunk, **kw)
+        rows = spread_stats(tr, args.workers)
+        big = [r for r in rows if r["frontier_edges"] >= 0.05 * max(x["frontier_edges"] for x in rows)]
+        prof = profile_ms(csr, "bfs", src, num_gpus=args.workers, chunk_edges=args.chunk, **kw)
+        fs[name] = dict(run_ms=round(st.ms, 4), advance_us_total=round(sum(r["advance_us"] for r in rows), 1),
+                        max_spread_big_iters=max((r["spread"] or 1) for r in big),
+                        starvation_us_total=round(sum(r["starvation_us"] for r in rows), 1),
+                        chunks_stolen=st.chunks_stolen, edges_stolen=st.edges_stolen,
+                        control_ms=round(prof.get("control_ms", 0.0), 4), advance_ms=round(prof.get("advance_ms", 0.0), 4))
+        outs.append(out)
+    for name in ("queue", "planned"):
+        saved = fs["off"]["run_ms"] - fs[name]["run_ms"]
+        over = max(fs[name]["control_ms"] - fs["off"]["control_ms"], 0.0)
+        fs[name].update(saved_ms=round(saved, 4), overhead_ms=round(over, 4),
+                        ratio=round(saved / over, 1) if over > 0 else None)
+    fs["identical_outputs"] = all(np.array_equal(o, outs[0]) for o in outs)
+    fs["workload"] = (f"BFS RMAT-{args.scale} EF16 unscrambled (hubs at low ids: a statically skewed seg partition), "
+                      f"{args.workers} virtual workers on 1 B200, chunk {args.chunk}")
+    res["fsteal"] = fs
+    gg = inputs.grid(args.grid, seed=3)
+    gcsr = gum.build_csr(gg.num_vertices, gg.src, gg.dst, gg.w)
+    os_, outs = {}, []
+    for name, kw in (("off", dict(osteal=False)), ("cost", dict(osteal="cost", osteal_sync_edges=0.0))):
+        st, tr, out = run(gcsr, "sssp", 0, reps=2, num_gpus=args.workers, sssp_delta=args.delta, tail_vertices=0, **kw)
+        prof = profile_ms(gcsr, "sssp", 0, reps=1, num_gpus=args.workers, sssp_delta=args.delta, tail_vertices=0, **kw)
+        os_[name] = dict(run_ms=round(st.ms, 3), iterations=st.iterations, final_owners=st.final_owners,
+                         osteal_iteration=st.osteal_iteration, osteal_p=st.osteal_p, p_samples=st.osteal_p_samples,
+                         control_ms=round(prof.get("control_ms", 0.0), 3), advance_ms=round(prof.get("advance_ms", 0.0), 3))
+        outs.append(out)
+    saved = os_["off"]["run_ms"] - os_["cost"]["run_ms"]
+    over = max(os_["cost"]["control_ms"] - os_["off"]["control_ms"], 0.0)
+    os_["cost"].update(saved_ms=round(saved, 3), overhead_ms=round(over, 3), ratio=round(saved / over, 1) if over > 0 else None)
+    os_["identical_outputs"] = bool(np.array_equal(outs[0], outs[1]))
+    os_["workload"] = (f"SSSP {args.grid}x{args.grid} grid, near-far delta {args.delta}, {args.workers} virtual workers on "
+                       f"1 B200, tail engine off (OSteal's owner shrink alone). On one GPU the evicted workers' CTAs "
+                       f"simply go idle: the sync cost OSteal removes across GPUs (barriers, launches per GPU) does "
+                       f"not exist here, so 'saved' is not the multi-GPU effect")
+    res["osteal"] = os_
+    return res
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--fsteal", action="store_true")
@@ -167,6 +240,7 @@ def main():
     ap.add_argument("--next1", action="store_true")
     ap.add_argument("--tail", type=int, default=None, help="tail engine threshold (default: the library's)")
     ap.add_argument("--hub-degree", type=int, default=64)
+    ap.add_argument("--table4", action="store_true")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     global TAIL
@@ -197,6 +271,19 @@ def main():
                           f"absorbed {r['absorbed_by_mirror']:>12d}  flush {r['mirror_flush_bytes']:>12d} B  "
                           f"hub-copy edges {r['stolen_edges_from_hub_copy']}")
             print(f"{alg:5s} identical outputs: {rows['identical_outputs']}")
+    if args.table4:
+        out["table4"] = table4(args)
+        t = out["table4"]
+        for k in ("off", "queue", "planned"):
+            r = t["fsteal"][k]
+            print(f"FSteal {k:8s} {r['run_ms']:8.3f} ms  spread {r['max_spread_big_iters']}  starvation "
+                  f"{r['starvation_us_total']} us  control {r['control_ms']} ms  saved {r.get('saved_ms')}  "
+                  f"overhead {r.get('overhead_ms')}  ratio {r.get('ratio')}")
+        for k in ("off", "cost"):
+            r = t["osteal"][k]
+            print(f"OSteal {k:5s} {r['run_ms']:8.3f} ms  owners {r['final_owners']}  control {r['control_ms']} ms  "
+                  f"p {r['osteal_p']:.0f} ({r['p_samples']})  saved {r.get('saved_ms')}  overhead {r.get('overhead_ms')}  "
+                  f"ratio {r.get('ratio')}")
     if args.out:
         json.dump(out, open(args.out, "w"), indent=1)
 
