@@ -122,7 +122,7 @@ def osteal(args):
     res["workload"] = (f"SSSP on a {args.grid}x{args.grid} grid (w in [1,255]), source 0, {args.workers} "
                        f"{'split-unit' if args.split else 'virtual'} workers on 1 B200, OSteal threshold {thr} "
                        f"active vertices; near-far delta {args.delta}; OSteal on includes the m'=1 tail engine "
-                       f"(single launch unit only)")
+                       f"(on unit 0 across every fragment; with --split the other units park in their graphs)")
     return res
 
 

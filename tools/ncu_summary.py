@@ -25,17 +25,27 @@ for r in rows[2:]:
 src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=sass"], capture_output=True,
                      text=True).stdout
 rows = list(csv.reader(io.StringIO(src)))
-if len(rows) > 2:
-    h = rows[1]
-    data = rows[2:]
+col = "Warp Stall Sampling (All Samples)"
+hi = next((i for i, r in enumerate(rows) if col in r), None)  # (the header row; one per kernel in the report)
+
+
+def num(x):
+    try:
+        return float(x)
+    except ValueError:
+        return 0.0
+
+
+if hi is not None:
+    h = rows[hi]
+    data = [r for r in rows[hi + 1:] if len(r) == len(h) and col not in r]
     ix = {n: i for i, n in enumerate(h)}
-    col = "Warp Stall Sampling (All Samples)"
-    tot = sum(float(r[ix[col]] or 0) for r in data) or 1
+    tot = sum(num(r[ix[col]]) for r in data) or 1
     stalls = [n for n in h if n.startswith("stall_") and "Not Issued" not in n]
-    agg = sorted(((sum(float(r[ix[n]] or 0) for r in data) / tot * 100, n) for n in stalls), reverse=True)[:8]
+    agg = sorted(((sum(num(r[ix[n]]) for r in data) / tot * 100, n) for n in stalls), reverse=True)[:8]
     print("  stall reasons (% of samples):", ", ".join(f"{n[6:]} {v:.1f}" for v, n in agg))
     print("  top instructions:")
-    for r in sorted(data, key=lambda r: -float(r[ix[col]] or 0))[:int(sys.argv[2]) if len(sys.argv) > 2 else 12]:
-        smp = float(r[ix[col]] or 0)
-        br = sorted(((float(r[ix[n]] or 0), n[6:]) for n in stalls), reverse=True)[:2]
+    for r in sorted(data, key=lambda r: -num(r[ix[col]]))[:int(sys.argv[2]) if len(sys.argv) > 2 else 12]:
+        smp = num(r[ix[col]])
+        br = sorted(((num(r[ix[n]]), n[6:]) for n in stalls), reverse=True)[:2]
         print(f"    {smp / tot * 100:5.1f}%  {r[1][:58]:58s} {br}")

@@ -37,7 +37,7 @@ def check(config, n_sources=4, part=None):
     import paper_conf_icde_menggltyz23_b200 as gum
 
     alg = bench.DEFAULT_ALG[config]
-    part = part or ("degree" if alg == "bfs" else "seg")
+    part = part or ("degree" if alg in ("bfs", "pr") else "seg")  # bench.py's layouts
     t0 = time.perf_counter()
     g = inputs.make_config(config, weighted=(alg == "sssp"))
     sources, outdeg = bench.pick_sources(g, int(config[1]), n_sources)
