@@ -653,12 +653,12 @@ def main():
 
     # ---------------------------------------------------------------- end to end through the C ABI
     e2e = None
-    if not args.no_e2e and N == 1:
+    if not args.no_e2e:  # (N > 1 without torchrun: the single-process multi-device context)
         rp_t = torch.from_numpy(row_ptr.view(np.int64)).pin_memory()
         col_t = torch.from_numpy(col.view(np.int32)).pin_memory()
         w_t = torch.from_numpy(w.view(np.int32)).pin_memory() if w is not None else None
         out_t = torch.empty(g.num_vertices * (8 if alg in ("pr", "dpr") else 4), dtype=torch.uint8).pin_memory()
-        ectx = gum.Context(streams=[stream], use_torch_allocator=True, **ctx_kw)
+        ectx = gum.Context(streams=[stream] if N == 1 else None, use_torch_allocator=True, **ctx_kw)
         h2d = rp_t.numel() * 8 + col_t.numel() * 4 + (w_t.numel() * 4 if w_t is not None else 0)
         d2h = out_t.numel()
         K2 = max(3, min(args.steps, 10))

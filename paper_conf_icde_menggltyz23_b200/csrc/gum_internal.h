@@ -57,6 +57,7 @@ struct alignas(128) FragCtl {
     unsigned long long activations;
     unsigned long long frontier_vertices; // sum over iterations of qlen
     unsigned long long far_cnt;        // SSSP near-far: vertices currently parked in the far set
+    unsigned int far_n[2];             // SSSP near-far: entries of the far lists (by sweep parity)
     unsigned int far_min[2];           // SSSP near-far: min distance of far vertices, by sweep parity
     unsigned int tcnt[3];              // tail engine: list counters (current / next / next-but-one)
     unsigned long long tedges[3];      // tail engine: out-edges of the listed vertices
@@ -156,6 +157,7 @@ struct FragPtrs {
     unsigned int* vis;                  // [ceil(V_f/32)] BFS visited bitmap (check-before-update)
     unsigned int* bm2;                  // [ceil(V_f/32)] tail engine: dedupe bits of odd-iteration lists
     unsigned int* far;                  // [ceil(V_f/32)] SSSP near-far: parked (far) vertices
+    unsigned int* farl;                 // [2][V_f] SSSP near-far: the far set as lists (bit set <=> listed)
     unsigned int* app;                  // [V_f] activation list (sparse next frontier)
     unsigned int* q_v;                  // [V_f] frontier queue (local ids, out-degree > 0)
     unsigned long long* q_off;          // [V_f + 1] exclusive prefix of out-degrees over the queue

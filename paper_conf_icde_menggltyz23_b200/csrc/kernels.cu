@@ -141,6 +141,7 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->frontier_vertices = 0;
         ct->far_cnt = 0;
         ct->far_min[0] = ct->far_min[1] = GUM_INF;
+        ct->far_n[0] = ct->far_n[1] = 0;
         ct->pull_checked = 0;
         ct->remote_filtered = 0;
         ct->hub_edges = 0;
@@ -287,6 +288,7 @@ constexpr unsigned kLongInline = 2;
 __shared__ unsigned s_long_n;
 __shared__ unsigned s_long_pos[kLongCap], s_long_t0[kLongCap], s_long_t1[kLongCap];
 __shared__ QPtrs s_qo;  // the filter CTA's output queue (queue_of the fragment under its current owner)
+__shared__ const unsigned* s_src;  // the filter CTA's sparse input: the activation list, or a far list (sweep)
 
 __device__ __forceinline__ void emit_vertex(const FragPtrs& F, unsigned chunk, unsigned v, unsigned long long rp,
                                             unsigned long long deg, unsigned long long pos, unsigned long long off) {
@@ -359,6 +361,8 @@ enum { FT_CLASSIFY = 0, FT_COUNT = 1, FT_EMIT = 2 };
 struct NfAcc {
     unsigned long long parked = 0, unparked = 0;
     unsigned min_dist = 0xFFFFFFFFu;
+    unsigned fslot = 0;       // far list receiving new / still-parked vertices (nf_sweeps & 1)
+    bool sweep_list = false;  // this filter sweeps the previous far list (its entries are all parked)
 };
 // Acceptance of a thread's 8 candidates (bit q of cand: vertex vs[q] has out-degree > 0) under the
 // near-far split, batched so that the 8 state loads and then the 8 far-bit atomics are each in flight
@@ -382,14 +386,28 @@ __device__ __forceinline__ unsigned filter_accept8(const FragPtrs& F, const unsi
 #pragma unroll
         for (int q = 0; q < 8; q++)
             ob[q] = ((park >> q) & 1u) ? atomicOr(F.far + (vs[q] >> 5), 1u << (vs[q] & 31)) : 0xFFFFFFFFu;
+        // the far set is also a list: a newly parked vertex is appended, and a sweep re-appends the entries
+        // of the previous list that stay parked (a far bit is set <=> the vertex is in the current list)
+        unsigned lst = 0;
 #pragma unroll
         for (int q = 0; q < 8; q++) {
             if (!((park >> q) & 1u)) continue;
-            if (!(ob[q] & (1u << (vs[q] & 31)))) acc.parked++;
+            const bool fresh = !(ob[q] & (1u << (vs[q] & 31)));
+            if (fresh) acc.parked++;
+            if (fresh || acc.sweep_list) lst |= 1u << q;
             acc.min_dist = st[q] < acc.min_dist ? st[q] : acc.min_dist;
         }
+        if (lst && F.farl) {
+            unsigned pos = atomicAdd(&F.ctl->far_n[acc.fslot], (unsigned)__popc(lst));
+            unsigned* fl = F.farl + (size_t)acc.fslot * F.V;
+#pragma unroll
+            for (int q = 0; q < 8; q++)
+                if ((lst >> q) & 1u) fl[pos++] = vs[q];
+        }
     }
-    if (MODE == FT_EMIT && ok) {
+    // with far lists a vertex leaves the far set only when a sweep takes it: an entry accepted in a normal
+    // iteration keeps its bit and is looked at again by the next sweep (one extra look, no duplicate entry)
+    if (MODE == FT_EMIT && ok && (acc.sweep_list || !F.farl)) {
         // accepted vertices leave the far set (their bit may be left from an earlier parking)
         unsigned fw[8], ob[8];
 #pragma unroll
@@ -436,7 +454,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
         unsigned word = 0;
         if (wi < nwords) {
             word = F.bm[wi];
-            if (sweep) word |= F.far[wi];
+            if (sweep) word |= F.far[wi];  // (sweep without a far list: the bitmap)
         }
         if (MODE == FT_EMIT) {
             __syncwarp();
@@ -516,7 +534,7 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
             items[j] = 0xFFFFFFFFu;
-            if ((unsigned)j < ipt && ibase + j < app_cnt) items[j] = F.app[ibase + j];
+            if ((unsigned)j < ipt && ibase + j < app_cnt) items[j] = s_src[ibase + j];
         }
 #pragma unroll
         for (int j = 0; j < kFilterAppPerThread; j++) {
@@ -701,9 +719,13 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
             const unsigned long long T = vload(&rc->nf_T);
             p.nfT = nf ? (unsigned)(T < 0xFFFFFFFFull ? T : 0xFFFFFFFFull) : GUM_INF;
             p.fslot = vload(&rc->nf_sweeps) & 1u;
-            // the advance that produced these activations either appended them (sparse) or only set bits
-            p.dense = p.sweep || vload(&rc->next_dense) != 0;
-            p.app_cnt = p.dense ? 0u : vload(&ct->app_cnt);
+            // the advance that produced these activations either appended them (sparse) or only set bits;
+            // a near-far sweep (the near frontier is empty) reads the previous far list, or scans the far
+            // bitmap when the list is not kept
+            const bool swl = p.sweep && F.farl;
+            p.dense = (p.sweep && !swl) || (!p.sweep && vload(&rc->next_dense) != 0);
+            p.app_cnt = swl ? vload(&ct->far_n[p.fslot ^ 1u]) : (p.dense ? 0u : vload(&ct->app_cnt));
+            s_src = swl ? F.farl + (size_t)(p.fslot ^ 1u) * F.V : F.app;
             p.epoch = vload(&rc->epoch);
             // BFS: activations of advance k-1 have depth k = the iteration counter before control runs
             p.depth = c.bfs_filter_depth ? vload(&rc->iter) : GUM_INF;
@@ -763,6 +785,8 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
     // ---- pass 1: aggregate of this CTA's tile range
     Pair mine{0, 0};
     NfAcc nfa;
+    nfa.fslot = fslot;
+    nfa.sweep_list = sweep && !dense;
     for (unsigned t = t_lo; t < t_hi; t++) {
         const Pair q = filter_tile<FT_CLASSIFY, DPR>(F, nfa, keep_fbm, depth, (unsigned)((unsigned long long)t * stride % n_tiles), dense, sweep, nf, nfT, nwords, app_cnt, ipt, chunk, 0, 0, dd);
         mine.cnt += q.cnt;
@@ -897,7 +921,10 @@ __device__ __noinline__ void control_body(const DevCtx& c, const int alg, int w0
             rc->nf_sweeps = rc->nf_sweeps + 1;
             // the next epoch's minimum slot starts empty (only the owner resets; others read `slot`)
             for (int f = 0; f < c.P; f++)
-                if ((int)rc->owner[f] >= w0 && (int)rc->owner[f] < w0 + nw) c.f[f].ctl->far_min[slot ^ 1u] = GUM_INF;
+                if ((int)rc->owner[f] >= w0 && (int)rc->owner[f] < w0 + nw) {
+                    c.f[f].ctl->far_min[slot ^ 1u] = GUM_INF;
+                    c.f[f].ctl->far_n[slot ^ 1u] = 0;  // consumed by the previous sweep; receives this one's
+                }
         }
     }
     bool done;
@@ -2219,9 +2246,12 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                             if (sval >= nfT) {
                                 park = true;
                                 const unsigned ob = atomicOr(F.far + (v >> 5), bit);
-                                if (!(ob & bit)) atomicAdd(&F.ctl->far_cnt, 1ull);
+                                if (!(ob & bit)) {
+                                    atomicAdd(&F.ctl->far_cnt, 1ull);
+                                    if (F.farl) F.farl[(size_t)fslot * F.V + atomicAdd(&F.ctl->far_n[fslot], 1u)] = v;
+                                }
                                 atomicMin(&F.ctl->far_min[fslot], sval);
-                            } else if (fw & bit) {
+                            } else if ((fw & bit) && !F.farl) {
                                 const unsigned ob = atomicAnd(F.far + (v >> 5), ~bit);
                                 if (ob & bit) atomicAdd(&F.ctl->far_cnt, ~0ull);
                             }

@@ -50,6 +50,7 @@ struct FragBufs {
     unsigned* vis = nullptr;
     unsigned* bm2 = nullptr;
     unsigned* far = nullptr;
+    unsigned* farl = nullptr;  // SSSP near-far: [2][V] far lists (gum_prepare(SSSP) with sssp_delta)
     unsigned* app = nullptr;
     unsigned* q_v = nullptr;
     unsigned long long* q_off = nullptr;
@@ -395,6 +396,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
         p.vis = F.vis;
         p.bm2 = F.bm2;
         p.far = F.far;
+        p.farl = (alg == GUM_SSSP) ? F.farl : nullptr;
         p.app = F.app;
         p.q_v = F.q_v;
         p.q_off = F.q_off;
@@ -547,7 +549,7 @@ int mp_fields(gum_ctx* c, int f, void** out[kMpFields]) {
     GUM_FLD(F.ctl); GUM_FLD(F.pr_col); GUM_FLD(F.pr_q_v); GUM_FLD(F.pr_q_off); GUM_FLD(F.pr_tile);
     GUM_FLD(F.sq_col); GUM_FLD(F.sq_q_v); GUM_FLD(F.sq_q_off); GUM_FLD(F.sq_tile); GUM_FLD(F.in_row_ptr);
     GUM_FLD(F.in_col); GUM_FLD(c->lb[f]); GUM_FLD(c->rctl[f]); GUM_FLD(c->trace[f]); GUM_FLD(c->pad[f]);
-    GUM_FLD(F.mbuf); GUM_FLD(F.pl_off); GUM_FLD(F.pl_col); GUM_FLD(F.pl_tx); GUM_FLD(F.pl_tb); GUM_FLD(c->cxg[f]);
+    GUM_FLD(F.mbuf); GUM_FLD(F.farl); GUM_FLD(F.pl_off); GUM_FLD(F.pl_col); GUM_FLD(F.pl_tx); GUM_FLD(F.pl_tb); GUM_FLD(c->cxg[f]);
     for (int g = 0; g < kMaxW; g++) {  // worker f's foster queues (NEXT-3 copy-migration)
         GUM_FLD(c->fq[f][g].q_v); GUM_FLD(c->fq[f][g].q_off); GUM_FLD(c->fq[f][g].q_base); GUM_FLD(c->fq[f][g].tile);
     }
@@ -1787,6 +1789,23 @@ gum_status gum_prepare(gum_ctx* c, gum_alg alg) {
         if (st == GUM_OK) st = build_in(c);
     }
     if (st == GUM_OK) st = build_hub(c, alg);  // worker-local copies: nothing to publish
+    if (st == GUM_OK && alg == GUM_SSSP && c->cfg.sssp_delta) {
+        // near-far: the far set also kept as two lists, so a sweep reads the parked vertices instead of
+        // scanning the whole far bitmap (one sweep per distance bucket)
+        static const int env_fl = getenv("GUM_FAR_LIST") ? atoi(getenv("GUM_FAR_LIST")) : 1;
+        bool any = false;
+        for (int f = 0; f < c->P && env_fl; f++) {
+            FragBufs& F = c->fr[f];
+            if (!frag_local(c, f) || F.farl) continue;
+            F.farl = (unsigned*)dalloc(c, F.dev, 2ull * std::max<size_t>(F.V, 1) * 4, c->part_allocs);
+            if (!F.farl) st = fail(c, GUM_ENOMEM, "far list alloc failed (fragment %d)", f);
+            any = true;
+        }
+        if (any) {
+            drop_graphs(c);
+            built = true;
+        }
+    }
     if (st == GUM_OK && alg != GUM_PR) {
         bool fb = false;
         st = build_foster(c, &fb);
