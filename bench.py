@@ -191,11 +191,11 @@ def load_peak():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def load_ncu_traffic(config, alg):
+def load_ncu_traffic(config, alg, pr_push=False):
     p = os.path.join(ROOT, "profiles", "ncu_advance_traffic.json")
     try:
         d = json.load(open(p))
-        return d.get(f"{config}_{alg}")
+        return d.get(f"{config}_{alg}" + ("_push" if alg == "pr" and pr_push else ""))
     except Exception:  # noqa: BLE001
         return None
 
@@ -375,7 +375,8 @@ def run_multiprocess(args, alg, metric, cfg_desc, ctx_kw, rank, world):
         peak, peak_src = load_peak()
         per_gpu = adv_b / world / (adv_max / 1e3) / 1e9 if adv_max else 0.0
         roof = {"bound": "hbm", "achieved": round(per_gpu, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(per_gpu / peak, 4), "traffic": None, "kernel": "k_advance", "peak_source": peak_src,
+                "frac": round(per_gpu / peak, 4), "traffic": None,
+                "kernel": "k_pr_pull" if alg == "pr" and not args.pr_push else "k_advance", "peak_source": peak_src,
                 "per": "GPU: the job's algorithmic advance bytes / N over the slowest rank's advance time",
                 "bytes_per_run": adv_b / min(len(sources), 4), "advance_ms_max_rank": adv_max / min(len(sources), 4),
                 "how": "CUDA events around every launch on each rank's stream (GUM_CFG_PROFILE, host loop), max over ranks",
@@ -439,6 +440,7 @@ def main():
                          "(C1/C2: 8 iterations, no long tail; the engine's per-iteration launch costs more than it "
                          "saves -- C2 1.622 ms with it, 1.595 ms without), where it is 0")
     ap.add_argument("--bfs-pull", type=int, default=0, help="NEXT-4 direction-optimising BFS (bottom-up iterations)")
+    ap.add_argument("--pr-push", type=int, default=0, help="PR advance as the push (red.add.f64) instead of the pull")
     args = ap.parse_args()
     alg = args.alg or DEFAULT_ALG[args.config]
     if args.part is None:
@@ -476,7 +478,8 @@ def main():
 
     if world > 1 and args.impl == "ours":
         ctx_kw = dict(fsteal=bool(args.fsteal), osteal=osteal_kw, sssp_delta=sssp_delta,
-                      tail_vertices=args.tail, bfs_direction_opt=bool(args.bfs_pull), dpr_tolerance=DPR_TOL)
+                      tail_vertices=args.tail, bfs_direction_opt=bool(args.bfs_pull), dpr_tolerance=DPR_TOL,
+                      pr_push=bool(args.pr_push))
         run_multiprocess(args, alg, metric, cfg_desc, ctx_kw, rank, world)
         return
     if rank != 0:
@@ -522,7 +525,7 @@ def main():
     dev_ids = list(range(N)) if N > 1 else None
     ctx_kw = dict(num_gpus=N, device_ids=dev_ids, fsteal=bool(args.fsteal), osteal=osteal_kw,
                   sssp_delta=sssp_delta, tail_vertices=args.tail, bfs_direction_opt=bool(args.bfs_pull),
-                  dpr_tolerance=DPR_TOL)
+                  dpr_tolerance=DPR_TOL, pr_push=bool(args.pr_push))
 
     # ---------------------------------------------------------------- device-resident timed region
     ctx = gum.Context(streams=[stream] * N if N == 1 else None, **ctx_kw)
@@ -602,14 +605,15 @@ def main():
             tail_b += tail_bytes(alg, st)
         pctx.close()
         achieved = adv_bytes / (adv_ms / 1e3) / 1e9 if adv_ms else 0.0
-        traffic = load_ncu_traffic(args.config, alg)  # (dram bytes per launch from a committed ncu capture)
+        traffic = load_ncu_traffic(args.config, alg, args.pr_push)  # (dram bytes per launch, committed ncu capture)
         how = "CUDA events around every launch on its stream (profile pass, host loop)"
         roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "traffic_source": ("profiles/ncu_advance_traffic.json: dram__bytes_read+write per k_advance launch "
                                    "from an ncu --set full capture of this config (not measured in this run)")
                 if traffic is not None else None,
-                "kernel": "k_advance", "peak_source": peak_src,
+                "kernel": ("k_pr_pull (the source-block passes of one iteration)" if alg == "pr" and not args.pr_push
+                           else "k_advance"), "peak_source": peak_src,
                 "bytes_per_launch": adv_bytes / max(adv_launches, 1),
                 "avg_launch_ms": adv_ms / max(adv_launches, 1), "how": how,
                 "bytes_model": "per edge col 4 + state 4 (+w 4 SSSP; PR acc 8), per frontier vertex 24 (PR 20), "

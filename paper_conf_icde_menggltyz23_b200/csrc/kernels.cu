@@ -1044,6 +1044,12 @@ __device__ __noinline__ void control_body(const DevCtx& c, const int alg, int w0
                     prev = hi;
                 }
             }
+#ifdef GUM_PLAN_DEBUG
+            printf("[plan] k=%u loads %llu %llu %llu %llu z=%.1f X0 %.1f %.1f %.1f %.1f lo0 %u %u %u %u hi0 %u %u %u %u nt0 %llu\n", k,
+                   lw[0], lw[1], lw[2], lw[3], rc->plan_z, X[0], X[1], X[2], X[3], rc->plan_lo[0][0], rc->plan_lo[0][1],
+                   rc->plan_lo[0][2], rc->plan_lo[0][3], rc->plan_hi[0][0], rc->plan_hi[0][1], rc->plan_hi[0][2],
+                   rc->plan_hi[0][3], vload(&c.f[0].ctl->ntiles));
+#endif
         }
         // frontier density switch: expanding more than V/dense_div edges is expected to activate a
         // dense next frontier -> the advance only sets bitmap bits (fire-and-forget) and the next
@@ -1248,17 +1254,26 @@ template <int ALG, bool MULTI, bool PB = false, bool NX = false>
 #endif
 __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_BFS * 256 / kAdvThreads : 4 * 256 / kAdvThreads) k_advance(const __grid_constant__ DevCtx c, int w0, int nw) {
     typedef typename ValT<ALG>::T VT;
-    __shared__ unsigned s_base[kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
+    // BFS (no propagation blocking / reducers): the chunk's staging buffers are double-buffered by tile parity
+    // (GUM_ADV_DB), so the barrier at the end of a chunk -- it kept the next chunk's staging from overwriting
+    // what slow warps still expand -- is not needed (3 CTA barriers per chunk instead of 4)
+#ifndef GUM_ADV_DB
+#define GUM_ADV_DB 0
+#endif
+    constexpr int NB = (GUM_ADV_DB && ALG == ALG_BFS && !PB && !NX) ? 2 : 1;
+    __shared__ unsigned s_base_b[NB][kTileMax + 1];  // col index of the chunk's first edge of each vertex (E_f < 2^32)
     __shared__ VT s_val[(ALG == ALG_BFS) ? 1 : (kTileMax + 1)];
     static_assert(kTileMax <= 4096, "s_head tags keep the vertex slot in 12 bits");
-    __shared__ __align__(16) unsigned s_head[kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
+    __shared__ __align__(16) unsigned s_head_b[NB][kTileMax];  // (tile seq << 12) | vertex slot; untagged after the scan
+    unsigned* s_base = s_base_b[0];
+    unsigned* s_head = s_head_b[0];
     // BFS propagation blocking: per-chunk counting sort of discovered-candidate ids by destination block
     constexpr int PBB = (ALG == ALG_BFS && !MULTI && PB) ? kPbMaxBins : 1;  // (own instantiation:
     // the shared arrays would otherwise shrink L1, which the random probes of the plain path live on)
     constexpr int PBS = (ALG == ALG_BFS && !MULTI && PB) ? kTileMax : 1;
     __shared__ unsigned s_pbcnt[PBB], s_pboff[PBB], s_pbg[PBB];
     __shared__ unsigned short s_stbin[PBS];
-    unsigned* const s_stage = s_head;  // s_head is dead once the chunk's col ids are loaded
+    unsigned* const s_stage = s_head_b[0];  // s_head is dead once the chunk's col ids are loaded (NB == 1 here)
     __shared__ unsigned s_wmax[kAdvThreads / 32];
     // NEXT-1 hub cache: per staged vertex, 1 = its list is expanded from this worker's local copy
     __shared__ unsigned char s_hub[(MULTI && NX) ? kTileMax : 1];
@@ -1315,7 +1330,8 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
     }
     const unsigned long long t0 = globaltimer();
     const unsigned CH = c.chunk;
-    for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kAdvThreads) s_head[e] = 0;
+    for (int q = 0; q < NB; q++)
+        for (unsigned e = threadIdx.x; e < (unsigned)kTileMax; e += kAdvThreads) s_head_b[q][e] = 0;
     unsigned seq = 0;    // tile sequence number of this CTA (tags s_head entries; no per-tile clearing)
     int own_cursor = 0;  // fragments (w + i) % P for i < own_cursor are drained
     unsigned long long e_own = 0, e_stolen = 0, remote = 0, acts = 0, filtered = 0, hub_e = 0;
@@ -1501,6 +1517,10 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
 
         // ---- stage the chunk's frontier vertices (merge path over the degree prefix, CTA-local)
         seq++;
+        if (NB == 2) {
+            s_base = s_base_b[seq & 1u];
+            s_head = s_head_b[seq & 1u];
+        }
         for (unsigned kk = threadIdx.x; kk < nv; kk += kAdvThreads) {
             unsigned long long off;
             unsigned base, u;
@@ -1884,7 +1904,7 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                 e_own += tlen;
             }
         }
-        __syncthreads();
+        if (NB == 1) __syncthreads();  // (double-buffered: the next chunk stages into the other buffers)
         cur = nxt;
     }
     // run counters (warp-reduced) and the per-worker busy window of this iteration

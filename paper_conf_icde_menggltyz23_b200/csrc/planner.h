@@ -7,7 +7,7 @@
 // Alg. 1 hands to SCIP) then has a closed form (SURVEY c-7): donors (l_i > z) keep z of their own edges
 // and give l_i - z away; receivers (l_j <= z) keep all of theirs and take (z - l_j)/b; z solves
 //     sum_i max(l_i - z, 0) = sum_j max(z - l_j, 0) / b,
-// found by bisection (the left side minus the right is decreasing in z). X is filled donor-major
+// found exactly by waterfill_z (the left side minus the right is decreasing and piecewise linear in z). X is filled donor-major
 // ("north-west corner" over increasing worker ids). Rounding to whole chunks happens in the caller.
 #pragma once
 
@@ -19,24 +19,47 @@
 
 namespace gum {
 
+// The balance point of the closed form, exactly: the balance function
+//     extra + sum_i max(v_i - z, 0) - sum_i max(z - v_i, 0) / b
+// is decreasing and linear between consecutive loads (the loads below z are receivers, the others donors:
+// extra + S_donors - n_d z - (n_r z - S_recv)/b), so z is the root of the one segment that contains it,
+// found from the balance at the loads themselves -- O(m^2) cheap operations, where a bisection took hundreds
+// of fp64 divisions on the control kernel's single thread (0.1-0.9 ms per iteration, measured in round 2).
+// extra = work that must move off evicted fragments (OSteal), 0 for FSteal. v_i >= 0, m in 1..8, b >= 1.
+GUM_HD inline double waterfill_balance(const double* v, int m, double extra, double b, double z) {
+    double f = extra;
+    for (int i = 0; i < m; i++) f += v[i] > z ? v[i] - z : -(z - v[i]) / b;
+    return f;
+}
+GUM_HD inline double waterfill_z(const double* v, int m, double extra, double b) {
+    // the segment [lo, hi) between consecutive loads where the balance changes sign: lo = the largest load
+    // (or 0) with balance >= 0; on it the loads <= lo are receivers and the others donors
+    double lo = 0.0;
+    for (int i = 0; i < m; i++)
+        if (v[i] > lo && waterfill_balance(v, m, extra, b, v[i]) >= 0.0) lo = v[i];
+    double num = extra, den = 0.0;
+    for (int i = 0; i < m; i++) {
+        if (v[i] > lo) {
+            num += v[i];
+            den += 1.0;
+        } else {
+            num += v[i] / b;
+            den += 1.0 / b;
+        }
+    }
+    return num / den;
+}
+
 GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double b, double* X) {
     for (int i = 0; i < n * n; i++) X[i] = 0.0;
     if (n <= 0) return 0.0;
     if (b < 1.0) b = 1.0;
-    double lo = 0.0, hi = 0.0;
-    for (int i = 0; i < n; i++) hi = (double)l[i] > hi ? (double)l[i] : hi;
-    for (int it = 0; it < 200; it++) {  // bisection on the balance function
-        const double z = 0.5 * (lo + hi);
-        double give = 0.0, take = 0.0;
-        for (int i = 0; i < n; i++) {
-            const double li = (double)l[i];
-            if (li > z) give += li - z;
-            else take += (z - li) / b;
-        }
-        if (give > take) lo = z;
-        else hi = z;
-    }
-    const double z = hi;
+    double v[8];
+    for (int i = 0; i < n; i++) v[i] = (double)l[i];
+    const double zz = waterfill_z(v, n, 0.0, b);
+    double hi = 0.0;
+    for (int i = 0; i < n; i++) hi = v[i] > hi ? v[i] : hi;
+    const double z = zz < hi ? zz : hi;  // (all loads equal: the root is that load)
     double g[8], r[8];
     for (int i = 0; i < n; i++) {
         const double li = (double)l[i];
@@ -52,7 +75,7 @@ GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double
             g[i] -= t;
             r[j] -= t;
         }
-        X[i * n + i] += g[i];  // bisection residue stays with its owner
+        X[i * n + i] += g[i];  // rounding residue stays with its owner
     }
     return z;
 }
@@ -67,25 +90,12 @@ GUM_HD inline double osteal_makespan(const unsigned long long* l, int n, int m, 
     if (n <= 0 || m <= 0) return 0.0;
     if (m > n) m = n;
     if (b < 1.0) b = 1.0;
-    double evicted = 0.0, hi = 0.0;
+    double v[8], evicted = 0.0;
     for (int i = 0; i < n; i++) {
-        if (i >= m) evicted += (double)l[i];
-        hi = (double)l[i] > hi ? (double)l[i] : hi;
+        if (i < m) v[i] = (double)l[i];
+        else evicted += (double)l[i];
     }
-    hi += evicted * b;  // z <= max own load + all evicted work on one survivor
-    double lo = 0.0;
-    for (int it = 0; it < 200; it++) {
-        const double z = 0.5 * (lo + hi);
-        double give = evicted, take = 0.0;
-        for (int j = 0; j < m; j++) {
-            const double lj = (double)l[j];
-            if (lj > z) give += lj - z;
-            else take += (z - lj) / b;
-        }
-        if (give > take) lo = z;
-        else hi = z;
-    }
-    return hi;
+    return waterfill_z(v, m, evicted, b);
 }
 
 // Alg. 2: enumerate m = 1..n, E(m) = z(m) + p*m (Eq. 4), keep the first strict minimum. cost[m-1] =
