@@ -26,25 +26,27 @@ namespace gum {
 // found from the balance at the loads themselves -- O(m^2) cheap operations, where a bisection took hundreds
 // of fp64 divisions on the control kernel's single thread (0.1-0.9 ms per iteration, measured in round 2).
 // extra = work that must move off evicted fragments (OSteal), 0 for FSteal. v_i >= 0, m in 1..8, b >= 1.
-GUM_HD inline double waterfill_balance(const double* v, int m, double extra, double b, double z) {
+GUM_HD inline double waterfill_balance(const double* v, int m, double extra, double ib, double z) {
     double f = extra;
-    for (int i = 0; i < m; i++) f += v[i] > z ? v[i] - z : -(z - v[i]) / b;
+    for (int i = 0; i < m; i++) f += v[i] > z ? v[i] - z : (v[i] - z) * ib;
     return f;
 }
 GUM_HD inline double waterfill_z(const double* v, int m, double extra, double b) {
     // the segment [lo, hi) between consecutive loads where the balance changes sign: lo = the largest load
-    // (or 0) with balance >= 0; on it the loads <= lo are receivers and the others donors
+    // (or 0) with balance >= 0; on it the loads <= lo are receivers and the others donors. (Multiplications
+    // by 1/b: a single thread's fp64 divisions were the control kernel's cost.)
+    const double ib = 1.0 / b;
     double lo = 0.0;
     for (int i = 0; i < m; i++)
-        if (v[i] > lo && waterfill_balance(v, m, extra, b, v[i]) >= 0.0) lo = v[i];
+        if (v[i] > lo && waterfill_balance(v, m, extra, ib, v[i]) >= 0.0) lo = v[i];
     double num = extra, den = 0.0;
     for (int i = 0; i < m; i++) {
         if (v[i] > lo) {
             num += v[i];
             den += 1.0;
         } else {
-            num += v[i] / b;
-            den += 1.0 / b;
+            num += v[i] * ib;
+            den += ib;
         }
     }
     return num / den;

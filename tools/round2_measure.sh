@@ -18,5 +18,10 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_ad
   python tools/profile_run.py --config C2 --alg bfs --part degree --runs 1 > $O/ncu_adv_C2.log 2>&1; python tools/ncu_summary.py $O/adv_C2.ncu-rep 12 > $O/ncu_full_k_advance_C2_bfs_peak.txt 2>&1; head -25 $O/ncu_full_k_advance_C2_bfs_peak.txt
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_pr_pull -s 14 -c 1 -o $O/pull_C5 -f \
   python tools/profile_run.py --config C5 --alg pr --part degree --runs 1 > $O/ncu_pull_C5.log 2>&1; python tools/ncu_summary.py $O/pull_C5.ncu-rep 12 > $O/ncu_full_k_pr_pull_C5.txt 2>&1; head -25 $O/ncu_full_k_pr_pull_C5.txt
+timeout 900 python tools/ablation.py --next1 --scale 20 --workers 8 --out $O/abl_next1.json > $O/abl_next1.txt 2>&1; cat $O/abl_next1.txt
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_C3_sssp.csv \
+  python tools/profile_run.py --config C3 --alg sssp --runs 1 > $O/launches_C3.log 2>&1; python tools/launches.py $O/launches_C3_sssp.csv > $O/launches_C3_sssp_summary.txt; head -8 $O/launches_C3_sssp_summary.txt
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_tail -s 5 -c 1 -o $O/tail_C3 -f \
+  python tools/profile_run.py --config C3 --alg sssp --runs 1 > $O/ncu_tail_C3.log 2>&1; python tools/ncu_summary.py $O/tail_C3.ncu-rep 12 > $O/ncu_full_k_tail_C3_sssp.txt 2>&1; head -25 $O/ncu_full_k_tail_C3_sssp.txt
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_C5_pr.csv \
   python tools/profile_run.py --config C5 --alg pr --part degree --runs 1 > $O/launches_C5.log 2>&1; python tools/launches.py $O/launches_C5_pr.csv > $O/launches_C5_pr_summary.txt; head -8 $O/launches_C5_pr_summary.txt
