@@ -1216,6 +1216,16 @@ struct ValT<ALG_DPR> {
 
 // Warp-aggregated append of this thread's activations (bit j of need: slot j) to the owner
 // fragments' activation lists: one reservation atomic per warp and target fragment.
+// TMA bulk prefetch of [p, p + bytes) into L2 (cp.async.bulk.prefetch: 16-byte granules, no registers held)
+#ifndef GUM_ADV_PF
+#define GUM_ADV_PF 0
+#endif
+__device__ __forceinline__ void prefetch_l2_range(const void* p, unsigned bytes) {
+    const unsigned long long a = (unsigned long long)p & ~15ull;
+    const unsigned long long e = ((unsigned long long)p + bytes + 15ull) & ~15ull;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((unsigned)(e - a)));
+}
+
 template <bool MULTI>
 __device__ __forceinline__ unsigned append_activations(const DevCtx& c, unsigned need, const unsigned char* tfv,
                                                        const unsigned* lvv) {
@@ -1623,6 +1633,26 @@ __global__ void __launch_bounds__(kAdvThreads, (ALG == ALG_BFS) ? GUM_ADV_MINB_B
                         vv[j] = GUM_INF;
                     }
                     cv[j] = (VT)(unsigned)nd;
+                }
+            }
+        }
+        if (GUM_ADV_PF && !(MULTI && NX)) {
+            // L2 bulk prefetch of the next chunk's adjacency (col, SSSP w): the next chunk's staging values
+            // were issued before this chunk's col loads and have arrived by now; the TMA engine pulls the
+            // vertex's run of the next chunk into L2, so its col loads wait for L2 instead of HBM latency
+            const unsigned long long n_off = __shfl_down_sync(0xffffffffu, p_off, 1);
+            if (nxt.f >= 0 && threadIdx.x < nxt.nv) {
+                const unsigned long long ntb = nxt.t * CH;
+                const long long r0 = (long long)p_off - (long long)ntb;
+                const bool last = lane_id() == 31 || threadIdx.x + 1 >= nxt.nv;
+                const long long r1 = last ? (long long)nxt.tlen : (long long)n_off - (long long)ntb;
+                const long long a = r0 > 0 ? r0 : 0, b = r1 < (long long)nxt.tlen ? r1 : (long long)nxt.tlen;
+                if (b > a) {
+                    const FragPtrs& Fn = c.f[nxt.f];
+                    const bool nsq = ALG == ALG_WCC && blk && Fn.sq_col != nullptr;
+                    const unsigned ci = (unsigned)(p_base + (unsigned)a);
+                    prefetch_l2_range((nsq ? Fn.sq_col : Fn.col) + ci, (unsigned)(b - a) * 4u);
+                    if (ALG == ALG_SSSP) prefetch_l2_range(Fn.w + ci, (unsigned)(b - a) * 4u);
                 }
             }
         }
