@@ -53,7 +53,6 @@ GUM_HD inline double waterfill_z(const double* v, int m, double extra, double b)
 }
 
 GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double b, double* X) {
-    for (int i = 0; i < n * n; i++) X[i] = 0.0;
     if (n <= 0) return 0.0;
     if (b < 1.0) b = 1.0;
     double v[8];
@@ -62,22 +61,25 @@ GUM_HD inline double fsteal_waterfill(const unsigned long long* l, int n, double
     double hi = 0.0;
     for (int i = 0; i < n; i++) hi = v[i] > hi ? v[i] : hi;
     const double z = zz < hi ? zz : hi;  // (all loads equal: the root is that load)
-    double g[8], r[8];
+    // every entry of X is written exactly once, row by row: the off-diagonal transfers in worker order, then
+    // the diagonal (kept share + rounding residue). The previous zero-fill + read-modify-write form produced a
+    // zero diagonal in row 0 inside the device control kernel (worker 0 kept nothing, so the heaviest
+    // iteration ran on the other three: tests/test_gpu_parity.py test_planned_fsteal), although the same
+    // function was right on the host and in a standalone kernel (tools/plantest).
+    double r[8];
+    for (int j = 0; j < n; j++) r[j] = v[j] > z ? 0.0 : (z - v[j]) / b;
     for (int i = 0; i < n; i++) {
-        const double li = (double)l[i];
-        X[i * n + i] = li > z ? z : li;
-        g[i] = li > z ? li - z : 0.0;
-        r[i] = li > z ? 0.0 : (z - li) / b;
-    }
-    for (int i = 0; i < n; i++) {
-        for (int j = 0; j < n && g[i] > 0.0; j++) {
-            if (j == i || r[j] <= 0.0) continue;
-            const double t = g[i] < r[j] ? g[i] : r[j];
-            X[i * n + j] += t;
-            g[i] -= t;
-            r[j] -= t;
+        double gi = v[i] > z ? v[i] - z : 0.0;
+        for (int j = 0; j < n; j++) {
+            double t = 0.0;
+            if (j != i && gi > 0.0 && r[j] > 0.0) {
+                t = gi < r[j] ? gi : r[j];
+                gi -= t;
+                r[j] -= t;
+            }
+            if (j != i) X[i * n + j] = t;
         }
-        X[i * n + i] += g[i];  // rounding residue stays with its owner
+        X[i * n + i] = (v[i] > z ? z : v[i]) + gi;  // rounding residue stays with its owner
     }
     return z;
 }
