@@ -70,7 +70,13 @@ struct alignas(128) FragCtl {
     unsigned int qown, pad_q;            // NEXT-3 copy-migration: the worker whose memory holds the current queue
                                          // (set by the filter that generated it; the advance may run after an
                                          // owner change, so it follows this, not the current owner)
+    unsigned long long fpack;            // one-pass filter: (queue entries << kFpackShift) | out-edges reserved so far
+    unsigned int fdone, pad_f;           // one-pass filter: CTAs finished (the last one publishes and resets)
 };
+// one-pass filter reservation counter: entries in the high 27 bits, edges in the low 37 (runtime checks V_g and
+// E_g fit, else the two-pass filter runs)
+constexpr unsigned kFpackShift = 37;
+constexpr unsigned long long kFpackEdgeMask = (1ull << kFpackShift) - 1;
 
 // Per launch unit (device) run-control replica: decisions are computed redundantly and
 // identically by every unit from the same gathered counts (no policy broadcast).
@@ -257,6 +263,7 @@ struct DevCtx {
     unsigned int bfs_pull;      // direction-optimising BFS enabled (in-CSR built)
     unsigned long long total_edges;  // sum of the fragments' out-edges
     int mirrors;                // NEXT-1 outer-vertex mirrors (P > 1 only)
+    unsigned int filter_onepass;  // filter: one pass, queue ranges reserved per tile with one packed atomic
     unsigned int filter_swizzle;  // filter: spread each CTA's tile range over the id space (stride permutation)
     unsigned int bfs_filter_depth;  // BFS: the filter writes the depth of the vertices it takes from the
                                     // activations (the advance only sets visited / frontier bits)

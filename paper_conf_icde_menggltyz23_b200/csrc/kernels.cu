@@ -572,10 +572,24 @@ __device__ __forceinline__ Pair filter_tile(const FragPtrs& F, NfAcc& acc, bool 
 // block scan for the per-thread offsets and the emit in one walk of the tile (FT_COUNT + FT_EMIT read the
 // bitmap word and the row_ptr run twice). Only the 8-bit accepted mask stays live across the scan; the
 // row_ptr run is re-read after it from L1 (the same thread's lines). Returns the tile's totals.
+// one-pass filter: thread 0 reserves the tile's queue range [cnt, cnt + tot.cnt) and edge range with ONE
+// atomic on the packed counter (both ranges in the same order, so q_off stays the prefix of the degrees in
+// queue order) and broadcasts the base; every thread returns the base in (pos, off)
+__device__ __forceinline__ void filter_reserve(unsigned long long* fpack, const Pair& tot, unsigned long long& pos,
+                                               unsigned long long& off) {
+    __shared__ unsigned long long s_fbase;
+    if (threadIdx.x == 0)
+        s_fbase = tot.cnt ? atomicAdd(fpack, (tot.cnt << kFpackShift) | tot.deg) : 0ull;
+    __syncthreads();
+    pos = s_fbase >> kFpackShift;
+    off = s_fbase & kFpackEdgeMask;
+}
+
 template <bool DPR = false>
 __device__ __forceinline__ Pair filter_tile_dense_fused(const FragPtrs& F, bool keep_fbm, unsigned depth, unsigned tile,
                                                         unsigned nwords, unsigned chunk, unsigned long long pos,
-                                                        unsigned long long off, Pair* s_warp, double dd = 0.0) {
+                                                        unsigned long long off, Pair* s_warp, double dd = 0.0,
+                                                        unsigned long long* fpack = nullptr) {
     const unsigned lane = lane_id();
     const unsigned wbase = tile * kDenseWordsPerPart + (threadIdx.x >> 5) * kDenseWordsPerWarp;
     const unsigned vb = wbase * 32u + lane * kDenseVertsPerThread;
@@ -642,6 +656,7 @@ __device__ __forceinline__ Pair filter_tile_dense_fused(const FragPtrs& F, bool 
     }
     Pair tot;
     const Pair tex = block_excl_scan_tile(mine, s_warp, tot);
+    if (fpack) filter_reserve(fpack, tot, pos, off);  // one-pass filter (CTA-uniform)
     if (ok) {
         unsigned long long p = pos + tex.cnt, o = off + tex.deg;
 #pragma unroll
@@ -782,6 +797,53 @@ __global__ void __launch_bounds__(kThreads, GUM_FILTER_MINB) k_filter(const __gr
         if (stride >= n_tiles) stride = 1;
     }
 
+    if (!NF && c.filter_onepass) {
+        // ---- one pass: per tile count -> block scan -> one packed atomic reserves the tile's queue and edge
+        // ranges -> emit. No look-back and no second walk; the queue is in reservation order (nothing depends
+        // on it being sorted: q_off is the prefix of the degrees in queue order, the chunk table follows it)
+        unsigned long long* fpack = &ct->fpack;
+        NfAcc nfo;
+        for (unsigned t = t_lo; t < t_hi; t++) {
+            const unsigned pt = (unsigned)((unsigned long long)t * stride % n_tiles);
+            if (dense) {
+                filter_tile_dense_fused<DPR>(F, keep_fbm, depth, pt, nwords, chunk, 0, 0, s_warp, dd, fpack);
+            } else {
+                const Pair q = filter_tile<FT_COUNT, DPR>(F, nfo, keep_fbm, depth, pt, dense, sweep, false, nfT, nwords,
+                                                          app_cnt, ipt, chunk, 0, 0, dd);
+                Pair tot;
+                const Pair tex = block_excl_scan_tile(q, s_warp, tot);
+                unsigned long long bp, bo;
+                filter_reserve(fpack, tot, bp, bo);
+                // (always: the emit walk also clears the consumed bitmap words and writes BFS depths)
+                filter_tile<FT_EMIT, DPR>(F, nfo, keep_fbm, depth, pt, dense, sweep, false, nfT, nwords, app_cnt, ipt,
+                                          chunk, bp + tex.cnt, bo + tex.deg, dd);
+            }
+            filter_flush_long(F);
+        }
+        // the last of the G participating CTAs publishes the queue and re-arms the counters
+        __threadfence();
+        __syncthreads();
+        if (threadIdx.x == 0 && atomicAdd(&ct->fdone, 1u) == G - 1) {
+            __threadfence();
+            const unsigned long long pk = atomicExch(fpack, 0ull);
+            ct->fdone = 0;
+            const unsigned long long tc = pk >> kFpackShift, td = pk & kFpackEdgeMask;
+            s_qo.q_off[tc] = td;
+            ct->qlen = tc;
+            ct->qown = vload(&rc->owner[f]);
+            if (c.migrate && s_qo.q_v != F.q_v) ct->migrated_q += tc;
+            ct->qedges = td;
+            ct->ntiles = (td + chunk - 1) / chunk;
+            ct->claim = 0;
+            for (int q = 0; q < kMaxW; q++) ct->pclaim[q] = 0;
+            ct->app_cnt = 0;
+            ct->dense = dense ? 1u : 0u;
+            ct->frontier_edges += td;
+            ct->frontier_vertices += tc;
+        }
+        if (fuse_ctl) filter_arrive(c, w0, nw, h, use_h);
+        return;
+    }
     // ---- pass 1: aggregate of this CTA's tile range
     Pair mine{0, 0};
     NfAcc nfa;

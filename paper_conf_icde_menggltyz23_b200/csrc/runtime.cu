@@ -495,6 +495,14 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
     static const int env_sw = getenv("GUM_FILTER_SWIZZLE") ? atoi(getenv("GUM_FILTER_SWIZZLE")) : 1;
     d.filter_swizzle = env_sw ? 1u : 0u;
+    // one-pass filter (queue ranges reserved per tile with one packed atomic): needs every fragment's queue
+    // length < 2^27 and out-edges (symmetric for WCC) < 2^37, the packed counter's two fields
+    static const int env_op = getenv("GUM_FILTER_ONEPASS") ? atoi(getenv("GUM_FILTER_ONEPASS")) : 1;
+    bool op_fits = true;
+    for (int f = 0; f < c->P; f++)
+        op_fits = op_fits && c->fr[f].V < (1ull << (64 - kFpackShift)) &&
+                  std::max(c->fr[f].E, c->fr[f].sE) <= kFpackEdgeMask;
+    d.filter_onepass = (env_op && op_fits) ? 1u : 0u;
     d.bfs_filter_depth = alg == GUM_BFS ? 1u : 0u;  // (the advance no longer writes BFS depths)
     static const int env_wb = getenv("GUM_WCC_BLOCKED") ? atoi(getenv("GUM_WCC_BLOCKED")) : 1;
     d.wcc_blocked = (alg == GUM_WCC && c->fr[0].sq_col && c->cfg.fsteal != 2 && env_wb) ? 1u : 0u;
