@@ -2872,9 +2872,13 @@ cudaError_t pr_push_occupancy(int* blocks_per_sm) {
 // global fp64 atomic: <= 2 atomics per tile instead of one red.add.f64 per edge.
 // (A three-stage cp.async pipeline -- ids, then 8-byte async gathers, then the reduction -- measured 2x
 // slower on C5: DESIGN.md §6.)
+__device__ __forceinline__ unsigned pull_slot(unsigned e) { return e + (e >> 3); }
+
 __global__ void __launch_bounds__(kThreads) k_pr_pull(const __grid_constant__ DevCtx c, int w0, int nw, int pass) {
     __shared__ unsigned s_re[kPullTile + 1];  // row ends (relative to the pass's first edge) of the tile's rows
-    __shared__ double s_val[kPullTile];       // x[u]/outdeg(u) of the tile's edges
+    // x[u]/outdeg(u) of the tile's edges, one pad slot after every 8 (pull_slot): the walk's lanes read items
+    // ~8 apart, i.e. 64 bytes apart unpadded -- a 16-way bank conflict per LDS.64; padded, 72 bytes apart
+    __shared__ double s_val[kPullTile + kPullTile / 8];
     __shared__ double s_acc[kPullTile + 1];   // acc of the tile's rows (rows x0 .. x1)
     __shared__ unsigned s_key[kThreads];
     __shared__ double s_inc[kThreads];
@@ -2941,7 +2945,7 @@ __global__ void __launch_bounds__(kThreads) k_pr_pull(const __grid_constant__ De
 #pragma unroll
             for (int j = 0; j < kPullIPT; j++) {
                 const unsigned e = threadIdx.x + j * kThreads;
-                if (e < ne_t) s_val[e] = __ldg(cx + cu[j]);
+                if (e < ne_t) s_val[pull_slot(e)] = __ldg(cx + cu[j]);
             }
         }
         const unsigned nr = (x1 < Vf ? x1 : Vf - 1u) - x0 + 1u;
@@ -2971,7 +2975,7 @@ __global__ void __launch_bounds__(kThreads) k_pr_pull(const __grid_constant__ De
         for (int k = 0; k < kPullIPT; k++) {
             if ((unsigned)k < ni) {
                 if (yi < s_re[xi - x0]) {
-                    sum += s_val[yi - y0];
+                    sum += s_val[pull_slot(yi - y0)];
                     yi++;
                 } else {
                     if (!has_first) {
