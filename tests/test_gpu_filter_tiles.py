@@ -57,3 +57,31 @@ def test_filter_stride_coprime_6159_tiles():
     s = int(src[0])
     check(g, "bfs", s, csr=csr, force_mode="dense", tail_vertices=0)
     check(g, "bfs", s, csr=csr, force_mode="sparse", tail_vertices=0)
+
+
+CHILD_TWO_PASS = r"""
+import sys
+sys.path.insert(0, ROOT)
+import inputs
+from tests.gpu_helpers import check, csr_of
+g = inputs.rmat(16, 16, seed=35)
+s = inputs.pick_source(g, 35)
+csr = csr_of(g)
+for alg in ("bfs", "sssp", "wcc", "pr"):
+    for kw in (dict(), dict(num_gpus=3, part="random"), dict(force_mode="sparse", tail_vertices=0),
+               dict(force_mode="dense", tail_vertices=0)):
+        check(g, alg, s, csr=csr, **kw)
+        print("ok", alg, flush=True)
+"""
+
+
+@pytest.mark.parametrize("onepass", ["0", "1"])
+def test_filter_one_and_two_pass(onepass):
+    """The one-pass filter (default: one packed atomic reserves each tile's queue and edge ranges) and the
+    two-pass reduce-then-scan filter (GUM_FILTER_ONEPASS=0, read once per process) give the oracle's results
+    for every algorithm, on one and three workers, forced sparse and dense."""
+    env = dict(os.environ, GUM_FILTER_ONEPASS=onepass, GUM_FILTER_CTAS_PER_SM="1")
+    r = subprocess.run([sys.executable, "-c", f"ROOT = {ROOT!r}\n" + CHILD_TWO_PASS], cwd=ROOT, env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert r.stdout.count("ok ") == 16, r.stdout
