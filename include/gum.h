@@ -208,7 +208,8 @@ typedef struct {
     uint64_t hub_cached_edges;/* NEXT-1 hub cache: edges of non-local fragments expanded from a local copy */
     uint64_t mirror_flush_bytes; /* PR mirrors: bytes the finalize read from peer mirrors */
     uint32_t blocked_iterations; /* WCC: iterations run on the static destination-blocked queue */
-    uint32_t pad0;
+    uint32_t tail_overflows;  /* tail-engine hand-backs whose next list (no-dedupe mode) outgrew its buffer and
+                                 went back to the regular path as a bitmap (0 in practice) */
     /* of edges_expanded / vertices_frontier (list entries) / activations: the share done inside the tail
      * engine (k_tail), so per-kernel byte counts can be attributed (bench.py roofline) */
     uint64_t tail_edges;

@@ -82,7 +82,7 @@ class gum_run_stats(ctypes.Structure):
                 ("pr_last_residual", ctypes.c_double), ("kernel_launches", ctypes.c_uint64),
                 ("remote_filtered", ctypes.c_uint64), ("hub_cached_edges", ctypes.c_uint64),
                 ("mirror_flush_bytes", ctypes.c_uint64), ("blocked_iterations", ctypes.c_uint32),
-                ("pad0", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
+                ("tail_overflows", ctypes.c_uint32), ("tail_edges", ctypes.c_uint64), ("tail_vertices", ctypes.c_uint64),
                 ("tail_activations", ctypes.c_uint64), ("unit_barriers", ctypes.c_uint32 * MAX_WORKERS),
                 ("unit_last_iter", ctypes.c_uint32 * MAX_WORKERS), ("host_launches", ctypes.c_uint64),
                 ("osteal_p", ctypes.c_double), ("osteal_p_samples", ctypes.c_uint32), ("pad1", ctypes.c_uint32),
@@ -197,7 +197,7 @@ class RunStats:
     hub_cached_edges: int = 0
     mirror_flush_bytes: int = 0
     blocked_iterations: int = 0
-    pad0: int = 0
+    tail_overflows: int = 0
     tail_edges: int = 0
     tail_vertices: int = 0
     tail_activations: int = 0

@@ -26,6 +26,7 @@ constexpr int kDenseWordsPerPart = (kThreads / 32) * kDenseWordsPerWarp;  // 64 
 constexpr int kFilterAppPerThread = 8;                            // sparse filter: list entries per thread
 constexpr int kFilterAppPerPart = kThreads * kFilterAppPerThread; // 2048
 constexpr int kTraceMax = 1 << 16;
+constexpr unsigned kTailSlack = 1u << 20;  // tail-engine lists (q_v, app): entries beyond V (no-dedupe duplicates)
 constexpr int kPbMaxBins = 1024;       // propagation blocking: max destination blocks per fragment
 constexpr unsigned kPrPiece = 64;      // PR warp-task path: max edges per queue entry
 #ifndef GUM_PULL_IPT
@@ -71,7 +72,8 @@ struct alignas(128) FragCtl {
                                          // (set by the filter that generated it; the advance may run after an
                                          // owner change, so it follows this, not the current owner)
     unsigned long long fpack;            // one-pass filter: (queue entries << kFpackShift) | out-edges reserved so far
-    unsigned int fdone, pad_f;           // one-pass filter: CTAs finished (the last one publishes and resets)
+    unsigned int fdone;                  // one-pass filter: CTAs finished (the last one publishes and resets)
+    unsigned int tail_ovf;               // tail-engine hand-backs after a no-dedupe list overflow (stats)
 };
 // one-pass filter reservation counter: entries in the high 27 bits, edges in the low 37 (runtime checks V_g and
 // E_g fit, else the two-pass filter runs)
@@ -257,6 +259,8 @@ struct DevCtx {
     unsigned int nf_delta;      // SSSP near-far split increment (0 = plain BSP frontier, the paper's)
     unsigned int tail_enter;    // tail engine: enter when the frontier has <= tail_enter vertices (0 = off)
     unsigned int tail_exit;     // tail engine: hand back when the next frontier exceeds tail_exit vertices
+    unsigned int tail_slack;    // tail engine: list entries usable beyond V (<= kTailSlack; smaller only to test the overflow path)
+    unsigned int tail_nodedupe; // tail engine: improvements by returning atomicMin, no dedupe bits (duplicates allowed)
     unsigned int tail_local;    // tail engine: local relaxation rounds per CTA before each grid barrier
     unsigned int pb_shift;      // BFS propagation blocking: log2(block size); 0 = off
     unsigned int pb_nb;         // bins of fragment 0 (single-fragment only)

@@ -146,6 +146,9 @@ __global__ void k_init(const __grid_constant__ DevCtx c, int f0) {
         ct->remote_filtered = 0;
         ct->hub_edges = 0;
         ct->tail_edges = ct->tail_vertices = ct->tail_acts = 0;
+        ct->tail_ovf = 0;
+        ct->fpack = 0;  // one-pass filter reservation (a run that stopped mid-filter leaves no residue)
+        ct->fdone = 0;
         ct->qown = (unsigned)f;
         ct->migrated_q = 0;
         if (sq) {
@@ -2090,6 +2093,15 @@ constexpr unsigned kTailSplitCap = 8192;
 
 // Expands edges [e_lo, e_hi) of vertex v (fragment F, value sval) with one warp: check -> red.min ->
 // dedupe on this iteration's next-list bitmap -> warp-aggregated append (+ its out-degree).
+// tail-engine list append with a capacity check: the lists hold V entries plus kTailSlack (no-dedupe mode may
+// list a vertex twice). An append past that keeps the vertex as a bit of the fragment's frontier bitmap
+// instead; the reservation counter then exceeds the engine's exit bound, so the engine stops after this
+// iteration and hands its frontier back to the regular path as a bitmap (dense), listed vertices included.
+__device__ __forceinline__ void tail_put(const DevCtx& c, const FragPtrs& T, unsigned* nxt, unsigned idx, unsigned v) {
+    if (idx < T.V + c.tail_slack) nxt[idx] = v;
+    else atomicOr(T.bm + (v >> 5), 1u << (v & 31));
+}
+
 template <int ALG, bool MULTI>
 __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs& F, unsigned sval,
                                                 unsigned long long e_lo, unsigned long long e_hi, unsigned k,
@@ -2126,7 +2138,11 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
                     }
                     cand = (unsigned)nd;
                 }
-                if (ok && cand < vload(T.state + lu)) {
+                if (ok && c.tail_nodedupe) {
+                    // one returning atomic: whoever lowers the value appends v (the lists may hold a vertex
+                    // twice; its second expansion relaxes nothing new)
+                    need = cand < atomicMin(T.state + lu, cand);
+                } else if (ok && cand < vload(T.state + lu)) {
                     atomicMin(T.state + lu, cand);
                     // the next list of iteration `it` dedupes on bm (it even) / bm2 (it odd)
                     unsigned* const dw = ((it & 1) ? T.bm2 : T.bm) + (lu >> 5);
@@ -2145,7 +2161,7 @@ __device__ __forceinline__ unsigned tail_expand(const DevCtx& c, const FragPtrs&
             if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
             base = __shfl_sync(grp, base, leader);
             unsigned* nxt = (it & 1) ? T.q_v : T.app;
-            nxt[base + __popc(grp & lanemask_lt())] = lu;
+            tail_put(c, T, nxt, base + __popc(grp & lanemask_lt()), lu);
             acts++;
         }
         // out-edges of the appended vertices: one atomic per group (the counter is a single address)
@@ -2225,7 +2241,9 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
                     }
                     cand = (unsigned)nd;
                 }
-                if (ok && cand < vload(T.state + lu)) {
+                if (ok && c.tail_nodedupe) {
+                    need = cand < atomicMin(T.state + lu, cand);  // (see tail_expand)
+                } else if (ok && cand < vload(T.state + lu)) {
                     atomicMin(T.state + lu, cand);
                     unsigned* const dw = ((it & 1) ? T.bm2 : T.bm) + (lu >> 5);
                     // (release ordering is only needed when local rounds take entries out of the list)
@@ -2258,7 +2276,7 @@ __device__ __forceinline__ unsigned tail_expand_g(const DevCtx& c, const FragPtr
                 if (lane == leader) base = atomicAdd(&T.ctl->tcnt[ns], (unsigned)__popc(grp));
                 base = __shfl_sync(grp, base, leader);
                 unsigned* nxt = (it & 1) ? T.q_v : T.app;
-                nxt[base + __popc(grp & lanemask_lt())] = lu;
+                tail_put(c, T, nxt, base + __popc(grp & lanemask_lt()), lu);
                 if (lane == leader) atomicAdd(&T.ctl->tedges[ns], gdeg);
             }
             acts++;
@@ -2345,10 +2363,11 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
                     if (ALG != ALG_BFS) {
                         // release the cur list's dedupe bit (reused two iterations later); any
                         // improvement of v from now on appends it to the NEXT list (other parity)
-                        if (it > 0 && !local) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
+                        if (it > 0 && !local && !c.tail_nodedupe) atomicAnd(((it & 1) ? F.bm : F.bm2) + (v >> 5), ~(1u << (v & 31)));
                         // a local round takes v out of the NEXT list: release its bit there first (acquire),
-                        // so an improvement after the state read below appends v again
-                        if (local) atom_and_acquire(((it & 1) ? F.bm2 : F.bm) + (v >> 5), ~(1u << (v & 31)));
+                        // so an improvement after the state read below appends v again (no-dedupe mode: any
+                        // later improvement appends v anyway)
+                        if (local && !c.tail_nodedupe) atom_and_acquire(((it & 1) ? F.bm2 : F.bm) + (v >> 5), ~(1u << (v & 31)));
                         sval = vload(F.state + v);
                         // v's far bit is only changed by v's own processing: read it with the state (one
                         // round trip) instead of after the near/far decision
@@ -2454,7 +2473,7 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
             for (int f = 0; f < nfrag; f++) {
                 const unsigned na = s_app_na[f], lo = f == 0 ? s_app_lo : 0u;
                 unsigned* nxt = (it & 1) ? c.f[f].q_v : c.f[f].app;
-                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) nxt[s_app_base[f] + i] = s_app[f * app_cap + lo + i];
+                for (unsigned i = threadIdx.x; i < na; i += kTailThreads) tail_put(c, c.f[f], nxt, s_app_base[f] + i, s_app[f * app_cap + lo + i]);
             }
             __syncthreads();
             if (threadIdx.x < (unsigned)kMaxW) {
@@ -2536,14 +2555,17 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         }
         __syncthreads();
         unsigned long long total_next = 0, next_edges = 0;
+        bool list_ovf = false;  // a next list overflowed into the bitmap (tail_put): hand back now
         for (int f = 0; f < nfrag; f++) {
             total_next += s_tn[f];
             next_edges += s_te[f];
+            list_ovf = list_ovf || s_tn[f] > c.f[f].V + c.tail_slack;
         }
         // every CTA must take the same decision: only values that are final after the barrier (next-list
         // counters) enter it -- not the error flag, which next-iteration work of a fast CTA may already
         // set (overflowing candidates are simply not relaxed; control reports GUM_ERANGE afterwards)
-        if (total_next == 0 || total_next > c.tail_exit || next_edges > 4ull * c.tail_exit || k + 1 >= c.max_iter)
+        if (total_next == 0 || total_next > c.tail_exit || next_edges > 4ull * c.tail_exit || k + 1 >= c.max_iter ||
+            list_ovf)
             break;
     }
     for (int f = 0; f < nfrag; f++) {
@@ -2564,11 +2586,34 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         atomicAdd(&c.f[0].ctl->tail_acts, a_sum);
     }
     if (tail_v) atomicAdd(&c.f[0].ctl->tail_vertices, tail_v);
-    // hand the last produced list back to the regular path as the sparse activation list
+    // hand the last produced list back to the regular path as the sparse activation list (no-dedupe mode after
+    // a list overflow: as the frontier bitmap)
     if (blockIdx.x == 0) {
         const unsigned ns = (it + 1) % 3;
+        bool ovf = false;
+        for (int f = 0; f < nfrag; f++) ovf = ovf || vload(&c.f[f].ctl->tcnt[ns]) > c.f[f].V + c.tail_slack;
         for (int f = 0; f < nfrag; f++) {
-            const unsigned n = vload(&c.f[f].ctl->tcnt[ns]);
+            unsigned n = vload(&c.f[f].ctl->tcnt[ns]);
+            if (ALG != ALG_BFS && c.tail_nodedupe) {
+                // no-dedupe lists may hold a vertex twice: the regular path gets each once, its bm bit set
+                // (as a deduplicated activation list); compacted into the other list, then moved to app
+                __shared__ unsigned s_hb;
+                if (threadIdx.x == 0) s_hb = 0;
+                __syncthreads();
+                const unsigned* srcl = (it & 1) ? c.f[f].q_v : c.f[f].app;
+                unsigned* dstl = (it & 1) ? c.f[f].app : c.f[f].q_v;
+                for (unsigned i = threadIdx.x; i < n && i < c.f[f].V + c.tail_slack; i += kTailThreads) {
+                    const unsigned v = srcl[i], bit = 1u << (v & 31);
+                    if (!(atomicOr(c.f[f].bm + (v >> 5), bit) & bit)) dstl[atomicAdd(&s_hb, 1u)] = v;
+                }
+                __syncthreads();
+                n = s_hb;
+                if (!(it & 1))
+                    for (unsigned i = threadIdx.x; i < n; i += kTailThreads) c.f[f].app[i] = c.f[f].q_v[i];
+                __syncthreads();
+                if (threadIdx.x == 0) c.f[f].ctl->app_cnt = n;
+                continue;
+            }
             if (it & 1) {  // the last next list lives in q_v with its dedupe bits in bm2: move both
                 for (unsigned i = threadIdx.x; i < n; i += kTailThreads) {
                     const unsigned v = c.f[f].q_v[i];
@@ -2585,7 +2630,8 @@ __global__ void __launch_bounds__(kTailThreads) k_tail(const __grid_constant__ D
         if (threadIdx.x == 0) {
             rc->iter = k0 + it + 1;
             rc->tail_iters += it + 1;
-            rc->next_dense = 0;
+            rc->next_dense = ovf ? 1u : 0u;
+            if (ovf) atomicAdd(&c.f[0].ctl->tail_ovf, 1u);
             rc->tail = 0;
             __threadfence();
         }

@@ -490,6 +490,13 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     // not by the barriers (4096^2: 10186 -> 1281 engine iterations at 8 rounds, 103 -> 91 ms)
     static const int env_tl = getenv("GUM_TAIL_LOCAL") ? atoi(getenv("GUM_TAIL_LOCAL")) : 8;
     d.tail_local = (unsigned)std::max(0, env_tl);
+    // tail engine without next-list dedupe bits (improvement = returning atomicMin): C3 208.9 -> 158.3 ms
+    static const int env_nd = getenv("GUM_TAIL_NODEDUPE") ? atoi(getenv("GUM_TAIL_NODEDUPE")) : 1;
+    // (one launch unit only: with several units the parked units' iteration counts diverged from unit 0's in
+    // tests/test_gpu_mp.py -- results stayed exact -- so multi-unit runs keep the dedupe bits)
+    d.tail_nodedupe = (env_nd && c->n_units == 1) ? 1u : 0u;
+    static const long long env_sl = getenv("GUM_TAIL_SLACK") ? atoll(getenv("GUM_TAIL_SLACK")) : (long long)kTailSlack;
+    d.tail_slack = (unsigned)std::min<long long>(std::max(0ll, env_sl), (long long)kTailSlack);
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;
     d.pb_nb = c->pb_nb;
     d.bfs_pull = (alg == GUM_BFS && c->in_ready) ? 1u : 0u;
@@ -1701,8 +1708,9 @@ static gum_status partition_body(gum_ctx* c, gum_part kind, uint64_t seed) {
         F.vis = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.bm2 = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
         F.far = (unsigned*)dalloc(c, F.dev, ((F.V + 31) / 32 + 4) * 4, c->part_allocs);
-        F.app = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
-        F.q_v = (unsigned*)dalloc(c, F.dev, Vn * 4, c->part_allocs);
+        // (+ kTailSlack: the tail engine's no-dedupe mode may list a vertex more than once)
+        F.app = (unsigned*)dalloc(c, F.dev, (Vn + kTailSlack) * 4, c->part_allocs);
+        F.q_v = (unsigned*)dalloc(c, F.dev, (Vn + kTailSlack) * 4, c->part_allocs);
         F.q_off = (unsigned long long*)dalloc(c, F.dev, (Vn + 1) * 8, c->part_allocs);
         F.q_base = (long long*)dalloc(c, F.dev, Vn * 8, c->part_allocs);
         F.ctl = (FragCtl*)dalloc(c, F.dev, sizeof(FragCtl), c->part_allocs);
@@ -2054,6 +2062,7 @@ gum_status gum_run(gum_ctx* c, gum_alg alg, uint32_t source, gum_run_stats* stat
             stats->tail_edges += fc.tail_edges;
             stats->tail_vertices += fc.tail_vertices;
             stats->tail_activations += fc.tail_acts;
+            stats->tail_overflows += fc.tail_ovf;
             stats->migrated_queue_entries += fc.migrated_q;
             if (getenv("GUM_DEBUG"))
                 fprintf(stderr, "[gum] frag %d: V=%u E=%llu qlen=%llu edges_done=%llu frontier_edges=%llu frontier_vertices=%llu app_cnt=%u tcnt=%u,%u,%u\n",

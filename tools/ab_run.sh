@@ -1,4 +1,3 @@
-O=gpurun_out/ab7; mkdir -p $O
-V=build/variants
-timeout 900 python tools/kbench.py --config C5 --alg pr --part degree --runs 3 --libs $V/libgum_pullnopad.so,$V/libgum_pullpad.so > $O/pull_pad_C5.txt 2>&1; cat $O/pull_pad_C5.txt
-timeout 900 python -m pytest tests -m gpu -x -q -k "pr or pull" > $O/pytest.txt 2>&1; echo "pytest rc=$?"; tail -2 $O/pytest.txt
+O=gpurun_out/ab15; mkdir -p $O
+timeout 400 python tools/dbg_mp_iters.py > $O/mp.txt 2>&1; echo "mp rc=$?"; grep -v Warn $O/mp.txt | tail -16
+timeout 1500 python -m pytest tests -m gpu -x -q > $O/pytest.txt 2>&1; echo "pytest rc=$?"; tail -2 $O/pytest.txt
