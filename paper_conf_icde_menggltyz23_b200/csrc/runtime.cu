@@ -488,7 +488,8 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     // local relaxation rounds per CTA before each grid barrier of the tail engine (SSSP/WCC, one fragment):
     // C3 8192^2 grid 252 -> 241 ms at 6 rounds; the tail is bound by the per-hop chain of dependent loads,
     // not by the barriers (4096^2: 10186 -> 1281 engine iterations at 8 rounds, 103 -> 91 ms)
-    static const int env_tl = getenv("GUM_TAIL_LOCAL") ? atoi(getenv("GUM_TAIL_LOCAL")) : 8;
+    // (32 rounds with the no-dedupe engine: C3 157.2 -> 153.6 ms at threshold 32768; ab_c3_tail_sweep.txt)
+    static const int env_tl = getenv("GUM_TAIL_LOCAL") ? atoi(getenv("GUM_TAIL_LOCAL")) : 32;
     d.tail_local = (unsigned)std::max(0, env_tl);
     // tail engine without next-list dedupe bits (improvement = returning atomicMin): C3 208.9 -> 158.3 ms
     static const int env_nd = getenv("GUM_TAIL_NODEDUPE") ? atoi(getenv("GUM_TAIL_NODEDUPE")) : 1;

@@ -13,7 +13,11 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
         "lts__t_requests_srcunit_tex_op_red.sum", "lts__t_requests_srcunit_tex_op_atom.sum",
         "sm__cycles_elapsed.avg.per_second"]
-raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+import os
+
+# NCU_IMPORT_ARGS: extra import filters, e.g. "--launch-skip 7 --launch-count 1" (one kernel of a multi-kernel report)
+FILT = os.environ.get("NCU_IMPORT_ARGS", "").split()
+raw = subprocess.run(["ncu", "-i", rep] + FILT + ["--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(raw)))
 h, units = rows[0], rows[1]
 for r in rows[2:]:
@@ -22,7 +26,7 @@ for r in rows[2:]:
         if k in h:
             i = h.index(k)
             print(f"  {k:62s} {r[i]:>18s} {units[i]}")
-src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=sass"], capture_output=True,
+src = subprocess.run(["ncu", "-i", rep] + FILT + ["--page", "source", "--csv", "--print-source=sass"], capture_output=True,
                      text=True).stdout
 rows = list(csv.reader(io.StringIO(src)))
 col = "Warp Stall Sampling (All Samples)"
