@@ -11,4 +11,4 @@ timeout 900 python tools/ablation.py --osteal --grid 2048 --workers 8 --delta 10
 timeout 900 python tools/ablation.py --osteal --grid 2048 --workers 8 --delta 1024 --split --out $O/abl_osteal_split.json > $O/abl_osteal_split.txt 2>&1; cat $O/abl_osteal_split.txt
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_C3_sssp.csv \
   python tools/profile_run.py --config C3 --alg sssp --runs 1 > $O/launches_C3.log 2>&1; python tools/launches.py $O/launches_C3_sssp.csv > $O/launches_C3_sssp_summary.txt; head -8 $O/launches_C3_sssp_summary.txt
-bash tools/ncu_longest.sh $O/ncu_tail k_tail 150 40 --config C3 --alg sssp --runs 1
+bash tools/ncu_longest.sh $O/ncu_tail k_tail 150 20 --config C3 --alg sssp --runs 1; rm -f $O/ncu_tail/*.ncu-rep

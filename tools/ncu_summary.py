@@ -42,7 +42,8 @@ def num(x):
 
 if hi is not None:
     h = rows[hi]
-    data = [r for r in rows[hi + 1:] if len(r) == len(h) and col not in r]
+    nxt = next((i for i in range(hi + 1, len(rows)) if col in rows[i]), len(rows))  # (first kernel only)
+    data = [r for r in rows[hi + 1:nxt] if len(r) == len(h) and col not in r]
     ix = {n: i for i, n in enumerate(h)}
     tot = sum(num(r[ix[col]]) for r in data) or 1
     stalls = [n for n in h if n.startswith("stall_") and "Not Issued" not in n]
