@@ -449,8 +449,8 @@ def main():
         args.part = "degree" if alg in ("bfs", "pr") else "seg"
     if args.tail is None:
         # C3: a larger tail-engine threshold keeps more of the grid's near-far wavefront in the engine
-        # (profiles/round2/ab_c3_tail_sweep.txt: 157.3 -> 153.6 ms with 32 local rounds)
-        args.tail = 0 if (alg == "bfs" and args.config in ("C1", "C2")) else (32768 if args.config == "C3" else 16384)
+        # (profiles/round2/ab_c3_tail_sweep.txt: 157.3 -> 148.9 ms at 65536 with 32 local rounds)
+        args.tail = 0 if (alg == "bfs" and args.config in ("C1", "C2")) else (65536 if args.config == "C3" else 16384)
     rank = env_int("RANK", 0)
     world = env_int("WORLD_SIZE", 1)
     N = args.gpus

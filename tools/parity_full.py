@@ -29,7 +29,7 @@ import oracle  # noqa: E402
 
 
 def ctx_kwargs(config, alg):
-    tail = 0 if (alg == "bfs" and config in ("C1", "C2")) else (32768 if config == "C3" else 16384)  # = bench.py
+    tail = 0 if (alg == "bfs" and config in ("C1", "C2")) else (65536 if config == "C3" else 16384)  # = bench.py
     return dict(fsteal=True, osteal=True, sssp_delta=4096 if config == "C3" else 0, tail_vertices=tail)
 
 

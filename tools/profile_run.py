@@ -38,7 +38,7 @@ else:
 rp, col, w = gum.build_csr(g.num_vertices, g.src, g.dst, g.w if a.alg == "sssp" else None)
 delta = a.delta if a.delta is not None else (4096 if a.config == "C3" and a.alg == "sssp" else 0)
 tail = a.tail if a.tail is not None else (0 if a.alg == "bfs" and a.config in ("C1", "C2") and not (a.rmat or a.grid)
-                                          else (32768 if a.config == "C3" and not (a.rmat or a.grid) else 16384))
+                                          else (65536 if a.config == "C3" and not (a.rmat or a.grid) else 16384))
 with gum.Context(num_gpus=a.gpus, host_loop=bool(a.host_loop), profile=bool(a.host_loop), sssp_delta=delta,
                  osteal_threshold=a.osteal_threshold, tail_vertices=tail) as ctx:
     ctx.load_csr(rp, col, w)
