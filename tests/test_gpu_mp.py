@@ -42,7 +42,9 @@ def case_parity(rank, world, scale, part, kw):
             else:
                 ok = bool(np.array_equal(res, ref))
             out[alg] = dict(ok=ok, conserved=st.edges_expanded == st.edges_frontier, iters=st.iterations,
-                            stolen=st.edges_stolen, owners=st.final_owners, remote=st.remote_updates)
+                            stolen=st.edges_stolen, owners=st.final_owners, remote=st.remote_updates,
+                            tail_iters=st.tail_iterations, bodies=st.bodies, osteal_iter=st.osteal_iteration,
+                            barriers=list(st.unit_barriers)[:world], last=list(st.unit_last_iter)[:world])
     return out
 
 
