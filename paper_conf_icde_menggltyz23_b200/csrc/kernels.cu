@@ -1171,6 +1171,9 @@ __device__ __noinline__ void control_body(const DevCtx& c, const int alg, int w0
             if (m != 1) rc->osteal_iter = k;
             m = 1;
             rc->m = 1;
+            // the engine runs on unit 0 alone: a give-back decided above must not wake parked units now (they
+            // would rejoin as members while the engine advances unit 0's iteration count without them)
+            grow_to = 0;
             rc->steal_ok = 0;
             rc->pb = 0;
             rc->pull = 0;

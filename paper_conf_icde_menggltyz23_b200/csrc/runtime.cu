@@ -493,9 +493,7 @@ DevCtx make_devctx(const gum_ctx* c, int alg) {
     d.tail_local = (unsigned)std::max(0, env_tl);
     // tail engine without next-list dedupe bits (improvement = returning atomicMin): C3 208.9 -> 158.3 ms
     static const int env_nd = getenv("GUM_TAIL_NODEDUPE") ? atoi(getenv("GUM_TAIL_NODEDUPE")) : 1;
-    // (one launch unit only: with several units the parked units' iteration counts diverged from unit 0's in
-    // tests/test_gpu_mp.py -- results stayed exact -- so multi-unit runs keep the dedupe bits)
-    d.tail_nodedupe = ((env_nd && c->n_units == 1) || env_nd == 2) ? 1u : 0u;  // (2: every unit count; debugging)
+    d.tail_nodedupe = env_nd ? 1u : 0u;
     static const long long env_sl = getenv("GUM_TAIL_SLACK") ? atoll(getenv("GUM_TAIL_SLACK")) : (long long)kTailSlack;
     d.tail_slack = (unsigned)std::min<long long>(std::max(0ll, env_sl), (long long)kTailSlack);
     d.pb_shift = (alg == GUM_BFS && c->pb_ready) ? c->pb_shift : 0u;

@@ -1,5 +1,4 @@
-O=gpurun_out/ab17; mkdir -p $O
-for tv in 32768 65536 131072; do
-timeout 900 python tools/kbench.py --config C3 --alg sssp --part seg --runs 2 --kw "{\"tail_vertices\":$tv,\"sssp_delta\":4096}" > $O/C3_tv${tv}.txt 2>&1; echo "C3 tv=$tv $(cut -c1-200 $O/C3_tv${tv}.txt)"
-done
-timeout 900 python tools/kbench.py --config C4 --alg wcc --part seg --runs 3 --kw '{"tail_vertices":16384}' > $O/C4.txt 2>&1; echo "C4 $(cut -c1-200 $O/C4.txt)"
+O=gpurun_out/ab20; mkdir -p $O
+( time timeout 1800 python -m pytest tests -m gpu -q ) > $O/pytest.txt 2>&1; echo "pytest rc=$?"; grep passed $O/pytest.txt | tail -1
+timeout 900 python tools/ablation.py --osteal --grid 2048 --workers 8 --delta 1024 --split --out $O/abl_osteal_split.json > $O/abl_osteal_split.txt 2>&1; cat $O/abl_osteal_split.txt
+timeout 400 python tools/dbg_mp_iters.py > $O/mp.txt 2>&1; grep -v Warn $O/mp.txt | tail -8
